@@ -1,0 +1,207 @@
+/*
+ * mbir.h -- C-ABI of libmbir: a B200-native (sm_100a) implementation of the GPU-ICD hot path
+ * of Sabne et al., "Model-based Iterative CT Image Reconstruction on GPUs", PPoPP'17.
+ *
+ * Citations: "P:n" = line n of the paper text; "Alg k:i" = line i
+ * of Algorithm k.  DESIGN.md lists every reading of a passage the paper leaves open (R1...).
+ *
+ * What the library computes: model-based iterative reconstruction by SuperVoxel ICD.
+ *   minimise  f(x) = 1/2 (y - A x)^T W (y - A x) + sum_{j~r} b_jr rho(x_j - x_r),  x >= 0
+ * (Eq. 1 at P:351 plus the prior of reading R1) by Alg. 1 single-voxel updates
+ * run with the three levels of parallelism of P:155-161: within a voxel (threads over the
+ * voxel's views), within a SuperVoxel (sequential-exact, pipelined across warps), and across
+ * SuperVoxels of one checkerboard colour and across slices.
+ *
+ * Conventions shared by every call:
+ *   - All functions are extern "C", never throw, and return 0 (MBIR_OK) or a negative code.
+ *     mbir_last_error(h) gives a human-readable message for the last failure on h.
+ *   - Image layout [nz_local][ny][nx] float32, x fastest, units mm^-1.
+ *   - Sinogram layout [nz_local][nviews][nchannels] float32, channel fastest (one sinogram
+ *     column per view angle).
+ *   - `where` = MBIR_HOST (pageable or pinned host memory) or MBIR_DEVICE (a device pointer on
+ *     the handle's device, e.g. a torch CUDA tensor's data_ptr()).  All calls COPY; the caller
+ *     keeps ownership of every buffer it passes.  Device-side work is ordered on the handle's
+ *     stream; calls return after that stream has been synchronised unless stated otherwise.
+ *   - The library owns all of its device memory (allocated in mbir_create / set_sinogram and
+ *     released by mbir_destroy).
+ */
+#ifndef MBIR_H
+#define MBIR_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MBIR_OK 0
+#define MBIR_EINVAL (-1)   /* bad argument / unsupported size */
+#define MBIR_ENOMEM (-2)   /* device or host allocation failed */
+#define MBIR_ECUDA (-3)    /* CUDA runtime error (message in mbir_last_error) */
+#define MBIR_ESTATE (-4)   /* call out of order (e.g. reconstruct before set_sinogram) */
+#define MBIR_ENUMERIC (-5) /* NaN/Inf detected in the state */
+#define MBIR_ENCCL (-6)    /* NCCL error (multi-GPU) */
+#define MBIR_ENOTSUP (-7)  /* feature not built in */
+
+#define MBIR_HOST 0
+#define MBIR_DEVICE 1
+
+typedef struct mbir_handle mbir_handle;
+
+/* Parallel-beam scanner + image grid (readings R4, R5).
+ * Pixel centres ((ix-(nx-1)/2)*dxy, (iy-(ny-1)/2)*dxy); slices have pitch dxy.
+ * View k has angle angles[k] (host array of nviews doubles, copied) or k*pi/nviews if NULL.
+ * Channel i covers [t0 + i*dchannel, t0 + (i+1)*dchannel), t0 = -nchannels*dchannel/2 +
+ * center_offset*dchannel.  nz_local slices starting at global slice z_offset of nz_total
+ * (z-slab partition across ranks). */
+typedef struct mbir_geometry {
+    int nx, ny;
+    int nz_local, z_offset, nz_total;
+    double dxy;
+    int nviews, nchannels;
+    double dchannel;
+    double center_offset;
+    const double* angles;
+} mbir_geometry;
+
+/* q-GGMRF prior (reading R1): rho(D) = |D|^p/(p sigma^p) * u/(1+u), u = |D/(T sigma)|^(q-p).
+ * Requirements: 1 <= p <= 2, q == 2, T > 0, sigma > 0.  neighborhood = 8 (in-slice) or 26
+ * (3-D, slices of pitch dxy); weights b_jr ~ 1/distance summing to 1 (reading R2), free boundary.
+ * positivity != 0 clips every update at 0 (reading R3). */
+typedef struct mbir_prior {
+    double p, q, T, sigma;
+    int neighborhood;
+    int positivity;
+} mbir_prior;
+
+/* Algorithmic options (Table 1).  Zero-initialise and
+ * call mbir_default_options() for the defaults. */
+typedef struct mbir_options {
+    int sv_side;           /* SuperVoxel side s; tiles of s x s voxels, default 9   */
+    double sv_fraction;    /* fraction of SVs per iteration >= 2, default 0.25  */
+    int batch_svs;         /* BATCH_SIZE: SVs per slice per launch (Alg3:25); 0 = a whole
+                              checkerboard colour group per launch (no threshold), default 0   */
+    int batch_threshold;   /* Alg3:26-27: drop a group's remainder smaller than this; -1 =
+                              batch_svs/4; ignored when batch_svs == 0                   */
+    int zero_skip;         /* P:115, default 1 (never in iteration 1; reading R9)               */
+    int quantize_A;        /* 1: A as uint8 codes + per-voxel scale, 0: fp32 values */
+    uint64_t seed;         /* voxel-order / random-SV-selection seed                            */
+    int deterministic;     /* debug: every iteration visits all SVs, one SV per launch, in
+                              (z-parity, colour, slice, SV index) order, voxels in raster order  */
+} mbir_options;
+
+/* Placement and (optional) multi-GPU slab partition.  device: CUDA ordinal.  stream: a
+ * cudaStream_t (NULL = the library creates its own).  For nranks > 1, nccl_unique_id points to
+ * the 128-byte ncclUniqueId produced by mbir_nccl_unique_id() on rank 0 and broadcast by the
+ * caller (e.g. over a torch.distributed process group); rank r must own slices
+ * [z_offset, z_offset + nz_local) with slabs contiguous in rank order. */
+typedef struct mbir_dist {
+    int device;
+    void* stream;
+    int rank, nranks;
+    const void* nccl_unique_id;
+} mbir_dist;
+
+/* Per-call statistics (P:277 equit accounting; Table 1). */
+typedef struct mbir_stats {
+    int64_t updates;       /* executed (non-skipped) voxel updates, all ranks        */
+    int64_t skipped;       /* zero-skipped voxel visits                               */
+    int64_t sv_visits;     /* (SV, slice) tasks executed                              */
+    int64_t iterations;    /* outer iterations (Alg3:16) executed by this call       */
+    double equits;         /* updates / (nx*ny*nz_total)                              */
+    double seconds;        /* device time of this call (CUDA events)                  */
+    double sum_abs_delta;  /* sum |delta| over the executed updates                   */
+    int64_t launches;      /* kernel launches issued by this call                     */
+} mbir_stats;
+
+/* Sizes of the internal layout (for tests, benchmarks and buffer allocation). */
+typedef struct mbir_sizes {
+    int nsv_x, nsv_y, nsv;          /* SuperVoxel tiles per slice                         */
+    int K;                          /* max channels per (voxel, view): 4                  */
+    int band_max;                   /* max SV band width over (SV, view), channels        */
+    int svb_rows;                   /* rows of the shared-memory SV buffer (>= band_max)  */
+    int threads_per_cta;            /* update-kernel block size                            */
+    int smem_bytes;                 /* update-kernel dynamic shared memory                 */
+    int64_t nnz;                    /* total non-zeros of the slice-plane system matrix    */
+    int64_t a_bytes;                /* device bytes of the compressed A                   */
+    int64_t band_entries;           /* sum over (SV, view) of band widths                  */
+} mbir_sizes;
+
+/* Fill defaults: sv_side 9, sv_fraction 0.25, batch_svs 0, batch_threshold -1, zero_skip 1,
+ * quantize_A 1, seed 3000, deterministic 0. */
+void mbir_default_options(mbir_options* o);
+/* p 1.2, q 2, T 1, sigma 0.005, neighborhood 26, positivity 1. */
+void mbir_default_prior(mbir_prior* p);
+
+/* Build a reconstruction context: validates arguments (MBIR_EINVAL), computes the system
+ * matrix on the device in double precision (strip-area model, reading R4) and compresses it
+ * per SuperVoxel (per-view band offsets + uint8 codes or fp32 values),
+ * builds the SV tiling and scheduler state, and (nranks > 1) joins the NCCL communicator.
+ * *out is set only on success.  Errors: EINVAL, ENOMEM, ECUDA, ENCCL. */
+int mbir_create(const mbir_geometry* g, const mbir_prior* p, const mbir_options* o,
+                const mbir_dist* d, mbir_handle** out);
+
+/* Load the measured sinogram y and its weights w (inverse noise variance), both
+ * [nz_local][nviews][nchannels].  Resets the error sinogram e = y - A x for the current image
+ * (Alg. 1 input) and the scheduler state.  Errors: EINVAL (NULL, NaN/Inf or negative w),
+ * ECUDA. */
+int mbir_set_sinogram(mbir_handle* h, const float* y, const float* w, int where);
+
+/* Set the image (warm start / resume; default 0).  x0 == NULL sets 0.  Recomputes e = y - A x
+ * if a sinogram is loaded.  Errors: EINVAL (negative values with positivity), ECUDA. */
+int mbir_set_image(mbir_handle* h, const float* x0, int where);
+
+/* Run whole iterations of GPU-ICD (Alg. 3 lines 16-31) until at least `equits` equits of
+ * executed updates have been done by this call (one equit = nx*ny*nz_total updates).
+ * Collective across ranks.  st may be NULL.  Errors: ESTATE (no sinogram), ENUMERIC, ECUDA,
+ * ENCCL. */
+int mbir_reconstruct(mbir_handle* h, double equits, mbir_stats* st);
+
+/* Run exactly n_iterations iterations (for convergence curves).  Same errors. */
+int mbir_iterate(mbir_handle* h, int n_iterations, mbir_stats* st);
+
+/* Copy the current image [nz_local][ny][nx] into x.  Errors: EINVAL, ECUDA. */
+int mbir_get_image(mbir_handle* h, float* x, int where);
+
+/* Copy the current error sinogram e [nz_local][nviews][nchannels] (test hook). */
+int mbir_get_error_sinogram(mbir_handle* h, float* e, int where);
+
+/* RMSE in Hounsfield units of the current image against `golden` ([nz_local][ny][nx],
+ * device or host), 1000*sqrt(mean((x-g)^2))/mu_water (reading R12), reduced over all
+ * ranks.  Device reduction. */
+int mbir_rmse_hu(mbir_handle* h, const float* golden, int where, double mu_water, double* out);
+
+int mbir_query_sizes(const mbir_handle* h, mbir_sizes* s);
+
+/* Export the slice-plane system matrix in the plain layout (test hook, host buffers, each may
+ * be NULL): first/count int32 [ny*nx][nviews] (first channel, number of channels), values
+ * float32 [ny*nx][nviews][K] (fp32 of the double-precision strip areas / dchannel; unused
+ * slots 0), codes uint8 [ny*nx][nviews][K] (P:267 codec), scales float32 [ny*nx]
+ * (max_j(A)/255). */
+int mbir_get_sysmatrix(mbir_handle* h, int32_t* first, int32_t* count, float* values,
+                       uint8_t* codes, float* scales);
+
+/* Same for n selected in-slice voxels (flat iy*nx + ix): row i of each output describes
+ * voxels[i] (test hook for full-size geometries). */
+int mbir_get_sysmatrix_columns(mbir_handle* h, const int64_t* voxels, int n, int32_t* first,
+                               int32_t* count, float* values, uint8_t* codes, float* scales);
+
+/* Alg. 1 steps 1-7 for n voxels at the CURRENT state, without applying them (test hook):
+ * voxels are flat local indices (z*ny + y)*nx + x; theta1/theta2/delta are host arrays of n
+ * floats, computed on the device from the library's A representation, e, w and x. */
+int mbir_probe_update(mbir_handle* h, const int64_t* voxels, int n, float* theta1,
+                      float* theta2, float* delta);
+
+/* Multi-GPU bootstrap: write a fresh 128-byte ncclUniqueId into id (call on rank 0 only).
+ * Returns ENOTSUP if the library was built without NCCL. */
+int mbir_nccl_unique_id(void* id128);
+
+void mbir_destroy(mbir_handle* h);
+const char* mbir_strerror(int code);
+const char* mbir_last_error(const mbir_handle* h);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MBIR_H */

@@ -1,0 +1,822 @@
+// libmbir C-ABI (include/mbir.h): handle lifecycle, host orchestration of Alg. 3,
+// the z-slab multi-GPU halo exchange over NCCL, and the test hooks.
+//
+// Host loop per iteration (Alg3:16-31):
+//   select (device: all / top 25 % / random 25 %, 4 checkerboard colours per slice)
+//   for z-parity half (3-D prior only): for colour 0..3: for batch: fused update kernel
+//   [multi-GPU] after each half: NCCL send/recv of the updated boundary slices (halo)
+//   counters -> equits, all-reduced across ranks
+#include <dlfcn.h>
+#include <math.h>
+#include <nccl.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "mbir_internal.h"
+
+using namespace mbir;
+
+namespace {
+
+// ---- NCCL through dlopen (only needed when nranks > 1) ----
+struct NcclApi {
+    bool ok = false;
+    ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                              cudaStream_t) = nullptr;
+    ncclResult_t (*GroupStart)() = nullptr;
+    ncclResult_t (*GroupEnd)() = nullptr;
+    const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+NcclApi& nccl()
+{
+    static NcclApi api;
+    static bool tried = false;
+    if (tried) return api;
+    tried = true;
+    void* lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!lib) lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!lib) lib = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!lib) return api;
+#define LOADSYM(f) api.f = (decltype(api.f))dlsym(lib, "nccl" #f)
+    LOADSYM(GetUniqueId);
+    LOADSYM(CommInitRank);
+    LOADSYM(CommDestroy);
+    LOADSYM(Send);
+    LOADSYM(Recv);
+    LOADSYM(AllReduce);
+    LOADSYM(GroupStart);
+    LOADSYM(GroupEnd);
+    LOADSYM(GetErrorString);
+#undef LOADSYM
+    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.Send && api.Recv &&
+             api.AllReduce && api.GroupStart && api.GroupEnd;
+    return api;
+}
+
+}  // namespace
+
+struct mbir_handle {
+    mbir_geometry g{};
+    std::vector<double> angles;
+    mbir_prior pr{};
+    mbir_options o{};
+    int device = 0;
+    cudaStream_t st = nullptr;
+    bool own_stream = false;
+    int rank = 0, nranks = 1;
+    ncclComm_t comm = nullptr;
+    int side = 0, nsvx = 0, nsvy = 0, nsv = 0, S2 = 0, nsv_pad = 0;
+    int rows = 0, band_max = 0;
+    int vpt = 1, nvw = 0, Vs = 0, threads = 0, smem = 0, blocks_per_sm = 1, nsm = 148;
+    int max_group = 0;
+    DevA A{};
+    double* d_cs = nullptr;
+    float *d_y = nullptr, *d_w = nullptr, *d_e = nullptr, *d_x = nullptr;
+    float *d_theta2 = nullptr, *d_amount = nullptr, *d_scratch = nullptr;
+    int *d_task_list = nullptr, *d_task_count = nullptr;
+    unsigned long long* d_counters = nullptr;  // [updates, skipped, visits]
+    double* d_sum_delta = nullptr;
+    int* d_flag = nullptr;
+    double* d_acc = nullptr;
+    unsigned long long* h_counters = nullptr;  // pinned [4] (3 counters + sum_delta bits)
+    bool have_sino = false;
+    int iter = 0;
+    int64_t nnz = 0, a_bytes = 0, band_entries = 0;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    std::string err;
+};
+
+namespace {
+
+int fail(mbir_handle* h, int code, const std::string& msg)
+{
+    if (h) h->err = msg;
+    return code;
+}
+
+#define CK(call)                                                                             \
+    do {                                                                                     \
+        cudaError_t e_ = (call);                                                             \
+        if (e_ != cudaSuccess)                                                               \
+            return fail(h, e_ == cudaErrorMemoryAllocation ? MBIR_ENOMEM : MBIR_ECUDA,       \
+                        std::string(#call) + ": " + cudaGetErrorString(e_));                 \
+    } while (0)
+
+#define CKN(call)                                                                            \
+    do {                                                                                     \
+        ncclResult_t r_ = (call);                                                            \
+        if (r_ != ncclSuccess)                                                               \
+            return fail(h, MBIR_ENCCL, std::string(#call) + ": " +                           \
+                               (nccl().GetErrorString ? nccl().GetErrorString(r_) : "nccl error")); \
+    } while (0)
+
+IcdParams make_params(mbir_handle* h)
+{
+    IcdParams p{};
+    p.nx = h->g.nx;
+    p.ny = h->g.ny;
+    p.nz_local = h->g.nz_local;
+    p.z_offset = h->g.z_offset;
+    p.nz_total = h->g.nz_total;
+    p.V = h->g.nviews;
+    p.M = h->g.nchannels;
+    p.side = h->side;
+    p.nsvx = h->nsvx;
+    p.nsv = h->nsv;
+    p.S2 = h->S2;
+    p.Vs = h->Vs;
+    p.rows = h->rows;
+    p.nvw = h->nvw;
+    p.A = h->A;
+    p.e = h->d_e;
+    p.w = h->d_w;
+    p.x = h->d_x;
+    p.theta2 = h->d_theta2;
+    p.scratch = h->d_scratch;
+    p.sv_amount = h->d_amount;
+    p.task_list = h->d_task_list;
+    p.task_count = h->d_task_count;
+    p.max_group = h->max_group;
+    p.counters = h->d_counters;
+    p.sum_delta = h->d_sum_delta;
+    p.seed = h->o.seed;
+    p.iter = h->iter;
+    p.deterministic = h->o.deterministic;
+    return p;
+}
+
+size_t sino_elems(const mbir_handle* h)
+{
+    return (size_t)h->g.nz_local * h->g.nviews * h->g.nchannels;
+}
+size_t plane_elems(const mbir_handle* h) { return (size_t)h->g.nx * h->g.ny; }
+
+cudaMemcpyKind kind_in(int where) { return where == MBIR_DEVICE ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice; }
+cudaMemcpyKind kind_out(int where) { return where == MBIR_DEVICE ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost; }
+
+// halo exchange of the boundary slices whose global parity is `parity` (-1: both ends).
+int exchange_halo(mbir_handle* h, int parity)
+{
+    if (h->nranks <= 1) return MBIR_OK;
+    const size_t pl = plane_elems(h);
+    const int z0 = h->g.z_offset, z1 = h->g.z_offset + h->g.nz_local - 1;
+    NcclApi& N = nccl();
+    CKN(N.GroupStart());
+    // my first slice -> rank-1 (its top halo); my last slice -> rank+1 (its bottom halo)
+    if (h->rank > 0) {
+        if (parity < 0 || (z0 & 1) == parity) CKN(N.Send(h->d_x + 1 * pl, pl, ncclFloat, h->rank - 1, h->comm, h->st));
+        if (parity < 0 || ((z0 - 1) & 1) == parity) CKN(N.Recv(h->d_x, pl, ncclFloat, h->rank - 1, h->comm, h->st));
+    }
+    if (h->rank < h->nranks - 1) {
+        if (parity < 0 || (z1 & 1) == parity)
+            CKN(N.Send(h->d_x + (size_t)h->g.nz_local * pl, pl, ncclFloat, h->rank + 1, h->comm, h->st));
+        if (parity < 0 || ((z1 + 1) & 1) == parity)
+            CKN(N.Recv(h->d_x + (size_t)(h->g.nz_local + 1) * pl, pl, ncclFloat, h->rank + 1, h->comm, h->st));
+    }
+    CKN(N.GroupEnd());
+    return MBIR_OK;
+}
+
+// e = y - A x (and theta2 when the weights changed)
+int refresh_error(mbir_handle* h, bool theta2)
+{
+    IcdParams p = make_params(h);
+    const bool q = h->o.quantize_A != 0;
+    CK(launch_forward(p, q, h->d_y, h->st));
+    if (theta2) CK(launch_theta2(p, q, h->st));
+    return MBIR_OK;
+}
+
+int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats* st)
+{
+    if (!h->have_sino) return fail(h, MBIR_ESTATE, "mbir_set_sinogram has not been called");
+    const double nvox_total = (double)h->g.nx * h->g.ny * h->g.nz_total;
+    const bool q = h->o.quantize_A != 0;
+    const int nnb = h->pr.neighborhood;
+    const int parities = (nnb == 26 && h->g.nz_total > 1) ? 2 : 1;
+    const int target_ctas = h->nsm * h->blocks_per_sm;
+    int64_t updates = 0, skipped = 0, visits = 0, iters = 0, launches = 0;
+    double sum_delta = 0.0;
+    CK(cudaEventRecord(h->ev0, h->st));
+    for (int it = 0;; ++it) {
+        if (n_iter >= 0 && it >= n_iter) break;
+        if (n_iter < 0 && (double)updates >= target_equits * nvox_total) break;
+        h->iter += 1;
+        CK(cudaMemsetAsync(h->d_counters, 0, 3 * sizeof(unsigned long long), h->st));
+        CK(cudaMemsetAsync(h->d_sum_delta, 0, sizeof(double), h->st));
+        // ---- SV selection (Alg3:17-23)
+        SchedParams sp{};
+        sp.nz_local = h->g.nz_local;
+        sp.z_offset = h->g.z_offset;
+        sp.nsvx = h->nsvx;
+        sp.nsvy = h->nsvy;
+        sp.nsv = h->nsv;
+        sp.nsv_pad = h->nsv_pad;
+        sp.max_group = h->max_group;
+        sp.seed = h->o.seed;
+        sp.iter = h->iter;
+        sp.sv_amount = h->d_amount;
+        sp.task_list = h->d_task_list;
+        sp.task_count = h->d_task_count;
+        if (h->o.deterministic) {
+            sp.mode = 3;
+            sp.nsel = h->nsv;
+        } else if (h->iter == 1) {
+            sp.mode = 0;
+            sp.nsel = h->nsv;
+        } else {
+            sp.mode = (h->iter % 2 == 0) ? 1 : 2;
+            sp.nsel = std::min(h->nsv, std::max(1, (int)ceil(h->o.sv_fraction * h->nsv - 1e-9)));
+        }
+        CK(launch_select(sp, h->st));
+        ++launches;
+        IcdParams p = make_params(h);
+        p.zero_skip_active = (h->o.zero_skip && h->iter > 1) ? 1 : 0;
+        for (int zp = 0; zp < parities; ++zp) {
+            // local slices whose global index has parity zp (all slices if 2-D prior)
+            int zfirst = 0, zstride = 1;
+            if (parities == 2) {
+                zfirst = ((zp - h->g.z_offset) % 2 + 2) % 2;
+                zstride = 2;
+            }
+            const int nzp = zfirst < h->g.nz_local ? (h->g.nz_local - zfirst + zstride - 1) / zstride : 0;
+            for (int colour = 0; colour < 4 && nzp > 0; ++colour) {
+                p.colour = colour;
+                p.zstride = zstride;
+                if (h->o.deterministic) {  // one SV per launch, fully sequential order
+                    p.batch = 1;
+                    p.thr = 0;
+                    p.zstride = 1;
+                    for (int z = zfirst; z < h->g.nz_local; z += zstride) {
+                        p.zfirst = z;
+                        for (int pos = 0; pos < h->max_group; ++pos) {
+                            p.batch_base = pos;
+                            CK(launch_icd(p, h->vpt, nnb, q, 1, 1, h->st));
+                            ++launches;
+                        }
+                    }
+                    continue;
+                }
+                p.zfirst = zfirst;
+                const int B = h->o.batch_svs > 0 ? h->o.batch_svs : h->max_group;
+                p.batch = B;
+                p.thr = h->o.batch_svs > 0 ? (h->o.batch_threshold >= 0 ? h->o.batch_threshold : B / 4) : 0;
+                const int gx = std::max(1, std::min(B, (target_ctas + nzp - 1) / nzp));
+                for (int base = 0; base < h->max_group; base += B) {
+                    p.batch_base = base;
+                    CK(launch_icd(p, h->vpt, nnb, q, gx, nzp, h->st));
+                    ++launches;
+                }
+            }
+            if (h->nranks > 1 && parities == 2) {
+                int r = exchange_halo(h, (h->g.z_offset + zfirst) & 1);
+                if (r) return r;
+            }
+        }
+        if (h->nranks > 1) {
+            CKN(nccl().AllReduce(h->d_counters, h->d_counters, 3, ncclUint64, ncclSum, h->comm, h->st));
+            CKN(nccl().AllReduce(h->d_sum_delta, h->d_sum_delta, 1, ncclFloat64, ncclSum, h->comm, h->st));
+        }
+        CK(cudaMemcpyAsync(h->h_counters, h->d_counters, 3 * sizeof(unsigned long long),
+                           cudaMemcpyDeviceToHost, h->st));
+        CK(cudaMemcpyAsync(h->h_counters + 3, h->d_sum_delta, sizeof(double), cudaMemcpyDeviceToHost,
+                           h->st));
+        CK(cudaStreamSynchronize(h->st));
+        updates += (int64_t)h->h_counters[0];
+        skipped += (int64_t)h->h_counters[1];
+        visits += (int64_t)h->h_counters[2];
+        double sd;
+        memcpy(&sd, h->h_counters + 3, sizeof(double));
+        if (!isfinite(sd)) return fail(h, MBIR_ENUMERIC, "non-finite update amount");
+        sum_delta += sd;
+        ++iters;
+        if (n_iter < 0 && h->h_counters[0] == 0 && h->h_counters[2] > 0 && h->o.zero_skip) {
+            // everything zero-skipped: the image is all zero and stays so; stop
+            break;
+        }
+    }
+    CK(cudaEventRecord(h->ev1, h->st));
+    CK(cudaEventSynchronize(h->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, h->ev0, h->ev1));
+    if (st) {
+        st->updates = updates;
+        st->skipped = skipped;
+        st->sv_visits = visits;
+        st->iterations = iters;
+        st->equits = (double)updates / nvox_total;
+        st->seconds = ms * 1e-3;
+        st->sum_abs_delta = sum_delta;
+        st->launches = launches;
+    }
+    return MBIR_OK;
+}
+
+template <typename T>
+int dalloc(mbir_handle* h, T** p, size_t n)
+{
+    cudaError_t e = cudaMalloc((void**)p, std::max<size_t>(n, 1) * sizeof(T));
+    if (e != cudaSuccess) return fail(h, MBIR_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    return MBIR_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void mbir_default_options(mbir_options* o)
+{
+    if (!o) return;
+    memset(o, 0, sizeof(*o));
+    o->sv_side = 9;
+    o->sv_fraction = 0.25;
+    o->batch_svs = 0;
+    o->batch_threshold = -1;
+    o->zero_skip = 1;
+    o->quantize_A = 1;
+    o->seed = 3000;
+    o->deterministic = 0;
+}
+
+void mbir_default_prior(mbir_prior* p)
+{
+    if (!p) return;
+    p->p = 1.2;
+    p->q = 2.0;
+    p->T = 1.0;
+    p->sigma = 0.005;
+    p->neighborhood = 26;
+    p->positivity = 1;
+}
+
+const char* mbir_strerror(int code)
+{
+    switch (code) {
+    case MBIR_OK: return "ok";
+    case MBIR_EINVAL: return "invalid argument";
+    case MBIR_ENOMEM: return "out of memory";
+    case MBIR_ECUDA: return "CUDA error";
+    case MBIR_ESTATE: return "call out of order";
+    case MBIR_ENUMERIC: return "non-finite value";
+    case MBIR_ENCCL: return "NCCL error";
+    case MBIR_ENOTSUP: return "not supported";
+    default: return "unknown error";
+    }
+}
+
+const char* mbir_last_error(const mbir_handle* h) { return h ? h->err.c_str() : "null handle"; }
+
+int mbir_nccl_unique_id(void* id128)
+{
+    if (!id128) return MBIR_EINVAL;
+    NcclApi& N = nccl();
+    if (!N.ok) return MBIR_ENOTSUP;
+    ncclUniqueId id;
+    if (N.GetUniqueId(&id) != ncclSuccess) return MBIR_ENCCL;
+    memcpy(id128, &id, sizeof(id));
+    return MBIR_OK;
+}
+
+void mbir_destroy(mbir_handle* h)
+{
+    if (!h) return;
+    if (h->st) cudaStreamSynchronize(h->st);
+    void* ptrs[] = {h->A.codes, h->A.vals, h->A.off, h->A.count, h->A.scale, h->A.band_start,
+                    h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
+                    h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count, h->d_counters, h->d_sum_delta,
+                    h->d_flag, h->d_acc};
+    for (void* p : ptrs)
+        if (p) cudaFree(p);
+    if (h->h_counters) cudaFreeHost(h->h_counters);
+    if (h->ev0) cudaEventDestroy(h->ev0);
+    if (h->ev1) cudaEventDestroy(h->ev1);
+    if (h->comm && nccl().CommDestroy) nccl().CommDestroy(h->comm);
+    if (h->own_stream && h->st) cudaStreamDestroy(h->st);
+    delete h;
+}
+
+int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options* o,
+                const mbir_dist* d, mbir_handle** out)
+{
+    if (!out) return MBIR_EINVAL;
+    *out = nullptr;
+    if (!g) return MBIR_EINVAL;
+    mbir_handle* h = new (std::nothrow) mbir_handle();
+    if (!h) return MBIR_ENOMEM;
+    auto bail = [&](int code) {
+        mbir_destroy(h);
+        return code;
+    };
+    h->g = *g;
+    if (pr)
+        h->pr = *pr;
+    else
+        mbir_default_prior(&h->pr);
+    if (o)
+        h->o = *o;
+    else
+        mbir_default_options(&h->o);
+    if (d) {
+        h->device = d->device;
+        h->st = (cudaStream_t)d->stream;
+        h->rank = d->rank;
+        h->nranks = d->nranks < 1 ? 1 : d->nranks;
+    }
+    // ---- validation (MBIR_EINVAL)
+    const mbir_geometry& G = h->g;
+    if (G.nz_total <= 0) h->g.nz_total = G.nz_local;
+    if (G.nx < 1 || G.ny < 1 || G.nz_local < 1 || G.nviews < 1 || G.nchannels < 1 || !(G.dxy > 0) ||
+        !(G.dchannel > 0) || G.z_offset < 0 || G.z_offset + G.nz_local > h->g.nz_total)
+        return bail(MBIR_EINVAL);
+    if (G.nviews > 960) return (fail(h, MBIR_EINVAL, "nviews > 960 not supported"), bail(MBIR_EINVAL));
+    if (G.nchannels > (1 << 24)) return bail(MBIR_EINVAL);
+    const mbir_prior& P = h->pr;
+    if (!(P.p >= 1.0 && P.p <= 2.0) || P.q != 2.0 || !(P.T > 0) || !(P.sigma > 0) ||
+        (P.neighborhood != 8 && P.neighborhood != 26))
+        return bail(MBIR_EINVAL);
+    if (h->o.sv_side < 1 || h->o.sv_side > 16 || !(h->o.sv_fraction > 0 && h->o.sv_fraction <= 1) ||
+        h->o.batch_svs < 0)
+        return bail(MBIR_EINVAL);
+    if (h->nranks > 1 && (!d || !d->nccl_unique_id || h->rank < 0 || h->rank >= h->nranks))
+        return bail(MBIR_EINVAL);
+    if (G.angles) h->angles.assign(G.angles, G.angles + G.nviews);
+    h->g.angles = nullptr;
+
+    if (cudaSetDevice(h->device) != cudaSuccess) return bail(MBIR_ECUDA);
+    if (!h->st) {
+        if (cudaStreamCreateWithFlags(&h->st, cudaStreamNonBlocking) != cudaSuccess) return bail(MBIR_ECUDA);
+        h->own_stream = true;
+    }
+    int r;
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, h->device) != cudaSuccess) return bail(MBIR_ECUDA);
+    h->nsm = prop.multiProcessorCount;
+
+    // ---- SuperVoxel tiling (reading R13: ceil tiles, no overlap)
+    h->side = h->o.sv_side;
+    h->S2 = h->side * h->side;
+    h->nsvx = (G.nx + h->side - 1) / h->side;
+    h->nsvy = (G.ny + h->side - 1) / h->side;
+    h->nsv = h->nsvx * h->nsvy;
+    if (h->nsv > 16384) return (fail(h, MBIR_EINVAL, "too many SuperVoxels per slice (> 16384)"), bail(MBIR_EINVAL));
+    h->nsv_pad = 1;
+    while (h->nsv_pad < h->nsv) h->nsv_pad <<= 1;
+    h->max_group = ((h->nsvx + 1) / 2) * ((h->nsvy + 1) / 2);
+
+    // ---- view angles as (cos, sin) in double, computed on the host
+    {
+        std::vector<double> cs(2 * (size_t)G.nviews);
+        for (int k = 0; k < G.nviews; ++k) {
+            const double th = h->angles.empty() ? (double)k * 3.14159265358979323846 / (double)G.nviews : h->angles[k];
+            cs[2 * k] = cos(th);
+            cs[2 * k + 1] = sin(th);
+        }
+        if ((r = dalloc(h, &h->d_cs, cs.size()))) return bail(r);
+        if (cudaMemcpy(h->d_cs, cs.data(), cs.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess) return bail(MBIR_ECUDA);
+    }
+
+    // ---- system matrix, compressed per SV (a1)
+    const bool quant = h->o.quantize_A != 0;
+    const size_t nA = (size_t)h->nsv * h->S2 * G.nviews;
+    h->A.nsv = h->nsv;
+    h->A.S2 = h->S2;
+    h->A.V = G.nviews;
+    if (quant) {
+        if ((r = dalloc(h, &h->A.codes, nA))) return bail(r);
+    } else {
+        if ((r = dalloc(h, &h->A.vals, nA))) return bail(r);
+    }
+    if ((r = dalloc(h, &h->A.off, nA))) return bail(r);
+    if ((r = dalloc(h, &h->A.count, nA))) return bail(r);
+    if ((r = dalloc(h, &h->A.scale, (size_t)h->nsv * h->S2))) return bail(r);
+    if ((r = dalloc(h, &h->A.band_start, (size_t)h->nsv * G.nviews))) return bail(r);
+    if ((r = dalloc(h, &h->A.band_width, (size_t)h->nsv * G.nviews))) return bail(r);
+    int* d_info = nullptr;  // [err, maxrow, maxwidth]
+    if ((r = dalloc(h, &d_info, 3))) return bail(r);
+    cudaMemsetAsync(d_info, 0, 3 * sizeof(int), h->st);
+    if (build_sysmatrix(h->g, h->d_cs, h->side, h->nsvx, h->nsvy, quant, h->A, d_info, d_info + 1, h->st) != cudaSuccess) {
+        cudaFree(d_info);
+        return (fail(h, MBIR_ECUDA, "system matrix build failed"), bail(MBIR_ECUDA));
+    }
+    int info[3] = {0, 0, 0};
+    cudaMemcpyAsync(info, d_info, sizeof(info), cudaMemcpyDeviceToHost, h->st);
+    if (cudaStreamSynchronize(h->st) != cudaSuccess) {
+        cudaFree(d_info);
+        return bail(MBIR_ECUDA);
+    }
+    cudaFree(d_info);
+    if (info[0] & 1) return (fail(h, MBIR_EINVAL, "a voxel meets more than 4 channels in one view (dchannel too small vs dxy)"), bail(MBIR_EINVAL));
+    if (info[0] & 2) return (fail(h, MBIR_EINVAL, "SV band wider than 255 channels"), bail(MBIR_EINVAL));
+    h->rows = info[1];
+    h->band_max = info[2];
+    if (h->rows > kMaxSvbRows)
+        return (fail(h, MBIR_EINVAL, "SV band needs " + std::to_string(h->rows) + " > 32 buffer rows: reduce sv_side"), bail(MBIR_EINVAL));
+    h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
+
+    // ---- update-kernel shape
+    h->vpt = G.nviews > 384 ? 2 : 1;
+    h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
+    if (h->nvw > 15) return (fail(h, MBIR_EINVAL, "too many views"), bail(MBIR_EINVAL));
+    h->Vs = h->nvw * 32 * h->vpt;
+    h->threads = 32 * (h->nvw + 1);
+    if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
+    {
+        IcdParams p = make_params(h);
+        h->smem = icd_smem_bytes(p, h->vpt, P.neighborhood);
+        if (h->smem > (int)prop.sharedMemPerBlockOptin)
+            return (fail(h, MBIR_EINVAL, "SV buffer (" + std::to_string(h->smem) + " B) exceeds shared memory: reduce sv_side"), bail(MBIR_EINVAL));
+        h->blocks_per_sm = std::max(1, std::min((int)(prop.sharedMemPerMultiprocessor / (h->smem + 1024)),
+                                                (int)(2048 / h->threads)));
+    }
+
+    // ---- state buffers
+    const size_t ns = sino_elems(h), pl = plane_elems(h);
+    if ((r = dalloc(h, &h->d_y, ns))) return bail(r);
+    if ((r = dalloc(h, &h->d_w, ns))) return bail(r);
+    if ((r = dalloc(h, &h->d_e, ns))) return bail(r);
+    if ((r = dalloc(h, &h->d_x, pl * (G.nz_local + 2)))) return bail(r);
+    if ((r = dalloc(h, &h->d_theta2, (size_t)G.nz_local * h->nsv * h->S2))) return bail(r);
+    if ((r = dalloc(h, &h->d_amount, (size_t)G.nz_local * h->nsv))) return bail(r);
+    // e_init tiles of the concurrently running SV visits: one per CTA of the largest grid
+    if ((r = dalloc(h, &h->d_scratch, (size_t)(h->nsm * h->blocks_per_sm + G.nz_local) * h->Vs * 32))) return bail(r);
+    if ((r = dalloc(h, &h->d_task_list, (size_t)G.nz_local * 4 * h->max_group))) return bail(r);
+    if ((r = dalloc(h, &h->d_task_count, (size_t)G.nz_local * 4))) return bail(r);
+    if ((r = dalloc(h, &h->d_counters, 3))) return bail(r);
+    if ((r = dalloc(h, &h->d_sum_delta, 1))) return bail(r);
+    if ((r = dalloc(h, &h->d_flag, 1))) return bail(r);
+    if ((r = dalloc(h, &h->d_acc, 1))) return bail(r);
+    if (cudaMallocHost((void**)&h->h_counters, 4 * sizeof(unsigned long long)) != cudaSuccess) return bail(MBIR_ENOMEM);
+    cudaMemsetAsync(h->d_x, 0, sizeof(float) * pl * (G.nz_local + 2), h->st);
+    cudaMemsetAsync(h->d_amount, 0, sizeof(float) * G.nz_local * h->nsv, h->st);
+    if (cudaEventCreate(&h->ev0) != cudaSuccess || cudaEventCreate(&h->ev1) != cudaSuccess) return bail(MBIR_ECUDA);
+
+    // ---- prior constants (reading R1-R2)
+    {
+        PriorConst pc{};
+        int n = 0;
+        for (int dz = -1; dz <= 1; ++dz)
+            for (int dy = -1; dy <= 1; ++dy)
+                for (int dx = -1; dx <= 1; ++dx) {
+                    if (dx == 0 && dy == 0 && dz == 0) continue;
+                    if (P.neighborhood == 8 && dz != 0) continue;
+                    const int m = abs(dx) + abs(dy) + abs(dz);
+                    const double norm = P.neighborhood == 8 ? 4.0 + 4.0 / sqrt(2.0)
+                                                            : 6.0 + 12.0 / sqrt(2.0) + 8.0 / sqrt(3.0);
+                    pc.dx[n] = dx;
+                    pc.dy[n] = dy;
+                    pc.dz[n] = dz;
+                    pc.b[n] = (float)((1.0 / sqrt((double)m)) / norm);
+                    ++n;
+                }
+        pc.nnb = n;
+        pc.c_phi = (float)(1.0 / (2.0 * pow(P.sigma, P.p) * pow(P.T * P.sigma, P.q - P.p)));
+        pc.pq = (float)(P.q / P.p);
+        pc.qmp = (float)(P.q - P.p);
+        pc.inv_Ts = (float)(1.0 / (P.T * P.sigma));
+        pc.positivity = P.positivity;
+        if (set_prior_constants(pc) != cudaSuccess) return bail(MBIR_ECUDA);
+    }
+
+    // ---- multi-GPU communicator (z-slab partition)
+    if (h->nranks > 1) {
+        NcclApi& N = nccl();
+        if (!N.ok) return (fail(h, MBIR_ENOTSUP, "libnccl.so.2 not found"), bail(MBIR_ENOTSUP));
+        ncclUniqueId id;
+        memcpy(&id, d->nccl_unique_id, sizeof(id));
+        if (N.CommInitRank(&h->comm, h->nranks, id, h->rank) != ncclSuccess)
+            return (fail(h, MBIR_ENCCL, "ncclCommInitRank failed"), bail(MBIR_ENCCL));
+    }
+    if (cudaStreamSynchronize(h->st) != cudaSuccess) return bail(MBIR_ECUDA);
+    {
+        // nnz and band statistics (for the roofline accounting)
+        std::vector<uint8_t> cnt(nA), bw((size_t)h->nsv * G.nviews);
+        cudaMemcpy(cnt.data(), h->A.count, nA, cudaMemcpyDeviceToHost);
+        cudaMemcpy(bw.data(), h->A.band_width, bw.size(), cudaMemcpyDeviceToHost);
+        int64_t s = 0, b = 0;
+        for (uint8_t c : cnt) s += c;
+        for (uint8_t c : bw) b += c;
+        h->nnz = s;
+        h->band_entries = b;
+    }
+    *out = h;
+    return MBIR_OK;
+}
+
+int mbir_set_sinogram(mbir_handle* h, const float* y, const float* w, int where)
+{
+    if (!h || !y || !w) return MBIR_EINVAL;
+    const size_t ns = sino_elems(h);
+    CK(cudaMemcpyAsync(h->d_y, y, ns * 4, kind_in(where), h->st));
+    CK(cudaMemcpyAsync(h->d_w, w, ns * 4, kind_in(where), h->st));
+    CK(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->st));
+    CK(launch_check_finite(h->d_y, (int64_t)ns, 0, h->d_flag, h->st));
+    CK(launch_check_finite(h->d_w, (int64_t)ns, 1, h->d_flag, h->st));
+    int flag = 0;
+    CK(cudaMemcpyAsync(&flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    if (flag) {
+        h->have_sino = false;
+        return fail(h, MBIR_EINVAL, "y must be finite and w finite and >= 0");
+    }
+    int r = refresh_error(h, true);
+    if (r) return r;
+    CK(cudaMemsetAsync(h->d_amount, 0, sizeof(float) * h->g.nz_local * h->nsv, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    h->have_sino = true;
+    h->iter = 0;
+    return MBIR_OK;
+}
+
+int mbir_set_image(mbir_handle* h, const float* x0, int where)
+{
+    if (!h) return MBIR_EINVAL;
+    const size_t pl = plane_elems(h);
+    if (x0) {
+        CK(cudaMemcpyAsync(h->d_x + pl, x0, pl * h->g.nz_local * 4, kind_in(where), h->st));
+        CK(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->st));
+        CK(launch_check_finite(h->d_x + pl, (int64_t)(pl * h->g.nz_local), h->pr.positivity, h->d_flag, h->st));
+        int flag = 0;
+        CK(cudaMemcpyAsync(&flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost, h->st));
+        CK(cudaStreamSynchronize(h->st));
+        if (flag) {
+            cudaMemsetAsync(h->d_x + pl, 0, pl * h->g.nz_local * 4, h->st);
+            return fail(h, MBIR_EINVAL, "x0 must be finite (and >= 0 with positivity)");
+        }
+    } else {
+        CK(cudaMemsetAsync(h->d_x + pl, 0, pl * h->g.nz_local * 4, h->st));
+    }
+    int r = exchange_halo(h, -1);
+    if (r) return r;
+    if (h->have_sino) {
+        r = refresh_error(h, false);
+        if (r) return r;
+    }
+    CK(cudaMemsetAsync(h->d_amount, 0, sizeof(float) * h->g.nz_local * h->nsv, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    h->iter = 0;
+    return MBIR_OK;
+}
+
+int mbir_reconstruct(mbir_handle* h, double equits, mbir_stats* st)
+{
+    if (!h || !(equits >= 0)) return MBIR_EINVAL;
+    return run_iterations(h, -1, equits, st);
+}
+
+int mbir_iterate(mbir_handle* h, int n_iterations, mbir_stats* st)
+{
+    if (!h || n_iterations < 0) return MBIR_EINVAL;
+    return run_iterations(h, n_iterations, 0.0, st);
+}
+
+int mbir_get_image(mbir_handle* h, float* x, int where)
+{
+    if (!h || !x) return MBIR_EINVAL;
+    const size_t pl = plane_elems(h);
+    CK(cudaMemcpyAsync(x, h->d_x + pl, pl * h->g.nz_local * 4, kind_out(where), h->st));
+    CK(cudaStreamSynchronize(h->st));
+    return MBIR_OK;
+}
+
+int mbir_get_error_sinogram(mbir_handle* h, float* e, int where)
+{
+    if (!h || !e) return MBIR_EINVAL;
+    CK(cudaMemcpyAsync(e, h->d_e, sino_elems(h) * 4, kind_out(where), h->st));
+    CK(cudaStreamSynchronize(h->st));
+    return MBIR_OK;
+}
+
+int mbir_rmse_hu(mbir_handle* h, const float* golden, int where, double mu_water, double* out)
+{
+    if (!h || !golden || !out || !(mu_water > 0)) return MBIR_EINVAL;
+    const size_t pl = plane_elems(h), n = pl * h->g.nz_local;
+    const float* g = golden;
+    float* tmp = nullptr;
+    if (where != MBIR_DEVICE) {
+        CK(cudaMallocAsync((void**)&tmp, n * 4, h->st));
+        CK(cudaMemcpyAsync(tmp, golden, n * 4, cudaMemcpyHostToDevice, h->st));
+        g = tmp;
+    }
+    CK(cudaMemsetAsync(h->d_acc, 0, sizeof(double), h->st));
+    CK(launch_rmse_partial(h->d_x + pl, g, (int64_t)n, h->d_acc, h->st));
+    if (h->nranks > 1) CKN(nccl().AllReduce(h->d_acc, h->d_acc, 1, ncclFloat64, ncclSum, h->comm, h->st));
+    double s = 0.0;
+    CK(cudaMemcpyAsync(&s, h->d_acc, sizeof(double), cudaMemcpyDeviceToHost, h->st));
+    if (tmp) CK(cudaFreeAsync(tmp, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    *out = 1000.0 * sqrt(s / ((double)pl * h->g.nz_total)) / mu_water;
+    return MBIR_OK;
+}
+
+int mbir_query_sizes(const mbir_handle* h, mbir_sizes* s)
+{
+    if (!h || !s) return MBIR_EINVAL;
+    s->nsv_x = h->nsvx;
+    s->nsv_y = h->nsvy;
+    s->nsv = h->nsv;
+    s->K = kK;
+    s->band_max = h->band_max;
+    s->svb_rows = h->rows;
+    s->threads_per_cta = h->threads;
+    s->smem_bytes = h->smem;
+    s->nnz = h->nnz;
+    s->a_bytes = h->a_bytes;
+    s->band_entries = h->band_entries;
+    return MBIR_OK;
+}
+
+static int export_sysmatrix(mbir_handle* h, const int64_t* voxels, int nvox, int32_t* first,
+                            int32_t* count, float* values, uint8_t* codes, float* scales)
+{
+    const size_t n = voxels ? (size_t)nvox : plane_elems(h), V = h->g.nviews;
+    int32_t *df = nullptr, *dc = nullptr;
+    float *dv = nullptr, *ds = nullptr;
+    uint8_t* dq = nullptr;
+    int64_t* dvox = nullptr;
+    int rc = MBIR_OK;
+    auto cleanup = [&]() {
+        if (df) cudaFree(df);
+        if (dc) cudaFree(dc);
+        if (dv) cudaFree(dv);
+        if (ds) cudaFree(ds);
+        if (dq) cudaFree(dq);
+        if (dvox) cudaFree(dvox);
+    };
+    if ((first && (rc = dalloc(h, &df, n * V))) || (count && (rc = dalloc(h, &dc, n * V))) ||
+        (values && (rc = dalloc(h, &dv, n * V * kK))) || (codes && (rc = dalloc(h, &dq, n * V * kK))) ||
+        (scales && (rc = dalloc(h, &ds, n))) || (voxels && (rc = dalloc(h, &dvox, n)))) {
+        cleanup();
+        return rc;
+    }
+    cudaError_t e = cudaSuccess;
+    if (voxels) e = cudaMemcpyAsync(dvox, voxels, n * 8, cudaMemcpyHostToDevice, h->st);
+    if (e == cudaSuccess)
+        e = launch_export_sysmatrix(h->A, h->g.nx, h->g.ny, h->side, h->nsvx, dvox, (int)n, df, dc, dv,
+                                    dq, ds, h->g, h->d_cs, h->st);
+    if (e == cudaSuccess && first) e = cudaMemcpyAsync(first, df, n * V * 4, cudaMemcpyDeviceToHost, h->st);
+    if (e == cudaSuccess && count) e = cudaMemcpyAsync(count, dc, n * V * 4, cudaMemcpyDeviceToHost, h->st);
+    if (e == cudaSuccess && values) e = cudaMemcpyAsync(values, dv, n * V * kK * 4, cudaMemcpyDeviceToHost, h->st);
+    if (e == cudaSuccess && codes) e = cudaMemcpyAsync(codes, dq, n * V * kK, cudaMemcpyDeviceToHost, h->st);
+    if (e == cudaSuccess && scales) e = cudaMemcpyAsync(scales, ds, n * 4, cudaMemcpyDeviceToHost, h->st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->st);
+    cleanup();
+    if (e != cudaSuccess) return fail(h, MBIR_ECUDA, cudaGetErrorString(e));
+    return MBIR_OK;
+}
+
+int mbir_get_sysmatrix(mbir_handle* h, int32_t* first, int32_t* count, float* values,
+                       uint8_t* codes, float* scales)
+{
+    if (!h) return MBIR_EINVAL;
+    return export_sysmatrix(h, nullptr, 0, first, count, values, codes, scales);
+}
+
+int mbir_get_sysmatrix_columns(mbir_handle* h, const int64_t* voxels, int n, int32_t* first,
+                               int32_t* count, float* values, uint8_t* codes, float* scales)
+{
+    if (!h || !voxels || n <= 0) return MBIR_EINVAL;
+    for (int i = 0; i < n; ++i)
+        if (voxels[i] < 0 || voxels[i] >= (int64_t)plane_elems(h)) return fail(h, MBIR_EINVAL, "voxel index out of range");
+    return export_sysmatrix(h, voxels, n, first, count, values, codes, scales);
+}
+
+int mbir_probe_update(mbir_handle* h, const int64_t* voxels, int n, float* theta1, float* theta2,
+                      float* delta)
+{
+    if (!h || !voxels || n <= 0 || !theta1 || !theta2 || !delta) return MBIR_EINVAL;
+    if (!h->have_sino) return fail(h, MBIR_ESTATE, "mbir_set_sinogram has not been called");
+    const int64_t nv = (int64_t)plane_elems(h) * h->g.nz_local;
+    for (int i = 0; i < n; ++i)
+        if (voxels[i] < 0 || voxels[i] >= nv) return fail(h, MBIR_EINVAL, "voxel index out of range");
+    int64_t* dvox = nullptr;
+    float* dout = nullptr;
+    CK(cudaMallocAsync((void**)&dvox, n * 8, h->st));
+    CK(cudaMallocAsync((void**)&dout, n * 12, h->st));
+    CK(cudaMemcpyAsync(dvox, voxels, n * 8, cudaMemcpyHostToDevice, h->st));
+    IcdParams p = make_params(h);
+    CK(launch_probe(p, h->o.quantize_A != 0, h->pr.neighborhood, dvox, n, dout, h->st));
+    std::vector<float> out((size_t)n * 3);
+    CK(cudaMemcpyAsync(out.data(), dout, n * 12, cudaMemcpyDeviceToHost, h->st));
+    CK(cudaFreeAsync(dvox, h->st));
+    CK(cudaFreeAsync(dout, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    for (int i = 0; i < n; ++i) {
+        theta1[i] = out[3 * i];
+        theta2[i] = out[3 * i + 1];
+        delta[i] = out[3 * i + 2];
+    }
+    return MBIR_OK;
+}
+
+}  // extern "C"

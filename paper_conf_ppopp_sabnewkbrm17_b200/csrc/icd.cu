@@ -1,0 +1,695 @@
+// Fused SuperVoxel ICD update kernel for sm_100a, plus the
+// theta2 precompute, forward projection and probe kernels that share its data layout.
+//
+// Paper: Alg. 1 is the per-voxel update; Alg. 3 runs it with
+// intra-voxel, intra-SV and inter-SV parallelism over SV buffers
+// created before and written back after the update.
+//
+// B200 design: one CTA owns one (slice, SV) task at a time
+// (persistent over the phase's task list).  Its threads own VIEWS: warp w, lane l owns views
+// (w*VPT + t)*32 + l, t < VPT.  The SV buffer (e and w over the SV's sinogram band) lives in
+// shared memory as [row = channel offset in band][view] with a view stride that is a multiple
+// of 32, so a warp's 32 lanes always hit 32 distinct banks whatever the voxel's per-view
+// offsets (conflict-free gather and scatter without atomics: a thread is the only writer of
+// its views).  Voxels of the SV are updated one after another in a random order, exactly as
+// sequential ICD within the SV: per voxel, every view thread gathers its part of
+// theta1 = -sum w A e from shared memory (A streamed from HBM, prefetched RING voxels ahead),
+// a warp-shuffle reduction and ONE __syncthreads hand the partial sums to every warp, a
+// dedicated prior warp has meanwhile computed the q-GGMRF surrogate terms over the voxel's
+// neighbourhood from a shared-memory x tile, and every warp derives the same delta and
+// scatters e -= A delta into its own views.  theta2 = A^T W A is fixed by w and is
+// precomputed per (slice, voxel) when the sinogram is loaded.  The SVB is packed and written
+// back with coalesced 128-byte row accesses transposed through warp shuffles; the write-back
+// adds the band's delta e atomically (red.global.add.f32) because same-colour SVs of a batch
+// share sinogram entries.
+#include "mbir_internal.h"
+
+namespace mbir {
+
+__constant__ PriorConst c_prior;
+
+cudaError_t set_prior_constants(const PriorConst& pc)
+{
+    return cudaMemcpyToSymbol(c_prior, &pc, sizeof(pc));
+}
+
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// phi(D) = rho'(D)/(2D) for the q-GGMRF potential with q = 2 (reading R1):
+//   phi = c_phi * (q/p + u) / (1 + u)^2,  u = |D/(T sigma)|^(q-p)   (|D|^(q-2) = 1)
+__device__ __forceinline__ float phi_f(float d)
+{
+    const float ad = fabsf(d);
+    float u;
+    if (c_prior.qmp == 0.f)
+        u = 1.f;
+    else
+        u = (ad == 0.f) ? 0.f : exp2f(c_prior.qmp * __log2f(ad * c_prior.inv_Ts));
+    const float opu = 1.f + u;
+    return c_prior.c_phi * (c_prior.pq + u) / (opu * opu);
+}
+
+// uint8 code i of a packed word -> float, via the 2^23 magic (PRMT + FADD, no I2F)
+__device__ __forceinline__ float dq(uint32_t word, int i)
+{
+    const uint32_t b = __byte_perm(word, 0x4B000000u, 0x7440u | (uint32_t)i);
+    return __uint_as_float(b) - 8388608.f;
+}
+
+// In-register 32x32 transpose across a warp: on return lane l holds in r[i] what lane i held
+// in r[l].  5 butterfly stages of 16 shuffles.
+__device__ __forceinline__ void transpose32(float (&r)[32], int lane)
+{
+#pragma unroll
+    for (int s = 4; s >= 0; --s) {
+        const int b = 1 << s;
+        const bool upper = (lane & b) != 0;
+#pragma unroll
+        for (int i = 0; i < 32; ++i) {
+            if ((i & b) == 0) {
+                const int j = i | b;
+                const float send = upper ? r[i] : r[j];
+                const float recv = __shfl_xor_sync(kFull, send, b);
+                if (upper)
+                    r[i] = recv;
+                else
+                    r[j] = recv;
+            }
+        }
+    }
+}
+
+__device__ __forceinline__ void red_add_f32(float* p, float v)
+{
+    asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z)
+{
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+struct PriSlot {
+    float sb, sbx, v, pad;
+};
+
+struct SmemLayout {
+    int sb_e, sb_w, xt, list, flags, red, pri, vscale, vth2, misc, total;
+};
+
+__host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
+
+__host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, int S2, int nnb)
+{
+    SmemLayout L;
+    const int TW = side + 2;
+    const int nzt = nnb == 26 ? 3 : 1;
+    int o = 0;
+    L.sb_e = o;  o = align16(o + rows * Vs * 4);
+    L.sb_w = o;  o = align16(o + rows * Vs * 4);
+    L.xt = o;    o = align16(o + nzt * TW * TW * 4);
+    L.list = o;  o = align16(o + S2 * 4);
+    L.flags = o; o = align16(o + S2 * 4);
+    L.red = o;   o = align16(o + 2 * 16 * 4);
+    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriSlot));
+    L.vscale = o; o = align16(o + S2 * 4);
+    L.vth2 = o;  o = align16(o + S2 * 4);
+    L.misc = o;  o = align16(o + 16 * 4);
+    L.total = o;
+    return L;
+}
+
+template <int VPT, bool U8, int NNB, int RING>
+__global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
+{
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int nvw = P.nvw;
+    const int V = P.V, M = P.M, Vs = P.Vs, S2 = P.S2, side = P.side;
+    const SmemLayout L = smem_layout(P.rows, Vs, side, S2, NNB);
+    float* sb_e = (float*)(smem + L.sb_e);
+    float* sb_w = (float*)(smem + L.sb_w);
+    float* xt = (float*)(smem + L.xt);
+    int* list = (int*)(smem + L.list);
+    int* flags = (int*)(smem + L.flags);
+    float* red = (float*)(smem + L.red);
+    PriSlot* pri = (PriSlot*)(smem + L.pri);
+    float* vscale = (float*)(smem + L.vscale);
+    float* vth2 = (float*)(smem + L.vth2);
+    const int TW = side + 2;
+    const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
+    const size_t plane = (size_t)P.nx * P.ny;
+
+    const int z = P.zfirst + blockIdx.y * P.zstride;  // local slice
+    if (z >= P.nz_local) return;
+    const int zg = P.z_offset + z;                    // global slice
+    const int tq = z * 4 + P.colour;
+    const int cnt = P.task_count[tq];
+    if (P.thr > 0 && cnt - P.batch_base < P.thr) return;  // Alg3:26-27 threshold break
+    const int pend = min(cnt, P.batch_base + P.batch);
+
+    for (int pos = P.batch_base + blockIdx.x; pos < pend; pos += gridDim.x) {
+        const int sv = P.task_list[(size_t)tq * P.max_group + pos];
+        const int bx = sv % P.nsvx, by = sv / P.nsvx;
+        const int gx0 = bx * side, gy0 = by * side;
+        const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
+
+        // ---- 1. x tile (+1 halo ring, +-1 slice in 3-D) into shared memory
+        for (int i = threadIdx.x; i < (NNB == 26 ? 3 : 1) * TW * TW; i += blockDim.x) {
+            const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
+            const int gx = gx0 - 1 + tx, gy = gy0 - 1 + ty;
+            const int zs = (NNB == 26) ? z + tz : z + 1;  // storage slice (halo at 0, nz+1)
+            float v = 0.f;
+            if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny) v = P.x[zs * plane + (size_t)gy * P.nx + gx];
+            xt[i] = v;
+        }
+        __syncthreads();
+
+        // ---- 2. zero-skip predicate at visit start (reading R9): slot v kept iff valid
+        //         and (skip inactive or x_j or a neighbour is non-zero)
+        int keep = 0;
+        const int v0 = threadIdx.x;
+        if (v0 < S2) {
+            const int lx = v0 % side, ly = v0 / side;
+            if (lx < tw && ly < th) {
+                keep = 1;
+                if (P.zero_skip_active) {
+                    keep = xt[(zc * TW + ly + 1) * TW + lx + 1] != 0.f;
+                    for (int r = 0; r < c_prior.nnb && !keep; ++r) {
+                        const int gx = gx0 + lx + c_prior.dx[r], gy = gy0 + ly + c_prior.dy[r];
+                        const int gz = zg + c_prior.dz[r];
+                        if (gx < 0 || gx >= P.nx || gy < 0 || gy >= P.ny || gz < 0 || gz >= P.nz_total) continue;
+                        keep = xt[((zc + c_prior.dz[r]) * TW + ly + 1 + c_prior.dy[r]) * TW + lx + 1 + c_prior.dx[r]] != 0.f;
+                    }
+                }
+            }
+            flags[v0] = keep;
+        }
+        const int nact = __syncthreads_count(keep);
+        if (nact == 0) {
+            if (threadIdx.x == 0) {
+                P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
+                atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
+                atomicAdd(P.counters + 2, 1ull);
+            }
+            __syncthreads();
+            continue;
+        }
+
+        // ---- 3. visiting order: random permutation of the tile, compacted to the kept
+        //         voxels with a warp ballot; per-voxel scale and theta2 staged in smem
+        if (warp == nvw) {
+            const uint64_t h = mix64(P.seed ^ mix64(((uint64_t)P.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)sv));
+            if (lane == 0) {
+                for (int i = 0; i < S2; ++i) list[i] = i;
+                if (!P.deterministic) {
+                    uint64_t st = h;
+                    for (int i = S2 - 1; i > 0; --i) {
+                        st += 0x9E3779B97F4A7C15ULL;
+                        const int r = (int)(mix64(st) % (uint64_t)(i + 1));
+                        const int t = list[i];
+                        list[i] = list[r];
+                        list[r] = t;
+                    }
+                }
+            }
+            __syncwarp();
+            int n = 0;
+            for (int base = 0; base < S2; base += 32) {
+                const int i = base + lane;
+                const int v = i < S2 ? list[i] : 0;
+                const bool k = i < S2 && flags[v];
+                const unsigned m = __ballot_sync(kFull, k);
+                __syncwarp();
+                if (k) list[n + __popc(m & ((1u << lane) - 1))] = v;
+                n += __popc(m);
+                __syncwarp();
+            }
+            for (int i = lane; i < nact; i += 32) {
+                const int v = list[i];
+                vscale[i] = P.A.scale[(size_t)sv * S2 + v];
+                vth2[i] = P.theta2[((size_t)z * P.nsv + sv) * S2 + v];
+            }
+        }
+        __syncthreads();
+
+        // ---- 4. view threads: A prefetch ring + SVB pack (w, then e with e_init kept in regs)
+        int kv[VPT];
+        bool kval[VPT];
+#pragma unroll
+        for (int t = 0; t < VPT; ++t) {
+            kv[t] = (warp * VPT + t) * 32 + lane;
+            kval[t] = warp < nvw && kv[t] < V;
+        }
+        const size_t abase = (size_t)sv * S2 * V;
+        uint32_t rc[VPT][RING];
+        uint32_t ro[VPT];  // RING 8-bit band offsets packed per view
+        float4 rv[VPT][RING];
+        // e_init (band of e at pack time) goes to this CTA's L2-resident scratch tile,
+        // row-major [view][32 channels], written and re-read with coalesced 128-byte rows
+        float* scr = P.scratch + ((size_t)blockIdx.y * gridDim.x + blockIdx.x) * (size_t)Vs * 32;
+        if (warp < nvw) {
+#pragma unroll
+            for (int u = 0; u < RING; ++u) {
+#pragma unroll
+                for (int t = 0; t < VPT; ++t) {
+                    rc[t][u] = 0u;
+                    if (u == 0) ro[t] = 0u;
+                    rv[t][u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (u < nact && kval[t]) {
+                        const size_t ai = abase + (size_t)list[u] * V + kv[t];
+                        if (U8)
+                            rc[t][u] = __ldg(P.A.codes + ai);
+                        else
+                            rv[t][u] = __ldg(P.A.vals + ai);
+                        ro[t] |= (uint32_t)__ldg(P.A.off + ai) << (8 * u);
+                    }
+                }
+            }
+            const float* wz = P.w + (size_t)z * V * M;
+            float* ez = P.e + (size_t)z * V * M;
+#pragma unroll 1
+            for (int t = 0; t < VPT; ++t) {
+                const int k0 = (warp * VPT + t) * 32;
+                const int kk = k0 + lane;
+                const int bw = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
+                // 32-bit element offset of this lane's band row; rows are broadcast by shuffle
+                const int roff = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
+                float r[32];
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                    const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
+                    r[i] = lane < wi ? __ldg(wz + oi + lane) : 0.f;
+                }
+                transpose32(r, lane);
+#pragma unroll
+                for (int c = 0; c < 32; ++c)
+                    if (c < P.rows) sb_w[c * Vs + kk] = r[c];
+                asm volatile("" ::: "memory");  // keep the e loads after the w tile is retired
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                    const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
+                    r[i] = lane < wi ? __ldcg(ez + oi + lane) : 0.f;
+                    __stcg(scr + (k0 + i) * 32 + lane, r[i]);
+                }
+                transpose32(r, lane);
+#pragma unroll
+                for (int c = 0; c < 32; ++c)
+                    if (c < P.rows) sb_e[c * Vs + kk] = r[c];
+            }
+        }
+        __syncthreads();
+
+        // ---- 5. sequential-exact voxel loop, one barrier per voxel
+        float amount = 0.f;
+        const int cslot = (zc * TW + 1) * TW + 1;  // tile index of local (0,0)
+        for (int base = 0; base < nact; base += RING) {
+#pragma unroll
+            for (int u = 0; u < RING; ++u) {
+                const int idx = base + u;
+                if (idx >= nact) break;
+                const int buf = idx & 1;
+                float ev[VPT][4];
+                uint32_t cw[VPT];
+                float4 av[VPT];
+                int oo[VPT];
+                if (warp < nvw) {
+                    float t1 = 0.f;
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t) {
+                        oo[t] = (int)((ro[t] >> (8 * u)) & 0xffu);
+                        cw[t] = rc[t][u];
+                        av[t] = rv[t][u];
+                        if (kval[t]) {
+                            const int o = oo[t];
+                            float acc = 0.f;
+#pragma unroll
+                            for (int i = 0; i < 4; ++i) {
+                                const float ee = sb_e[(o + i) * Vs + kv[t]];
+                                const float ww = sb_w[(o + i) * Vs + kv[t]];
+                                ev[t][i] = ee;
+                                const float a = U8 ? dq(cw[t], i)
+                                                   : (i == 0 ? av[t].x : i == 1 ? av[t].y : i == 2 ? av[t].z : av[t].w);
+                                acc = fmaf(ww * ee, a, acc);
+                            }
+                            t1 += acc;
+                        }
+                    }
+                    // refill this ring slot with voxel idx + RING
+                    if (idx + RING < nact) {
+                        const size_t vb = abase + (size_t)list[idx + RING] * V;
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t)
+                            if (kval[t]) {
+                                if (U8)
+                                    rc[t][u] = __ldg(P.A.codes + vb + kv[t]);
+                                else
+                                    rv[t][u] = __ldg(P.A.vals + vb + kv[t]);
+                                ro[t] = (ro[t] & ~(0xffu << (8 * u))) | ((uint32_t)__ldg(P.A.off + vb + kv[t]) << (8 * u));
+                            }
+                    }
+#pragma unroll
+                    for (int o = 16; o > 0; o >>= 1) t1 += __shfl_xor_sync(kFull, t1, o);
+                    if (lane == 0) red[buf * 16 + warp] = t1;
+                } else {
+                    // prior warp: surrogate terms of Alg1:7 over the neighbourhood (reading R1-R2)
+                    __syncwarp();  // lane 0's x-tile write of the previous voxel is visible
+                    const int slot = list[idx];
+                    const int lx = slot % side, ly = slot / side;
+                    const float v = xt[cslot + ly * TW + lx];
+                    float sbv = 0.f, sbx = 0.f;
+                    if (lane < NNB) {
+                        const int dx = c_prior.dx[lane], dy = c_prior.dy[lane], dz = c_prior.dz[lane];
+                        const int gx = gx0 + lx + dx, gy = gy0 + ly + dy, gz = zg + dz;
+                        if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
+                            const float xr = xt[cslot + (dz * TW + ly + dy) * TW + lx + dx];
+                            const float bt = c_prior.b[lane] * phi_f(v - xr);
+                            sbv = bt;
+                            sbx = bt * xr;
+                        }
+                    }
+#pragma unroll
+                    for (int o = 16; o > 0; o >>= 1) {
+                        sbv += __shfl_xor_sync(kFull, sbv, o);
+                        sbx += __shfl_xor_sync(kFull, sbx, o);
+                    }
+                    if (lane == 0) {
+                        PriSlot ps;
+                        ps.sb = sbv;
+                        ps.sbx = sbx;
+                        ps.v = v;
+                        ps.pad = 0.f;
+                        pri[buf] = ps;
+                    }
+                }
+                __syncthreads();
+                // every warp derives the same delta (identical inputs, identical order)
+                float s1 = 0.f;
+                {
+                    const float4* r4 = (const float4*)(red + buf * 16);
+                    float part[16];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const float4 a = r4[q];
+                        part[4 * q] = a.x;
+                        part[4 * q + 1] = a.y;
+                        part[4 * q + 2] = a.z;
+                        part[4 * q + 3] = a.w;
+                    }
+#pragma unroll
+                    for (int q = 0; q < 16; ++q)
+                        if (q < nvw) s1 += part[q];
+                }
+                const PriSlot ps = pri[buf];
+                const float scale = vscale[idx];
+                const float theta1 = -scale * s1;   // Alg1:5, theta1 = -sum w A e
+                const float theta2 = vth2[idx];     // Alg1:6, precomputed sum w A^2
+                const float num = theta2 * ps.v - theta1 + 2.f * ps.sbx;
+                const float den = theta2 + 2.f * ps.sb;
+                float unew = den > 0.f ? num / den : ps.v;
+                if (c_prior.positivity) unew = fmaxf(unew, 0.f);
+                const float delta = unew - ps.v;  // Alg1:7-8
+                if (warp < nvw) {
+                    if (delta != 0.f) {  // Alg1:9-11: e -= A delta on this thread's views
+                        const float sd = scale * delta;
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t)
+                            if (kval[t]) {
+#pragma unroll
+                                for (int i = 0; i < 4; ++i) {
+                                    const float a = U8 ? dq(cw[t], i)
+                                                       : (i == 0 ? av[t].x : i == 1 ? av[t].y : i == 2 ? av[t].z : av[t].w);
+                                    sb_e[(oo[t] + i) * Vs + kv[t]] = fmaf(-a, sd, ev[t][i]);
+                                }
+                            }
+                    }
+                } else if (lane == 0) {
+                    const int slot = list[idx];
+                    xt[cslot + (slot / side) * TW + slot % side] = unew;
+                    amount += fabsf(delta);
+                }
+            }
+        }
+        __syncthreads();
+
+        // ---- 6. write-back: delta e of the band, atomically, and the SV's voxels
+        if (warp < nvw) {
+            float* ez = P.e + (size_t)z * V * M;
+#pragma unroll 1
+            for (int t = 0; t < VPT; ++t) {
+                const int k0 = (warp * VPT + t) * 32;
+                const int kk = k0 + lane;
+                float r[32];
+#pragma unroll
+                for (int c = 0; c < 32; ++c)
+                    r[c] = (kk < V && c < P.rows) ? sb_e[c * Vs + kk] : 0.f;
+                transpose32(r, lane);
+                const int bw = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
+                const int roff = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                    const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
+                    if (lane < wi) {
+                        const float d = r[i] - __ldcg(scr + (k0 + i) * 32 + lane);
+                        if (d != 0.f) red_add_f32(ez + oi + lane, d);
+                    }
+                }
+            }
+        } else {
+            for (int i = lane; i < tw * th; i += 32) {
+                const int lx = i % tw, ly = i / tw;
+                P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] =
+                    xt[cslot + ly * TW + lx];
+            }
+            if (lane == 0) {
+                P.sv_amount[(size_t)z * P.nsv + sv] = amount;
+                atomicAdd(P.counters + 0, (unsigned long long)nact);
+                atomicAdd(P.counters + 1, (unsigned long long)(tw * th - nact));
+                atomicAdd(P.counters + 2, 1ull);
+                atomicAdd(P.sum_delta, (double)amount);
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// theta2[z][sv][slot] = sum_k sum_i w * A^2 (Alg1:6), fixed for a given sinogram.
+// One warp per voxel, lanes over views; reads w straight from HBM (setup-time kernel).
+template <bool U8>
+__global__ void k_theta2(const IcdParams P)
+{
+    const int lane = threadIdx.x & 31;
+    const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const int z = blockIdx.y;
+    if (gw >= P.nsv * P.S2) return;
+    const int sv = gw / P.S2, slot = gw % P.S2;
+    const size_t ab = ((size_t)sv * P.S2 + slot) * P.V;
+    const float* wz = P.w + (size_t)z * P.V * P.M;
+    const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
+    float acc = 0.f;
+    for (int k = lane; k < P.V; k += 32) {
+        const int f = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + k];
+        const int n = P.A.count[ab + k];
+        float a[4];
+        if (U8) {
+            const uint32_t c = P.A.codes[ab + k];
+            for (int i = 0; i < 4; ++i) a[i] = dq(c, i) * sc;
+        } else {
+            const float4 q = P.A.vals[ab + k];
+            a[0] = q.x; a[1] = q.y; a[2] = q.z; a[3] = q.w;
+        }
+        for (int i = 0; i < 4; ++i)
+            if (i < n) acc += wz[(size_t)k * P.M + f + i] * a[i] * a[i];
+    }
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(kFull, acc, o);
+    if (lane == 0) P.theta2[((size_t)z * P.nsv + sv) * P.S2 + slot] = acc;
+}
+
+// e[z] += -A x[z] for one (slice, SV) per block (e must hold y on entry).  Threads own views;
+// accumulates the SV's band in smem, then adds it to e atomically.  Setup-time kernel.
+template <bool U8>
+__global__ void k_forward(const IcdParams P)
+{
+    extern __shared__ __align__(16) unsigned char smem[];
+    float* acc = (float*)smem;  // [rows][Vs]
+    const int sv = blockIdx.x, z = blockIdx.y;
+    const int bx = sv % P.nsvx, by = sv / P.nsvx;
+    const int gx0 = bx * P.side, gy0 = by * P.side;
+    const int tw = min(P.side, P.nx - gx0), th = min(P.side, P.ny - gy0);
+    const size_t plane = (size_t)P.nx * P.ny;
+    for (int i = threadIdx.x; i < P.rows * P.Vs; i += blockDim.x) acc[i] = 0.f;
+    __syncthreads();
+    bool any = false;
+    for (int k = threadIdx.x; k < P.V; k += blockDim.x) {
+        for (int slot = 0; slot < P.S2; ++slot) {
+            const int lx = slot % P.side, ly = slot / P.side;
+            if (lx >= tw || ly >= th) continue;
+            const float xv = P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx];
+            if (xv == 0.f) continue;
+            any = true;
+            const size_t ai = ((size_t)sv * P.S2 + slot) * P.V + k;
+            const int o = P.A.off[ai];
+            const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
+            for (int i = 0; i < 4; ++i) {
+                float a;
+                if (U8) {
+                    a = dq(P.A.codes[ai], i) * sc;
+                } else {
+                    const float4 q = P.A.vals[ai];
+                    a = i == 0 ? q.x : i == 1 ? q.y : i == 2 ? q.z : q.w;
+                }
+                acc[(o + i) * P.Vs + k] += a * xv;
+            }
+        }
+    }
+    if (!__syncthreads_or(any)) return;
+    float* ez = P.e + (size_t)z * P.V * P.M;
+    for (int k = threadIdx.x; k < P.V; k += blockDim.x) {
+        const int bs = P.A.band_start[(size_t)sv * P.V + k];
+        const int bw = P.A.band_width[(size_t)sv * P.V + k];
+        for (int c = 0; c < bw; ++c) {
+            const float d = acc[c * P.Vs + k];
+            if (d != 0.f) red_add_f32(ez + (size_t)k * P.M + bs + c, -d);
+        }
+    }
+}
+
+// Alg. 1 steps 1-7 for given voxels at the current state, from GLOBAL e/w/x (test hook).
+template <bool U8>
+__global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
+{
+    const int q = blockIdx.x;
+    const int64_t j = vox[q];
+    const size_t plane = (size_t)P.nx * P.ny;
+    const int z = (int)(j / plane);
+    const int iy = (int)((j % plane) / P.nx), ix = (int)(j % P.nx);
+    const int sv = (iy / P.side) * P.nsvx + ix / P.side;
+    const int slot = (iy % P.side) * P.side + ix % P.side;
+    const size_t ab = ((size_t)sv * P.S2 + slot) * P.V;
+    const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
+    const float* wz = P.w + (size_t)z * P.V * P.M;
+    const float* ez = P.e + (size_t)z * P.V * P.M;
+    float t1 = 0.f, t2 = 0.f;
+    for (int k = threadIdx.x; k < P.V; k += blockDim.x) {
+        const int f = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + k];
+        const int n = P.A.count[ab + k];
+        for (int i = 0; i < 4 && i < n; ++i) {
+            float a;
+            if (U8) {
+                a = dq(P.A.codes[ab + k], i) * sc;
+            } else {
+                const float4 v4 = P.A.vals[ab + k];
+                a = i == 0 ? v4.x : i == 1 ? v4.y : i == 2 ? v4.z : v4.w;
+            }
+            const float ww = wz[(size_t)k * P.M + f + i];
+            t1 -= ww * a * ez[(size_t)k * P.M + f + i];
+            t2 += ww * a * a;
+        }
+    }
+    __shared__ float r1[32], r2[32];
+    for (int o = 16; o > 0; o >>= 1) {
+        t1 += __shfl_xor_sync(kFull, t1, o);
+        t2 += __shfl_xor_sync(kFull, t2, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        r1[threadIdx.x >> 5] = t1;
+        r2[threadIdx.x >> 5] = t2;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        float T1 = 0.f, T2 = 0.f;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
+            T1 += r1[w];
+            T2 += r2[w];
+        }
+        const float v = P.x[(size_t)(z + 1) * plane + (size_t)iy * P.nx + ix];
+        float sbv = 0.f, sbx = 0.f;
+        const int zg = P.z_offset + z;
+        for (int r = 0; r < c_prior.nnb; ++r) {
+            const int gx = ix + c_prior.dx[r], gy = iy + c_prior.dy[r], gz = zg + c_prior.dz[r];
+            if (gx < 0 || gx >= P.nx || gy < 0 || gy >= P.ny || gz < 0 || gz >= P.nz_total) continue;
+            const float xr = P.x[(size_t)(z + 1 + c_prior.dz[r]) * plane + (size_t)gy * P.nx + gx];
+            const float bt = c_prior.b[r] * phi_f(v - xr);
+            sbv += bt;
+            sbx += bt * xr;
+        }
+        const float num = T2 * v - T1 + 2.f * sbx, den = T2 + 2.f * sbv;
+        float u = den > 0.f ? num / den : v;
+        if (c_prior.positivity) u = fmaxf(u, 0.f);
+        out3[3 * q] = T1;
+        out3[3 * q + 1] = T2;
+        out3[3 * q + 2] = u - v;
+    }
+}
+
+}  // namespace
+
+int icd_smem_bytes(const IcdParams& p, int vpt, int nnb)
+{
+    (void)vpt;
+    return smem_layout(p.rows, p.Vs, p.side, p.S2, nnb).total;
+}
+
+template <int VPT, bool U8, int NNB>
+static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t st)
+{
+    constexpr int RING = U8 ? 4 : 2;
+    auto kern = k_icd_sv<VPT, U8, NNB, RING>;
+    const int smem = smem_layout(p.rows, p.Vs, p.side, p.S2, NNB).total;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    kern<<<dim3(gx, gy), 32 * (p.nvw + 1), smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int gx, int gy,
+                       cudaStream_t st)
+{
+    if (vpt == 1) {
+        if (quantize) return nnb == 26 ? launch_icd_t<1, true, 26>(p, gx, gy, st) : launch_icd_t<1, true, 8>(p, gx, gy, st);
+        return nnb == 26 ? launch_icd_t<1, false, 26>(p, gx, gy, st) : launch_icd_t<1, false, 8>(p, gx, gy, st);
+    }
+    if (quantize) return nnb == 26 ? launch_icd_t<2, true, 26>(p, gx, gy, st) : launch_icd_t<2, true, 8>(p, gx, gy, st);
+    return nnb == 26 ? launch_icd_t<2, false, 26>(p, gx, gy, st) : launch_icd_t<2, false, 8>(p, gx, gy, st);
+}
+
+cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st)
+{
+    const int wpb = 8;
+    dim3 grid((p.nsv * p.S2 + wpb - 1) / wpb, p.nz_local);
+    if (quantize)
+        k_theta2<true><<<grid, 32 * wpb, 0, st>>>(p);
+    else
+        k_theta2<false><<<grid, 32 * wpb, 0, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cudaStream_t st)
+{
+    cudaError_t e = cudaMemcpyAsync(p.e, y, sizeof(float) * (size_t)p.nz_local * p.V * p.M,
+                                    cudaMemcpyDeviceToDevice, st);
+    if (e != cudaSuccess) return e;
+    const int smem = p.rows * p.Vs * 4;
+    auto k = quantize ? k_forward<true> : k_forward<false>;
+    e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    k<<<dim3(p.nsv, p.nz_local), 256, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_probe(const IcdParams& p, bool quantize, int nnb, const int64_t* vox, int n,
+                         float* out3, cudaStream_t st)
+{
+    (void)nnb;
+    if (quantize)
+        k_probe<true><<<n, 256, 0, st>>>(p, vox, out3);
+    else
+        k_probe<false><<<n, 256, 0, st>>>(p, vox, out3);
+    return cudaGetLastError();
+}
+
+}  // namespace mbir

@@ -1,0 +1,107 @@
+// Internal declarations of libmbir (not part of the C-ABI).  See include/mbir.h for the public
+// contract and DESIGN.md for the data layout and kernel design.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/mbir.h"
+
+namespace mbir {
+
+constexpr int kK = 4;             // max channels per (voxel, view) (reading R5; K=4 for dc > 0.4714 dxy)
+constexpr int kMaxNbr = 26;       // 3-D neighbourhood (reading R2)
+constexpr int kRingDepth = 4;     // A-record prefetch depth (voxels) in the update kernel
+constexpr int kMaxSvbRows = 32;   // SV-buffer rows held by one 32-lane transpose tile
+constexpr int kMaxThreads = 1024;
+
+// ---- prior constants in __constant__ memory (set by set_prior_constants) ----
+struct PriorConst {
+    int nnb;                 // 8 or 26
+    int dx[kMaxNbr], dy[kMaxNbr], dz[kMaxNbr];
+    float b[kMaxNbr];        // b_jr (reading R2)
+    float c_phi;             // 1 / (2 sigma^p (T sigma)^(q-p))
+    float pq;                // q / p
+    float qmp;               // q - p
+    float inv_Ts;            // 1 / (T sigma)
+    int positivity;
+};
+
+// ---- compressed system matrix, per SuperVoxel ----
+struct DevA {
+    int nsv, S2, V;          // SVs per slice, slots per SV (side^2), views
+    uint32_t* codes;         // [nsv][S2][V] 4 uint8 codes (byte i = channel offset i), quantize_A
+    float4* vals;            // [nsv][S2][V] fp32 values, !quantize_A
+    uint8_t* off;            // [nsv][S2][V] first channel - band start
+    uint8_t* count;          // [nsv][S2][V] channels used (export only)
+    float* scale;            // [nsv][S2] amax_j / 255 (quantize_A) or 1
+    int32_t* band_start;     // [nsv][V] first channel of the SV band
+    uint8_t* band_width;     // [nsv][V] band width (channels)
+};
+
+// ---- parameters of the fused SuperVoxel update kernel ----
+struct IcdParams {
+    int nx, ny, nz_local, z_offset, nz_total;
+    int V, M;
+    int side, nsvx, nsv, S2;
+    int Vs;                  // shared-memory column stride (views), multiple of 32
+    int rows;                // shared-memory SVB rows (channels)
+    int nvw;                 // view warps (the prior warp is warp nvw)
+    DevA A;
+    float* e;                // [nz_local][V][M]
+    const float* w;          // [nz_local][V][M]
+    float* x;                // [nz_local + 2][ny][nx] (halo slice at each end)
+    float* theta2;           // [nz_local][nsv][S2]
+    float* scratch;          // [max CTAs][Vs][32] e_init tiles of the running SV visits
+    float* sv_amount;        // [nz_local][nsv] sum |delta| of the SV's last visit
+    const int* task_list;    // [nz_local][4][max_group]
+    const int* task_count;   // [nz_local][4]
+    int max_group;
+    int colour, zfirst, zstride, batch_base, batch, thr;
+    unsigned long long* counters;  // [0] updates [1] skipped [2] sv visits
+    double* sum_delta;
+    uint64_t seed;
+    int iter;
+    int zero_skip_active;
+    int deterministic;
+};
+
+struct SchedParams {
+    int nz_local, z_offset;
+    int nsvx, nsvy, nsv, nsv_pad;
+    int nsel;                // SVs selected per slice this iteration
+    int mode;                // 0 all (random order), 1 top by amount, 2 random, 3 all in index order
+    int max_group;
+    uint64_t seed;
+    int iter;
+    const float* sv_amount;
+    int* task_list;
+    int* task_count;
+};
+
+// kernels / launchers (sysmatrix.cu, icd.cu, sched.cu, aux.cu)
+cudaError_t set_prior_constants(const PriorConst& pc);
+cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, int side, int nsvx,
+                            int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxoff,
+                            cudaStream_t st);
+int icd_smem_bytes(const IcdParams& p, int vpt, int nnb);
+cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid_x, int grid_y,
+                       cudaStream_t st);
+cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st);
+cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cudaStream_t st);
+cudaError_t launch_probe(const IcdParams& p, bool quantize, int nnb, const int64_t* vox, int n,
+                         float* out3, cudaStream_t st);
+cudaError_t launch_select(const SchedParams& sp, cudaStream_t st);
+cudaError_t launch_rmse_partial(const float* x, const float* g, int64_t n, double* acc,
+                                cudaStream_t st);
+cudaError_t launch_check_finite(const float* a, int64_t n, int nonneg, int* flag, cudaStream_t st);
+cudaError_t launch_export_sysmatrix(const DevA& A, int nx, int ny, int side, int nsvx,
+                                    const int64_t* vox, int nvox, int32_t* first, int32_t* count,
+                                    float* vals, uint8_t* codes, float* scales,
+                                    const mbir_geometry& g, const double* d_angles_cs,
+                                    cudaStream_t st);
+
+}  // namespace mbir

@@ -1,0 +1,158 @@
+// Device-side SuperVoxel scheduler and small reduction kernels.
+//
+// Paper, Alg. 3 lines 17-23: iteration 1 updates all SVs; even iterations the
+// top 25 % by "update amount"; odd iterations a random 25 % (P:225 raises PSV-ICD's 20 % to 25 %
+// for GPU load balance); the chosen set is split into 4 checkerboard groups whose members share
+// no boundary (Fig. 3).  Reading R14: the update amount is sum |delta| of the SV's
+// most recent visit, the selection is made per slice, ties go to the lower SV index, and the
+// random subset is uniform without replacement from a counter-based hash of
+// (seed, iteration, slice, SV).
+//
+// One CTA per slice: keys in shared memory -> bitonic sort -> the first nsel keys are the
+// selection, in key order -> a block-wide scan of 4 packed 16-bit colour counters places every
+// selected SV into its colour's task list (order preserved).
+#include "mbir_internal.h"
+
+namespace mbir {
+
+namespace {
+
+__device__ __forceinline__ uint64_t mix64s(uint64_t z)
+{
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+constexpr int kSelThreads = 1024;
+
+__global__ void __launch_bounds__(kSelThreads) k_select(const SchedParams S)
+{
+    extern __shared__ unsigned long long keys[];  // [nsv_pad]
+    __shared__ unsigned long long wscan[kSelThreads / 32];
+    const int z = blockIdx.x, zg = S.z_offset + z;
+    const int n = S.nsv_pad;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        unsigned long long key = ~0ull;
+        if (i < S.nsv) {
+            if (S.mode == 1) {
+                const float a = S.sv_amount[(size_t)z * S.nsv + i];
+                const uint32_t bits = __float_as_uint(fmaxf(a, 0.f));
+                key = ((unsigned long long)(~bits) << 32) | (unsigned)i;  // larger amount first
+            } else if (S.mode == 3) {
+                key = (unsigned long long)i;
+            } else {
+                const uint64_t h = mix64s(S.seed ^ 0x5bd1e995ULL ^
+                                          mix64s(((uint64_t)S.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)i));
+                key = ((unsigned long long)(uint32_t)(h >> 32) << 32) | (unsigned)i;
+            }
+        }
+        keys[i] = key;
+    }
+    __syncthreads();
+    if (S.mode != 3) {
+        for (int k = 2; k <= n; k <<= 1)
+            for (int j = k >> 1; j > 0; j >>= 1) {
+                for (int i = threadIdx.x; i < n; i += blockDim.x) {
+                    const int ixj = i ^ j;
+                    if (ixj > i) {
+                        const bool up = (i & k) == 0;
+                        const unsigned long long a = keys[i], b = keys[ixj];
+                        if ((a > b) == up) {
+                            keys[i] = b;
+                            keys[ixj] = a;
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+    }
+    // colour of each selected SV, 4 x 16-bit counters packed in a uint64
+    const int nsel = S.nsel;
+    const int per = (nsel + blockDim.x - 1) / blockDim.x;
+    const int b0 = threadIdx.x * per, b1 = min(nsel, b0 + per);
+    unsigned long long local = 0;
+    for (int q = b0; q < b1; ++q) {
+        const int s = (int)(keys[q] & 0xffffffffu);
+        const int col = ((s % S.nsvx) & 1) + 2 * ((s / S.nsvx) & 1);
+        local += 1ull << (16 * col);
+    }
+    // block exclusive scan of `local`
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    unsigned long long incl = local;
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    if (lane == 31) wscan[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+        unsigned long long v = lane < (int)(blockDim.x >> 5) ? wscan[lane] : 0ull;
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long t = __shfl_up_sync(0xffffffffu, v, o);
+            if (lane >= o) v += t;
+        }
+        wscan[lane] = v;  // inclusive over warps
+    }
+    __syncthreads();
+    unsigned long long excl = incl - local + (wid > 0 ? wscan[wid - 1] : 0ull);
+    const unsigned long long total = wscan[(blockDim.x >> 5) - 1];
+    for (int q = b0; q < b1; ++q) {
+        const int s = (int)(keys[q] & 0xffffffffu);
+        const int col = ((s % S.nsvx) & 1) + 2 * ((s / S.nsvx) & 1);
+        const int p = (int)((excl >> (16 * col)) & 0xffffu);
+        S.task_list[((size_t)z * 4 + col) * S.max_group + p] = s;
+        excl += 1ull << (16 * col);
+    }
+    if (threadIdx.x < 4) S.task_count[z * 4 + threadIdx.x] = (int)((total >> (16 * threadIdx.x)) & 0xffffu);
+}
+
+__global__ void k_rmse(const float* __restrict__ x, const float* __restrict__ g, int64_t n,
+                       double* acc)
+{
+    double s = 0.0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const double d = (double)x[i] - (double)g[i];
+        s += d * d;
+    }
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if ((threadIdx.x & 31) == 0) atomicAdd(acc, s);
+}
+
+__global__ void k_finite(const float* __restrict__ a, int64_t n, int nonneg, int* flag)
+{
+    int bad = 0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const float v = a[i];
+        if (!isfinite(v) || (nonneg && v < 0.f)) bad = 1;
+    }
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(flag, 1);
+}
+
+}  // namespace
+
+cudaError_t launch_select(const SchedParams& sp, cudaStream_t st)
+{
+    const int smem = sp.nsv_pad * 8;
+    cudaError_t e = cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    k_select<<<sp.nz_local, kSelThreads, smem, st>>>(sp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_rmse_partial(const float* x, const float* g, int64_t n, double* acc,
+                                cudaStream_t st)
+{
+    k_rmse<<<296, 256, 0, st>>>(x, g, n, acc);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_check_finite(const float* a, int64_t n, int nonneg, int* flag, cudaStream_t st)
+{
+    k_finite<<<296, 256, 0, st>>>(a, n, nonneg, flag);
+    return cudaGetLastError();
+}
+
+}  // namespace mbir
