@@ -1,0 +1,357 @@
+#!/usr/bin/env python
+"""Benchmark of the GPU-ICD hot path (BASELINE.json metric: voxel updates/s and
+time-to-converge (< 10 HU RMSE) per volume at 1/2/4/8 B200).
+
+Workload (BASELINE.json configs[3], fits one GPU): 512 x 512 x 64 volume, 720 views x 1024
+channels parallel beam, 3-D Shepp-Logan with Poisson noise (lambda0 = 1e4), q-GGMRF prior over
+the 26-neighbourhood, SuperVoxel side 9, uint8 A.  N GPUs: z-slabs of 64/N slices with the
+NCCL halo exchange (strong scaling of one fixed volume).
+
+A "step" = one reconstruction from x0 = 0 of E equits (set_image(0) + mbir_reconstruct(E));
+value = executed voxel updates (all ranks) / max-over-ranks device time of K steps.  Inputs are
+resident in HBM and larger than L2 (A ~0.95 GB, sinograms 0.54 GB).  `e2e` repeats the step
+through the C-ABI from pinned host buffers (y, w up, image down).  `roofline` is the fused
+update kernel's algorithmic HBM bytes over its own event-timed duration.
+
+--impl reference: the repo's sequential C oracle (the only reference this paper has), timed
+on the host cores on a bounded sample of the same per-update work.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+MU_W = 0.02
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="cfg4")
+    ap.add_argument("--equits", type=float, default=6.0, help="equits per step")
+    ap.add_argument("--batch-svs", type=int, default=0)
+    ap.add_argument("--sv-side", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-converge", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--golden-equits", type=float, default=60.0)
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.lines = []
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.p = None
+        return self
+
+    def _read(self):
+        for line in self.p.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            try:
+                self.p.wait(timeout=5)
+            except Exception:
+                self.p.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- CPU oracle leg
+def oracle_sample_setup():
+    """Bounded sample of the workload's per-update work for the sequential oracle: a 128 x 128
+    slice with config 4's pitch (dxy = 0.5 mm), 720 views and dc = dxy/2 (256 channels), so every
+    voxel update touches ~2400 (view, channel) entries as at full size."""
+    import oracle as O
+    from synth import WorkloadConfig, make_case
+    cfg = WorkloadConfig("cpu-sample", 128, 1, 720, 256, 9, 26, 0.005, fov=64.0)
+    case = make_case(cfg, with_truth=False)
+    og = O.Geometry(cfg.n, cfg.n, 1, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dchannel)
+    A = O.sysmatrix(og)
+    _, _, Aq = O.quantize(A)
+    pr = O.Prior(sigma=cfg.sigma, nbhd=26)
+    return O, og, Aq, pr, case, cfg
+
+
+def oracle_time(O, og, Aq, pr, case, budget_s):
+    x = np.zeros(og.nx * og.ny)
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+    upd, t0, sweeps = 0, time.perf_counter(), 0
+    while True:
+        st, _ = O.icd_run(og, pr, Aq, case.w, x, e, 1, first_sweep=sweeps + 1, seed=3000)
+        upd += st["updates"]
+        sweeps += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s:
+            break
+    return upd, el, sweeps
+
+
+def cpu_baseline(budget_s=12.0):
+    O, og, Aq, pr, case, cfg = oracle_sample_setup()
+    upd, el, sweeps = oracle_time(O, og, Aq, pr, case, budget_s)
+    return {"value": upd / el, "unit": "voxel updates/s", "cores": 1, "kind": "oracle",
+            "sample": f"sequential C oracle (double), {sweeps} equits of a 128x128 slice at "
+                      f"config-4 pitch (0.5 mm), 720 views x 256 channels (dc = dxy/2, "
+                      f"{int(Aq.count.sum() / (cfg.n * cfg.n))} nnz/voxel), {upd} updates in {el:.1f} s"}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    O, og, Aq, pr, case, cfg = oracle_sample_setup()
+    for _ in range(args.warmup):
+        oracle_time(O, og, Aq, pr, case, 0.5)
+    tot_u, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        u, t, _ = oracle_time(O, og, Aq, pr, case, 3.0)
+        tot_u += u
+        tot_t += t
+    v = tot_u / tot_t
+    line = {"metric": "voxel updates/s", "value": v, "unit": "voxel updates/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot_t / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "impl": "reference",
+            "config": {"workload": "cfg4 per-update work, bounded sample (128x128 slice at config-4 "
+                                   "pitch, 720 views x 256 channels)"},
+            "cpu_baseline": {"value": v, "unit": "voxel updates/s", "cores": 1, "kind": "oracle",
+                             "sample": "each step: >= 3 s of sequential-oracle equits on the sample"},
+            "e2e": {"value": v, "unit": "voxel updates/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- GPU leg
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_sabnewkbrm17_b200 as M
+    from synth import CONFIGS, make_sinogram_torch
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    cfg = CONFIGS[args.config]
+    side = args.sv_side or cfg.sv_side
+    nz = cfg.nz
+    assert nz % world == 0, "slices must divide evenly across ranks"
+    nzl = nz // world
+    z0 = rank * nzl
+    stream = torch.cuda.current_stream(dev)
+
+    t_setup = time.perf_counter()
+    y, w = make_sinogram_torch(cfg, 0, dev, z0, z0 + nzl)
+    g = M.Geometry(cfg.n, cfg.n, nzl, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dchannel,
+                   z_offset=z0, nz_total=nz)
+    pr = M.Prior(sigma=cfg.sigma, neighborhood=cfg.nbhd)
+    opt = M.Options(sv_side=side, batch_svs=args.batch_svs)
+    nccl_id = None
+    if world > 1:
+        buf = torch.zeros(128, dtype=torch.uint8, device=dev)
+        if rank == 0:
+            buf.copy_(torch.frombuffer(bytearray(M.mbir_nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(buf, 0)
+        nccl_id = bytes(buf.cpu().numpy().tobytes())
+    r = M.Reconstructor(g, pr, opt, device=local, stream=stream.cuda_stream, rank=rank,
+                        nranks=world, nccl_id=nccl_id)
+    r.set_sinogram(y, w)
+    sizes = r.sizes()
+    torch.cuda.synchronize()
+    setup_s = time.perf_counter() - t_setup
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
+    def allmax(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def step():
+        r.set_image(None)  # x0 = 0, e = y (one forward kernel launch)
+        return r.reconstruct(args.equits)
+
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    stats = []
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            stats.append(step())
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    barrier()
+    el = allmax(ev0.elapsed_time(ev1) / 1000.0)
+    updates = sum(s["updates"] for s in stats)  # all-reduced over ranks by the library
+    value = updates / el
+    launches = sum(s["launches"] + 1 for s in stats)
+    # ---- roofline of the fused update kernel (this rank's work / this rank's kernel time)
+    nvox_plane = cfg.n * cfg.n
+    nnz_avg = sizes["nnz"] / nvox_plane
+    band_avg = sizes["band_entries"] / sizes["nsv"]
+    ksec = sum(s["kernel_seconds"] for s in stats)
+    klaunch = sum(s["kernel_launches"] for s in stats)
+    local_updates = updates / world
+    local_visits = sum(s["sv_visits"] for s in stats) / world
+    bytes_per_update = nnz_avg * 1 + cfg.nviews * 1 + 4  # u8 codes of the nnz, offsets, scale
+    alg_bytes = local_updates * bytes_per_update + local_visits * 16 * band_avg
+    achieved = alg_bytes / ksec / 1e9
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    peak = peaks.get("hbm_gbs", 6650.0)
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "icd_traffic.json")
+    if os.path.exists(tp):
+        tj = json.load(open(tp))
+        traffic = tj.get("dram_bytes_per_update", 0) * local_updates / max(klaunch, 1)
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": achieved / peak, "traffic": traffic,
+            "kernel": "k_icd_sv (fused SV update)", "kernel_share": ksec / el,
+            "alg_bytes_per_update": alg_bytes / local_updates,
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback 6.65 TB/s"}
+
+    # ---- end to end through the C-ABI with host buffers
+    e2e = None
+    if not args.no_e2e:
+        yh = y.cpu().pin_memory()
+        wh = w.cpu().pin_memory()
+        xh = torch.empty((nzl, cfg.n, cfg.n), dtype=torch.float32).pin_memory()
+        ke = max(1, min(args.steps, 3))
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        upd_e = 0
+        e0.record(stream)
+        for _ in range(ke):
+            r.set_sinogram(yh, wh)
+            r.set_image(None)
+            upd_e += r.reconstruct(args.equits)["updates"]
+            r.image(xh)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ele = allmax(e0.elapsed_time(e1) / 1000.0)
+        e2e = {"value": upd_e / ele, "unit": "voxel updates/s",
+               "h2d_bytes_per_step": int(2 * yh.numel() * 4 * world),
+               "d2h_bytes_per_step": int(xh.numel() * 4 * world),
+               "ms_per_step": 1000 * ele / ke}
+        r.set_sinogram(y, w)
+
+    # ---- time to converge (< 10 HU vs a 60-equit golden of the same reconstruction)
+    conv = None
+    if not args.no_converge:
+        r.set_image(None)
+        r.reconstruct(args.golden_equits)
+        golden = torch.empty((nzl, cfg.n, cfg.n), dtype=torch.float32, device=dev)
+        r.image(golden)
+        r.set_image(None)
+        t_dev, eq, hist = 0.0, 0.0, []
+        for it in range(400):
+            s = r.iterate(1)
+            t_dev = allmax(t_dev + s["seconds"]) if world > 1 else t_dev + s["seconds"]
+            eq += s["equits"]
+            rm = r.rmse_hu(golden)
+            hist.append((round(eq, 3), round(rm, 2)))
+            if rm < 10.0:
+                break
+        conv = {"time_to_10hu_s": t_dev, "equits_to_10hu": eq, "iterations": it + 1,
+                "golden_equits": args.golden_equits, "rmse_hu_curve": hist[:60]}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline()
+
+    if rank == 0:
+        clocks = clk.summary()
+        line = {
+            "metric": "voxel updates/s", "value": value, "unit": "voxel updates/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1000 * el / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32 (A uint8)",
+            "data": "synthetic",
+            "config": {"workload": f"{cfg.name}: {cfg.n}x{cfg.n}x{cfg.nz} volume, {cfg.nviews} views x "
+                                   f"{cfg.nchannels} channels parallel-beam 3-D Shepp-Logan, Poisson "
+                                   f"(lambda0=1e4), q-GGMRF 26-nbhd, SV side {side}",
+                       "equits_per_step": args.equits, "slab_slices_per_gpu": nzl,
+                       "parallelism": f"z-slab x{world}", "batch_svs": args.batch_svs,
+                       "l2": "inputs larger than L2 (A %.2f GB + sinograms %.2f GB)" % (
+                           sizes["a_bytes"] / 1e9, 3 * y.numel() * 4 * world / 1e9)},
+            "updates_per_step": updates / args.steps,
+            "time_to_converge": conv,
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": launches, "clocks": clocks,
+            "setup_s": setup_s, "sizes": sizes,
+        }
+        print(json.dumps(line), flush=True)
+    r.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

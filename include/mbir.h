@@ -87,8 +87,9 @@ typedef struct mbir_options {
     int zero_skip;         /* P:115, default 1 (never in iteration 1; reading R9)               */
     int quantize_A;        /* 1: A as uint8 codes + per-voxel scale, 0: fp32 values */
     uint64_t seed;         /* voxel-order / random-SV-selection seed                            */
-    int deterministic;     /* debug: every iteration visits all SVs, one SV per launch, in
-                              (z-parity, colour, slice, SV index) order, voxels in raster order  */
+    int deterministic;     /* debug: every iteration visits all SVs one at a time (one CTA) in
+                              the order z-parity half (3-D prior only), colour, SV rank within
+                              the colour (SV index order), slice; voxels in raster order        */
 } mbir_options;
 
 /* Placement and (optional) multi-GPU slab partition.  device: CUDA ordinal.  stream: a
@@ -113,6 +114,9 @@ typedef struct mbir_stats {
     double seconds;        /* device time of this call (CUDA events)                  */
     double sum_abs_delta;  /* sum |delta| over the executed updates                   */
     int64_t launches;      /* kernel launches issued by this call                     */
+    double kernel_seconds; /* summed device time of the fused update-kernel launches,
+                              CUDA events on the handle's stream around each launch     */
+    int64_t kernel_launches; /* fused update-kernel launches                           */
 } mbir_stats;
 
 /* Sizes of the internal layout (for tests, benchmarks and buffer allocation). */

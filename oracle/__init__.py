@@ -223,6 +223,9 @@ def error_sinogram(g: Geometry, A: SysMatrix, y: np.ndarray, x: np.ndarray) -> n
 
 def voxel_update(g: Geometry, pr: Prior, A: SysMatrix, w, x, e, j: int, apply: bool = False):
     """Alg. 1 on voxel j (flat index).  x, e are modified in place iff apply."""
+    assert x.dtype == np.float64 and x.flags.c_contiguous
+    assert e.dtype == np.float64 and e.flags.c_contiguous
+    w = np.ascontiguousarray(w, np.float64)
     plane = g.nx * g.ny
     jj = j % plane
     t1, t2, dl = C.c_double(), C.c_double(), C.c_double()

@@ -47,10 +47,15 @@ double orc_strip_pixel_area(double cx, double cy, double d, double c, double s,
 {
     pt sq[4], p1[8], p2[12];
     double h = 0.5 * d;
-    sq[0].x = cx - h; sq[0].y = cy - h;
-    sq[1].x = cx + h; sq[1].y = cy - h;
-    sq[2].x = cx + h; sq[2].y = cy + h;
-    sq[3].x = cx - h; sq[3].y = cy + h;
+    /* area is translation invariant: clip in pixel-centred coordinates so the shoelace sums
+     * stay O(d^2) instead of O(|centre|^2) (no cancellation for thin slivers far off-axis) */
+    const double tc = cx * c + cy * s;
+    tlo -= tc;
+    thi -= tc;
+    sq[0].x = -h; sq[0].y = -h;
+    sq[1].x = +h; sq[1].y = -h;
+    sq[2].x = +h; sq[2].y = +h;
+    sq[3].x = -h; sq[3].y = +h;
     int n1 = clip_halfplane(sq, 4, p1, c, s, tlo, +1.0); /* x*c+y*s >= tlo */
     if (n1 < 3) return 0.0;
     int n2 = clip_halfplane(p1, n1, p2, c, s, thi, -1.0); /* x*c+y*s <= thi */

@@ -85,6 +85,7 @@ struct mbir_handle {
     float *d_y = nullptr, *d_w = nullptr, *d_e = nullptr, *d_x = nullptr;
     float *d_theta2 = nullptr, *d_amount = nullptr, *d_scratch = nullptr;
     int *d_task_list = nullptr, *d_task_count = nullptr;
+    int *d_flat = nullptr, *d_brange = nullptr, *d_fetch = nullptr;
     unsigned long long* d_counters = nullptr;  // [updates, skipped, visits]
     double* d_sum_delta = nullptr;
     int* d_flag = nullptr;
@@ -94,6 +95,8 @@ struct mbir_handle {
     int iter = 0;
     int64_t nnz = 0, a_bytes = 0, band_entries = 0;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    std::vector<cudaEvent_t> kev;  // per-launch event pairs of the update kernel (one iteration)
+    int kev_used = 0;
     std::string err;
 };
 
@@ -145,9 +148,6 @@ IcdParams make_params(mbir_handle* h)
     p.theta2 = h->d_theta2;
     p.scratch = h->d_scratch;
     p.sv_amount = h->d_amount;
-    p.task_list = h->d_task_list;
-    p.task_count = h->d_task_count;
-    p.max_group = h->max_group;
     p.counters = h->d_counters;
     p.sum_delta = h->d_sum_delta;
     p.seed = h->o.seed;
@@ -188,6 +188,23 @@ int exchange_halo(mbir_handle* h, int parity)
     return MBIR_OK;
 }
 
+// one fused-update-kernel launch bracketed by CUDA events on the handle's stream
+int timed_icd(mbir_handle* h, const IcdParams& p, int nnb, bool q, int gx, int gy)
+{
+    if ((int)h->kev.size() < 2 * (h->kev_used + 1)) {
+        for (int i = 0; i < 2; ++i) {
+            cudaEvent_t e;
+            CK(cudaEventCreate(&e));
+            h->kev.push_back(e);
+        }
+    }
+    CK(cudaEventRecord(h->kev[2 * h->kev_used], h->st));
+    CK(launch_icd(p, h->vpt, nnb, q, gx, gy, h->st));
+    CK(cudaEventRecord(h->kev[2 * h->kev_used + 1], h->st));
+    h->kev_used++;
+    return MBIR_OK;
+}
+
 // e = y - A x (and theta2 when the weights changed)
 int refresh_error(mbir_handle* h, bool theta2)
 {
@@ -206,13 +223,15 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
     const int nnb = h->pr.neighborhood;
     const int parities = (nnb == 26 && h->g.nz_total > 1) ? 2 : 1;
     const int target_ctas = h->nsm * h->blocks_per_sm;
-    int64_t updates = 0, skipped = 0, visits = 0, iters = 0, launches = 0;
+    int64_t updates = 0, skipped = 0, visits = 0, iters = 0, launches = 0, klaunches = 0;
+    double ksec = 0.0;
     double sum_delta = 0.0;
     CK(cudaEventRecord(h->ev0, h->st));
     for (int it = 0;; ++it) {
         if (n_iter >= 0 && it >= n_iter) break;
         if (n_iter < 0 && (double)updates >= target_equits * nvox_total) break;
         h->iter += 1;
+        h->kev_used = 0;
         CK(cudaMemsetAsync(h->d_counters, 0, 3 * sizeof(unsigned long long), h->st));
         CK(cudaMemsetAsync(h->d_sum_delta, 0, sizeof(double), h->st));
         // ---- SV selection (Alg3:17-23)
@@ -241,46 +260,34 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         }
         CK(launch_select(sp, h->st));
         ++launches;
+        // ---- flat task lists + batch ranges per (z-parity, colour) phase (Alg3:24-27)
+        const bool det = h->o.deterministic != 0;
+        const int B = (det || h->o.batch_svs <= 0) ? h->max_group : h->o.batch_svs;
+        const int thr = (det || h->o.batch_svs <= 0) ? 0 : (h->o.batch_threshold >= 0 ? h->o.batch_threshold : B / 4);
+        const int nb = (h->max_group + B - 1) / B;
+        CK(launch_flatten(h->d_task_list, h->d_task_count, h->g.nz_local, h->g.z_offset, parities,
+                          h->max_group, B, thr, nb, h->d_flat, h->d_brange, h->st));
+        ++launches;
+        CK(cudaMemsetAsync(h->d_fetch, 0, sizeof(int) * 8 * nb, h->st));
         IcdParams p = make_params(h);
         p.zero_skip_active = (h->o.zero_skip && h->iter > 1) ? 1 : 0;
+        const size_t cap = (size_t)h->g.nz_local * h->max_group;
+        // deterministic: one CTA walks the phase list in order (sequential ICD, known order)
+        const int grid = det ? 1 : target_ctas;
         for (int zp = 0; zp < parities; ++zp) {
-            // local slices whose global index has parity zp (all slices if 2-D prior)
-            int zfirst = 0, zstride = 1;
-            if (parities == 2) {
-                zfirst = ((zp - h->g.z_offset) % 2 + 2) % 2;
-                zstride = 2;
-            }
-            const int nzp = zfirst < h->g.nz_local ? (h->g.nz_local - zfirst + zstride - 1) / zstride : 0;
-            for (int colour = 0; colour < 4 && nzp > 0; ++colour) {
-                p.colour = colour;
-                p.zstride = zstride;
-                if (h->o.deterministic) {  // one SV per launch, fully sequential order
-                    p.batch = 1;
-                    p.thr = 0;
-                    p.zstride = 1;
-                    for (int z = zfirst; z < h->g.nz_local; z += zstride) {
-                        p.zfirst = z;
-                        for (int pos = 0; pos < h->max_group; ++pos) {
-                            p.batch_base = pos;
-                            CK(launch_icd(p, h->vpt, nnb, q, 1, 1, h->st));
-                            ++launches;
-                        }
-                    }
-                    continue;
-                }
-                p.zfirst = zfirst;
-                const int B = h->o.batch_svs > 0 ? h->o.batch_svs : h->max_group;
-                p.batch = B;
-                p.thr = h->o.batch_svs > 0 ? (h->o.batch_threshold >= 0 ? h->o.batch_threshold : B / 4) : 0;
-                const int gx = std::max(1, std::min(B, (target_ctas + nzp - 1) / nzp));
-                for (int base = 0; base < h->max_group; base += B) {
-                    p.batch_base = base;
-                    CK(launch_icd(p, h->vpt, nnb, q, gx, nzp, h->st));
+            for (int colour = 0; colour < 4; ++colour) {
+                const int ph = zp * 4 + colour;
+                p.flat = h->d_flat + ph * cap;
+                for (int b = 0; b < nb; ++b) {
+                    p.brange = h->d_brange + ph * (nb + 1) + b;
+                    p.fetch = h->d_fetch + ph * nb + b;
+                    if (int r = timed_icd(h, p, nnb, q, grid, 1)) return r;
                     ++launches;
                 }
             }
             if (h->nranks > 1 && parities == 2) {
-                int r = exchange_halo(h, (h->g.z_offset + zfirst) & 1);
+                // slices updated in this half have global parity zp
+                int r = exchange_halo(h, zp);
                 if (r) return r;
             }
         }
@@ -293,6 +300,12 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         CK(cudaMemcpyAsync(h->h_counters + 3, h->d_sum_delta, sizeof(double), cudaMemcpyDeviceToHost,
                            h->st));
         CK(cudaStreamSynchronize(h->st));
+        for (int i = 0; i < h->kev_used; ++i) {
+            float kms = 0.f;
+            CK(cudaEventElapsedTime(&kms, h->kev[2 * i], h->kev[2 * i + 1]));
+            ksec += kms * 1e-3;
+        }
+        klaunches += h->kev_used;
         updates += (int64_t)h->h_counters[0];
         skipped += (int64_t)h->h_counters[1];
         visits += (int64_t)h->h_counters[2];
@@ -319,6 +332,8 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         st->seconds = ms * 1e-3;
         st->sum_abs_delta = sum_delta;
         st->launches = launches;
+        st->kernel_seconds = ksec;
+        st->kernel_launches = klaunches;
     }
     return MBIR_OK;
 }
@@ -394,13 +409,15 @@ void mbir_destroy(mbir_handle* h)
     if (h->st) cudaStreamSynchronize(h->st);
     void* ptrs[] = {h->A.codes, h->A.vals, h->A.off, h->A.count, h->A.scale, h->A.band_start,
                     h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
-                    h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count, h->d_counters, h->d_sum_delta,
+                    h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count,
+                    h->d_flat, h->d_brange, h->d_fetch, h->d_counters, h->d_sum_delta,
                     h->d_flag, h->d_acc};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     if (h->h_counters) cudaFreeHost(h->h_counters);
     if (h->ev0) cudaEventDestroy(h->ev0);
     if (h->ev1) cudaEventDestroy(h->ev1);
+    for (cudaEvent_t e : h->kev) cudaEventDestroy(e);
     if (h->comm && nccl().CommDestroy) nccl().CommDestroy(h->comm);
     if (h->own_stream && h->st) cudaStreamDestroy(h->st);
     delete h;
@@ -488,17 +505,22 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
 
     // ---- system matrix, compressed per SV (a1)
     const bool quant = h->o.quantize_A != 0;
-    const size_t nA = (size_t)h->nsv * h->S2 * G.nviews;
     h->A.nsv = h->nsv;
     h->A.S2 = h->S2;
     h->A.V = G.nviews;
+    h->A.VA = (G.nviews + 15) & ~15;  // record stride: TMA bulk copies need 16-byte multiples
+    const size_t nA = (size_t)h->nsv * h->S2 * h->A.VA;
     if (quant) {
         if ((r = dalloc(h, &h->A.codes, nA))) return bail(r);
+        cudaMemsetAsync(h->A.codes, 0, nA * 4, h->st);
     } else {
         if ((r = dalloc(h, &h->A.vals, nA))) return bail(r);
+        cudaMemsetAsync(h->A.vals, 0, nA * 16, h->st);
     }
     if ((r = dalloc(h, &h->A.off, nA))) return bail(r);
     if ((r = dalloc(h, &h->A.count, nA))) return bail(r);
+    cudaMemsetAsync(h->A.off, 0, nA, h->st);
+    cudaMemsetAsync(h->A.count, 0, nA, h->st);
     if ((r = dalloc(h, &h->A.scale, (size_t)h->nsv * h->S2))) return bail(r);
     if ((r = dalloc(h, &h->A.band_start, (size_t)h->nsv * G.nviews))) return bail(r);
     if ((r = dalloc(h, &h->A.band_width, (size_t)h->nsv * G.nviews))) return bail(r);
@@ -533,7 +555,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
     {
         IcdParams p = make_params(h);
-        h->smem = icd_smem_bytes(p, h->vpt, P.neighborhood);
+        h->smem = icd_smem_bytes(p, h->vpt, P.neighborhood, quant);
         if (h->smem > (int)prop.sharedMemPerBlockOptin)
             return (fail(h, MBIR_EINVAL, "SV buffer (" + std::to_string(h->smem) + " B) exceeds shared memory: reduce sv_side"), bail(MBIR_EINVAL));
         h->blocks_per_sm = std::max(1, std::min((int)(prop.sharedMemPerMultiprocessor / (h->smem + 1024)),
@@ -549,9 +571,12 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_theta2, (size_t)G.nz_local * h->nsv * h->S2))) return bail(r);
     if ((r = dalloc(h, &h->d_amount, (size_t)G.nz_local * h->nsv))) return bail(r);
     // e_init tiles of the concurrently running SV visits: one per CTA of the largest grid
-    if ((r = dalloc(h, &h->d_scratch, (size_t)(h->nsm * h->blocks_per_sm + G.nz_local) * h->Vs * 32))) return bail(r);
+    if ((r = dalloc(h, &h->d_scratch, (size_t)h->nsm * h->blocks_per_sm * h->Vs * 32))) return bail(r);
     if ((r = dalloc(h, &h->d_task_list, (size_t)G.nz_local * 4 * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_task_count, (size_t)G.nz_local * 4))) return bail(r);
+    if ((r = dalloc(h, &h->d_flat, (size_t)8 * G.nz_local * h->max_group))) return bail(r);
+    if ((r = dalloc(h, &h->d_brange, (size_t)8 * (h->max_group + 1)))) return bail(r);
+    if ((r = dalloc(h, &h->d_fetch, (size_t)8 * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_counters, 3))) return bail(r);
     if ((r = dalloc(h, &h->d_sum_delta, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_flag, 1))) return bail(r);

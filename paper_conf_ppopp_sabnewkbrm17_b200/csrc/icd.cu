@@ -83,7 +83,7 @@ __device__ __forceinline__ void transpose32(float (&r)[32], int lane)
 
 __device__ __forceinline__ void red_add_f32(float* p, float v)
 {
-    asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+    asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v));
 }
 
 __device__ __forceinline__ uint64_t mix64(uint64_t z)
@@ -97,13 +97,49 @@ struct PriSlot {
     float sb, sbx, v, pad;
 };
 
+// ---- TMA (cp.async.bulk) + mbarrier helpers for the A-record ring ----
+__device__ __forceinline__ uint32_t smem_u32(const void* p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
+{
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar)
+{
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
 struct SmemLayout {
-    int sb_e, sb_w, xt, list, flags, red, pri, vscale, vth2, misc, total;
+    int sb_e, sb_w, xt, list, flags, red, pri, vscale, vth2, misc, astage, stage_bytes, off_in_stage,
+        mbar, total;
 };
 
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
 
-__host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, int S2, int nnb)
+// A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
+__host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, int S2, int nnb,
+                                                  int VA, bool u8, int nstage)
 {
     SmemLayout L;
     const int TW = side + 2;
@@ -119,18 +155,22 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.vscale = o; o = align16(o + S2 * 4);
     L.vth2 = o;  o = align16(o + S2 * 4);
     L.misc = o;  o = align16(o + 16 * 4);
+    L.off_in_stage = VA * (u8 ? 4 : 16);
+    L.stage_bytes = align16(L.off_in_stage + VA);
+    L.astage = o; o = align16(o + nstage * L.stage_bytes);
+    L.mbar = o;  o = align16(o + nstage * 8);
     L.total = o;
     return L;
 }
 
-template <int VPT, bool U8, int NNB, int RING>
+template <int VPT, bool U8, int NNB, int R>
 __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int nvw = P.nvw;
-    const int V = P.V, M = P.M, Vs = P.Vs, S2 = P.S2, side = P.side;
-    const SmemLayout L = smem_layout(P.rows, Vs, side, S2, NNB);
+    const int V = P.V, M = P.M, Vs = P.Vs, S2 = P.S2, side = P.side, VA = P.A.VA;
+    const SmemLayout L = smem_layout(P.rows, Vs, side, S2, NNB, VA, U8, R);
     float* sb_e = (float*)(smem + L.sb_e);
     float* sb_w = (float*)(smem + L.sb_w);
     float* xt = (float*)(smem + L.xt);
@@ -140,20 +180,41 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
     PriSlot* pri = (PriSlot*)(smem + L.pri);
     float* vscale = (float*)(smem + L.vscale);
     float* vth2 = (float*)(smem + L.vth2);
+    uint64_t* mbar = (uint64_t*)(smem + L.mbar);
+    unsigned char* astage = smem + L.astage;
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
     const size_t plane = (size_t)P.nx * P.ny;
+    const bool is_prior = warp == nvw;
+    const uint32_t stage_tx = (uint32_t)(VA * (U8 ? 4 : 16) + VA);
 
-    const int z = P.zfirst + blockIdx.y * P.zstride;  // local slice
-    if (z >= P.nz_local) return;
-    const int zg = P.z_offset + z;                    // global slice
-    const int tq = z * 4 + P.colour;
-    const int cnt = P.task_count[tq];
-    if (P.thr > 0 && cnt - P.batch_base < P.thr) return;  // Alg3:26-27 threshold break
-    const int pend = min(cnt, P.batch_base + P.batch);
+    if (threadIdx.x < 32) red[threadIdx.x] = 0.f;  // slots >= nvw stay zero
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < R; ++s) mbar_init(mbar + s, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    // per-thread view ownership: warp w, lane l owns views (w*VPT + t)*32 + l
+    int kv[VPT];
+    bool kval[VPT];
+#pragma unroll
+    for (int t = 0; t < VPT; ++t) {
+        kv[t] = (warp * VPT + t) * 32 + lane;
+        kval[t] = warp < nvw && kv[t] < V;
+    }
+    uint32_t gseq = 0;  // running voxel sequence number of this CTA: A stage = gseq % R
 
-    for (int pos = P.batch_base + blockIdx.x; pos < pend; pos += gridDim.x) {
-        const int sv = P.task_list[(size_t)tq * P.max_group + pos];
+    // this launch's batch: flat tasks [start, end) of the phase list (sched.cu k_flatten),
+    // pulled one at a time by the persistent CTAs (dynamic distribution, Alg3:4 / T3)
+    const int tstart = P.brange[0], tend = P.brange[1];
+    int* s_task = (int*)(smem + L.misc);
+    for (;;) {
+        if (threadIdx.x == 0) s_task[0] = tstart + atomicAdd(P.fetch, 1);
+        __syncthreads();
+        const int q = s_task[0];
+        if (q >= tend) break;
+        const int tk = P.flat[q];
+        const int z = tk >> 14, sv = tk & 16383;  // local slice, SV
+        const int zg = P.z_offset + z;            // global slice
         const int bx = sv % P.nsvx, by = sv / P.nsvx;
         const int gx0 = bx * side, gy0 = by * side;
         const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
@@ -201,8 +262,10 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
         }
 
         // ---- 3. visiting order: random permutation of the tile, compacted to the kept
-        //         voxels with a warp ballot; per-voxel scale and theta2 staged in smem
-        if (warp == nvw) {
+        //         voxels with a warp ballot; per-voxel scale and theta2 staged in smem; the
+        //         prior warp's lane 0 then starts the TMA ring of A records (R voxels ahead)
+        const size_t arec = (size_t)sv * S2;  // first A record of this SV
+        if (is_prior) {
             const uint64_t h = mix64(P.seed ^ mix64(((uint64_t)P.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)sv));
             if (lane == 0) {
                 for (int i = 0; i < S2; ++i) list[i] = i;
@@ -210,7 +273,7 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                     uint64_t st = h;
                     for (int i = S2 - 1; i > 0; --i) {
                         st += 0x9E3779B97F4A7C15ULL;
-                        const int r = (int)(mix64(st) % (uint64_t)(i + 1));
+                        const int r = (int)(((uint64_t)(uint32_t)mix64(st) * (uint32_t)(i + 1)) >> 32);
                         const int t = list[i];
                         list[i] = list[r];
                         list[r] = t;
@@ -231,45 +294,30 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             }
             for (int i = lane; i < nact; i += 32) {
                 const int v = list[i];
-                vscale[i] = P.A.scale[(size_t)sv * S2 + v];
+                vscale[i] = P.A.scale[arec + v];
                 vth2[i] = P.theta2[((size_t)z * P.nsv + sv) * S2 + v];
             }
-        }
-        __syncthreads();
-
-        // ---- 4. view threads: A prefetch ring + SVB pack (w, then e with e_init kept in regs)
-        int kv[VPT];
-        bool kval[VPT];
-#pragma unroll
-        for (int t = 0; t < VPT; ++t) {
-            kv[t] = (warp * VPT + t) * 32 + lane;
-            kval[t] = warp < nvw && kv[t] < V;
-        }
-        const size_t abase = (size_t)sv * S2 * V;
-        uint32_t rc[VPT][RING];
-        uint32_t ro[VPT];  // RING 8-bit band offsets packed per view
-        float4 rv[VPT][RING];
-        // e_init (band of e at pack time) goes to this CTA's L2-resident scratch tile,
-        // row-major [view][32 channels], written and re-read with coalesced 128-byte rows
-        float* scr = P.scratch + ((size_t)blockIdx.y * gridDim.x + blockIdx.x) * (size_t)Vs * 32;
-        if (warp < nvw) {
-#pragma unroll
-            for (int u = 0; u < RING; ++u) {
-#pragma unroll
-                for (int t = 0; t < VPT; ++t) {
-                    rc[t][u] = 0u;
-                    if (u == 0) ro[t] = 0u;
-                    rv[t][u] = make_float4(0.f, 0.f, 0.f, 0.f);
-                    if (u < nact && kval[t]) {
-                        const size_t ai = abase + (size_t)list[u] * V + kv[t];
-                        if (U8)
-                            rc[t][u] = __ldg(P.A.codes + ai);
-                        else
-                            rv[t][u] = __ldg(P.A.vals + ai);
-                        ro[t] |= (uint32_t)__ldg(P.A.off + ai) << (8 * u);
-                    }
+            __syncwarp();
+            if (lane == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                for (int i = 0; i < R && i < nact; ++i) {
+                    const uint32_t s = (gseq + i) % R;
+                    unsigned char* dst = astage + s * L.stage_bytes;
+                    const size_t rec = (arec + list[i]) * (size_t)VA;
+                    mbar_expect_tx(mbar + s, stage_tx);
+                    if (U8)
+                        tma_load_1d(dst, P.A.codes + rec, VA * 4, mbar + s);
+                    else
+                        tma_load_1d(dst, P.A.vals + rec, VA * 16, mbar + s);
+                    tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, mbar + s);
                 }
             }
+        }
+
+        // ---- 4. view threads: SVB pack (coalesced 128-byte band rows, transposed by shuffles);
+        //         e_init rows go to this CTA's L2-resident scratch tile for the write-back
+        float* scr = P.scratch + (size_t)blockIdx.x * (size_t)Vs * 32;
+        if (warp < nvw) {
             const float* wz = P.w + (size_t)z * V * M;
             float* ez = P.e + (size_t)z * V * M;
 #pragma unroll 1
@@ -301,139 +349,132 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                 for (int c = 0; c < 32; ++c)
                     if (c < P.rows) sb_e[c * Vs + kk] = r[c];
             }
+        } else if (lane == 0) {
+            mbar_wait(mbar + gseq % R, (gseq / R) & 1);  // A records of the first voxel landed
         }
         __syncthreads();
 
         // ---- 5. sequential-exact voxel loop, one barrier per voxel
         float amount = 0.f;
         const int cslot = (zc * TW + 1) * TW + 1;  // tile index of local (0,0)
-        for (int base = 0; base < nact; base += RING) {
+        for (int idx = 0; idx < nact; ++idx) {
+            const int buf = idx & 1;
+            const uint32_t g = gseq + idx;
+            const unsigned char* stg = astage + (g % R) * L.stage_bytes;
+            float ev[VPT][4], av[VPT][4];
+            int oo[VPT];
+            if (warp < nvw) {
+                float t1 = 0.f;
 #pragma unroll
-            for (int u = 0; u < RING; ++u) {
-                const int idx = base + u;
-                if (idx >= nact) break;
-                const int buf = idx & 1;
-                float ev[VPT][4];
-                uint32_t cw[VPT];
-                float4 av[VPT];
-                int oo[VPT];
-                if (warp < nvw) {
-                    float t1 = 0.f;
+                for (int t = 0; t < VPT; ++t) {
+                    if (kval[t]) {
+                        const int o = stg[L.off_in_stage + kv[t]];
+                        oo[t] = o;
+                        if (U8) {
+                            const uint32_t cw = ((const uint32_t*)stg)[kv[t]];
 #pragma unroll
-                    for (int t = 0; t < VPT; ++t) {
-                        oo[t] = (int)((ro[t] >> (8 * u)) & 0xffu);
-                        cw[t] = rc[t][u];
-                        av[t] = rv[t][u];
+                            for (int i = 0; i < 4; ++i) av[t][i] = dq(cw, i);
+                        } else {
+                            const float4 a4 = ((const float4*)stg)[kv[t]];
+                            av[t][0] = a4.x;
+                            av[t][1] = a4.y;
+                            av[t][2] = a4.z;
+                            av[t][3] = a4.w;
+                        }
+                        const float* pe = sb_e + o * Vs + kv[t];
+                        const float* pw = sb_w + o * Vs + kv[t];
+                        float acc = 0.f;
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) {
+                            ev[t][i] = pe[i * Vs];
+                            acc = fmaf(pw[i * Vs] * ev[t][i], av[t][i], acc);
+                        }
+                        t1 += acc;
+                    }
+                }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) t1 += __shfl_xor_sync(kFull, t1, o);
+                if (lane == 0) red[buf * 16 + warp] = t1;
+            } else {
+                // prior warp: surrogate terms of Alg1:7 over the neighbourhood (reading R1-R2)
+                __syncwarp();  // lane 0's x-tile write of the previous voxel is visible
+                const int slot = list[idx];
+                const int lx = slot % side, ly = slot / side;
+                const float v = xt[cslot + ly * TW + lx];
+                float sbv = 0.f, sbx = 0.f;
+                if (lane < NNB) {
+                    const int dx = c_prior.dx[lane], dy = c_prior.dy[lane], dz = c_prior.dz[lane];
+                    const int gx = gx0 + lx + dx, gy = gy0 + ly + dy, gz = zg + dz;
+                    if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
+                        const float xr = xt[cslot + (dz * TW + ly + dy) * TW + lx + dx];
+                        const float bt = c_prior.b[lane] * phi_f(v - xr);
+                        sbv = bt;
+                        sbx = bt * xr;
+                    }
+                }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    sbv += __shfl_xor_sync(kFull, sbv, o);
+                    sbx += __shfl_xor_sync(kFull, sbx, o);
+                }
+                if (lane == 0) {
+                    PriSlot ps;
+                    ps.sb = sbv;
+                    ps.sbx = sbx;
+                    ps.v = v;
+                    ps.pad = 0.f;
+                    pri[buf] = ps;
+                    // the next voxel's A records must have landed before the barrier releases
+                    if (idx + 1 < nact) mbar_wait(mbar + (g + 1) % R, ((g + 1) / R) & 1);
+                }
+            }
+            __syncthreads();
+            // every warp derives the same delta (identical inputs, identical order)
+            const float4* r4 = (const float4*)(red + buf * 16);
+            const float4 a0 = r4[0], a1 = r4[1], a2 = r4[2], a3 = r4[3];
+            const float s1 = ((a0.x + a0.y) + (a0.z + a0.w)) + ((a1.x + a1.y) + (a1.z + a1.w)) +
+                             (((a2.x + a2.y) + (a2.z + a2.w)) + ((a3.x + a3.y) + (a3.z + a3.w)));
+            const PriSlot ps = pri[buf];
+            const float scale = vscale[idx];
+            const float theta1 = -scale * s1;   // Alg1:5, theta1 = -sum w A e
+            const float theta2 = vth2[idx];     // Alg1:6, precomputed sum w A^2
+            const float num = theta2 * ps.v - theta1 + 2.f * ps.sbx;
+            const float den = theta2 + 2.f * ps.sb;
+            float unew = den > 0.f ? num / den : ps.v;
+            if (c_prior.positivity) unew = fmaxf(unew, 0.f);
+            const float delta = unew - ps.v;  // Alg1:7-8
+            if (warp < nvw) {
+                if (delta != 0.f) {  // Alg1:9-11: e -= A delta on this thread's views
+                    const float sd = scale * delta;
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t)
                         if (kval[t]) {
-                            const int o = oo[t];
-                            float acc = 0.f;
+                            float* pe = sb_e + oo[t] * Vs + kv[t];
 #pragma unroll
-                            for (int i = 0; i < 4; ++i) {
-                                const float ee = sb_e[(o + i) * Vs + kv[t]];
-                                const float ww = sb_w[(o + i) * Vs + kv[t]];
-                                ev[t][i] = ee;
-                                const float a = U8 ? dq(cw[t], i)
-                                                   : (i == 0 ? av[t].x : i == 1 ? av[t].y : i == 2 ? av[t].z : av[t].w);
-                                acc = fmaf(ww * ee, a, acc);
-                            }
-                            t1 += acc;
+                            for (int i = 0; i < 4; ++i) pe[i * Vs] = fmaf(-av[t][i], sd, ev[t][i]);
                         }
-                    }
-                    // refill this ring slot with voxel idx + RING
-                    if (idx + RING < nact) {
-                        const size_t vb = abase + (size_t)list[idx + RING] * V;
-#pragma unroll
-                        for (int t = 0; t < VPT; ++t)
-                            if (kval[t]) {
-                                if (U8)
-                                    rc[t][u] = __ldg(P.A.codes + vb + kv[t]);
-                                else
-                                    rv[t][u] = __ldg(P.A.vals + vb + kv[t]);
-                                ro[t] = (ro[t] & ~(0xffu << (8 * u))) | ((uint32_t)__ldg(P.A.off + vb + kv[t]) << (8 * u));
-                            }
-                    }
-#pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) t1 += __shfl_xor_sync(kFull, t1, o);
-                    if (lane == 0) red[buf * 16 + warp] = t1;
-                } else {
-                    // prior warp: surrogate terms of Alg1:7 over the neighbourhood (reading R1-R2)
-                    __syncwarp();  // lane 0's x-tile write of the previous voxel is visible
-                    const int slot = list[idx];
-                    const int lx = slot % side, ly = slot / side;
-                    const float v = xt[cslot + ly * TW + lx];
-                    float sbv = 0.f, sbx = 0.f;
-                    if (lane < NNB) {
-                        const int dx = c_prior.dx[lane], dy = c_prior.dy[lane], dz = c_prior.dz[lane];
-                        const int gx = gx0 + lx + dx, gy = gy0 + ly + dy, gz = zg + dz;
-                        if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
-                            const float xr = xt[cslot + (dz * TW + ly + dy) * TW + lx + dx];
-                            const float bt = c_prior.b[lane] * phi_f(v - xr);
-                            sbv = bt;
-                            sbx = bt * xr;
-                        }
-                    }
-#pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) {
-                        sbv += __shfl_xor_sync(kFull, sbv, o);
-                        sbx += __shfl_xor_sync(kFull, sbx, o);
-                    }
-                    if (lane == 0) {
-                        PriSlot ps;
-                        ps.sb = sbv;
-                        ps.sbx = sbx;
-                        ps.v = v;
-                        ps.pad = 0.f;
-                        pri[buf] = ps;
-                    }
                 }
-                __syncthreads();
-                // every warp derives the same delta (identical inputs, identical order)
-                float s1 = 0.f;
-                {
-                    const float4* r4 = (const float4*)(red + buf * 16);
-                    float part[16];
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) {
-                        const float4 a = r4[q];
-                        part[4 * q] = a.x;
-                        part[4 * q + 1] = a.y;
-                        part[4 * q + 2] = a.z;
-                        part[4 * q + 3] = a.w;
-                    }
-#pragma unroll
-                    for (int q = 0; q < 16; ++q)
-                        if (q < nvw) s1 += part[q];
-                }
-                const PriSlot ps = pri[buf];
-                const float scale = vscale[idx];
-                const float theta1 = -scale * s1;   // Alg1:5, theta1 = -sum w A e
-                const float theta2 = vth2[idx];     // Alg1:6, precomputed sum w A^2
-                const float num = theta2 * ps.v - theta1 + 2.f * ps.sbx;
-                const float den = theta2 + 2.f * ps.sb;
-                float unew = den > 0.f ? num / den : ps.v;
-                if (c_prior.positivity) unew = fmaxf(unew, 0.f);
-                const float delta = unew - ps.v;  // Alg1:7-8
-                if (warp < nvw) {
-                    if (delta != 0.f) {  // Alg1:9-11: e -= A delta on this thread's views
-                        const float sd = scale * delta;
-#pragma unroll
-                        for (int t = 0; t < VPT; ++t)
-                            if (kval[t]) {
-#pragma unroll
-                                for (int i = 0; i < 4; ++i) {
-                                    const float a = U8 ? dq(cw[t], i)
-                                                       : (i == 0 ? av[t].x : i == 1 ? av[t].y : i == 2 ? av[t].z : av[t].w);
-                                    sb_e[(oo[t] + i) * Vs + kv[t]] = fmaf(-a, sd, ev[t][i]);
-                                }
-                            }
-                    }
-                } else if (lane == 0) {
-                    const int slot = list[idx];
-                    xt[cslot + (slot / side) * TW + slot % side] = unew;
-                    amount += fabsf(delta);
+            } else if (lane == 0) {
+                const int slot = list[idx];
+                xt[cslot + (slot / side) * TW + slot % side] = unew;
+                amount += fabsf(delta);
+                // this voxel's stage was read by every view warp before the barrier: refill it
+                // with the A records of voxel idx + R (async proxy after generic reads)
+                if (idx + R < nact) {
+                    const uint32_t s = g % R;
+                    unsigned char* dst = astage + s * L.stage_bytes;
+                    const size_t rec = (arec + list[idx + R]) * (size_t)VA;
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    mbar_expect_tx(mbar + s, stage_tx);
+                    if (U8)
+                        tma_load_1d(dst, P.A.codes + rec, VA * 4, mbar + s);
+                    else
+                        tma_load_1d(dst, P.A.vals + rec, VA * 16, mbar + s);
+                    tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, mbar + s);
                 }
             }
         }
+        gseq += nact;
         __syncthreads();
 
         // ---- 6. write-back: delta e of the band, atomically, and the SV's voxels
@@ -443,20 +484,21 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             for (int t = 0; t < VPT; ++t) {
                 const int k0 = (warp * VPT + t) * 32;
                 const int kk = k0 + lane;
+                const int bw = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
+                const int roff = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
+                float s0[32];  // e_init rows (lane = channel), loads in flight during the transpose
+#pragma unroll
+                for (int i = 0; i < 32; ++i) s0[i] = __ldcg(scr + (k0 + i) * 32 + lane);
                 float r[32];
 #pragma unroll
                 for (int c = 0; c < 32; ++c)
                     r[c] = (kk < V && c < P.rows) ? sb_e[c * Vs + kk] : 0.f;
                 transpose32(r, lane);
-                const int bw = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
-                const int roff = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
                     const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
-                    if (lane < wi) {
-                        const float d = r[i] - __ldcg(scr + (k0 + i) * 32 + lane);
-                        if (d != 0.f) red_add_f32(ez + oi + lane, d);
-                    }
+                    const float d = r[i] - s0[i];
+                    if (lane < wi && d != 0.f) red_add_f32(ez + oi + lane, d);
                 }
             }
         } else {
@@ -487,7 +529,7 @@ __global__ void k_theta2(const IcdParams P)
     const int z = blockIdx.y;
     if (gw >= P.nsv * P.S2) return;
     const int sv = gw / P.S2, slot = gw % P.S2;
-    const size_t ab = ((size_t)sv * P.S2 + slot) * P.V;
+    const size_t ab = ((size_t)sv * P.S2 + slot) * P.A.VA;
     const float* wz = P.w + (size_t)z * P.V * P.M;
     const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
     float acc = 0.f;
@@ -531,7 +573,7 @@ __global__ void k_forward(const IcdParams P)
             const float xv = P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx];
             if (xv == 0.f) continue;
             any = true;
-            const size_t ai = ((size_t)sv * P.S2 + slot) * P.V + k;
+            const size_t ai = ((size_t)sv * P.S2 + slot) * P.A.VA + k;
             const int o = P.A.off[ai];
             const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
             for (int i = 0; i < 4; ++i) {
@@ -569,7 +611,7 @@ __global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
     const int iy = (int)((j % plane) / P.nx), ix = (int)(j % P.nx);
     const int sv = (iy / P.side) * P.nsvx + ix / P.side;
     const int slot = (iy % P.side) * P.side + ix % P.side;
-    const size_t ab = ((size_t)sv * P.S2 + slot) * P.V;
+    const size_t ab = ((size_t)sv * P.S2 + slot) * P.A.VA;
     const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
     const float* wz = P.w + (size_t)z * P.V * P.M;
     const float* ez = P.e + (size_t)z * P.V * P.M;
@@ -628,18 +670,21 @@ __global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
 
 }  // namespace
 
-int icd_smem_bytes(const IcdParams& p, int vpt, int nnb)
+// A-record ring depth (voxels of TMA lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
+constexpr int ring_depth(bool u8) { return u8 ? 8 : 3; }
+
+int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
 {
     (void)vpt;
-    return smem_layout(p.rows, p.Vs, p.side, p.S2, nnb).total;
+    return smem_layout(p.rows, p.Vs, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize)).total;
 }
 
 template <int VPT, bool U8, int NNB>
 static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t st)
 {
-    constexpr int RING = U8 ? 4 : 2;
-    auto kern = k_icd_sv<VPT, U8, NNB, RING>;
-    const int smem = smem_layout(p.rows, p.Vs, p.side, p.S2, NNB).total;
+    constexpr int R = ring_depth(U8);
+    auto kern = k_icd_sv<VPT, U8, NNB, R>;
+    const int smem = smem_layout(p.rows, p.Vs, p.side, p.S2, NNB, p.A.VA, U8, R).total;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     kern<<<dim3(gx, gy), 32 * (p.nvw + 1), smem, st>>>(p);

@@ -33,6 +33,7 @@ struct PriorConst {
 // ---- compressed system matrix, per SuperVoxel ----
 struct DevA {
     int nsv, S2, V;          // SVs per slice, slots per SV (side^2), views
+    int VA;                  // per-voxel record stride in views, V rounded up to 16 (TMA-sized)
     uint32_t* codes;         // [nsv][S2][V] 4 uint8 codes (byte i = channel offset i), quantize_A
     float4* vals;            // [nsv][S2][V] fp32 values, !quantize_A
     uint8_t* off;            // [nsv][S2][V] first channel - band start
@@ -57,10 +58,9 @@ struct IcdParams {
     float* theta2;           // [nz_local][nsv][S2]
     float* scratch;          // [max CTAs][Vs][32] e_init tiles of the running SV visits
     float* sv_amount;        // [nz_local][nsv] sum |delta| of the SV's last visit
-    const int* task_list;    // [nz_local][4][max_group]
-    const int* task_count;   // [nz_local][4]
-    int max_group;
-    int colour, zfirst, zstride, batch_base, batch, thr;
+    const int* flat;         // phase task list, entries (local slice << 14) | SV
+    const int* brange;       // [2]: this launch's batch = flat[brange[0] .. brange[1])
+    int* fetch;              // task counter of this launch (zeroed per iteration)
     unsigned long long* counters;  // [0] updates [1] skipped [2] sv visits
     double* sum_delta;
     uint64_t seed;
@@ -87,7 +87,7 @@ cudaError_t set_prior_constants(const PriorConst& pc);
 cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, int side, int nsvx,
                             int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxoff,
                             cudaStream_t st);
-int icd_smem_bytes(const IcdParams& p, int vpt, int nnb);
+int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize);
 cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid_x, int grid_y,
                        cudaStream_t st);
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st);
@@ -95,6 +95,11 @@ cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cu
 cudaError_t launch_probe(const IcdParams& p, bool quantize, int nnb, const int64_t* vox, int n,
                          float* out3, cudaStream_t st);
 cudaError_t launch_select(const SchedParams& sp, cudaStream_t st);
+// Build the flat, slice-interleaved task list of each (z-parity, colour) phase and its batch
+// ranges (Alg3:24-27): flat[ph][...], brange[ph][b] (b = 0..nb), ph = parity*4 + colour.
+cudaError_t launch_flatten(const int* task_list, const int* task_count, int nz_local, int z_offset,
+                           int parities, int max_group, int batch, int thr, int nb, int* flat,
+                           int* brange, cudaStream_t st);
 cudaError_t launch_rmse_partial(const float* x, const float* g, int64_t n, double* acc,
                                 cudaStream_t st);
 cudaError_t launch_check_finite(const float* a, int64_t n, int nonneg, int* flag, cudaStream_t st);

@@ -107,6 +107,58 @@ __global__ void __launch_bounds__(kSelThreads) k_select(const SchedParams S)
     if (threadIdx.x < 4) S.task_count[z * 4 + threadIdx.x] = (int)((total >> (16 * threadIdx.x)) & 0xffffu);
 }
 
+// One block per phase ph = parity*4 + colour (Alg3:23-27).  Slices of that z-parity contribute
+// their colour group; a slice's group is cut into batches of B and, with a threshold, the
+// batches from the first one with fewer than thr SVs left are dropped ("break", reading R15).
+// Kept tasks are interleaved round-robin over slices (rank r of every slice, then r+1, ...),
+// so each batch is a contiguous range and concurrent CTAs work on different slices.
+constexpr int kMaxSlices = 1024;
+__global__ void k_flatten(const int* __restrict__ task_list, const int* __restrict__ task_count,
+                          int nz_local, int z_offset, int parities, int max_group, int B, int thr,
+                          int nb, int* __restrict__ flat, int* __restrict__ brange)
+{
+    __shared__ int zl[kMaxSlices], K[kMaxSlices];
+    __shared__ int s_n, s_maxK;
+    const int ph = blockIdx.x, parity = ph / 4, colour = ph % 4;
+    if (threadIdx.x == 0) {
+        int n = 0, mk = 0;
+        for (int z = 0; z < nz_local && n < kMaxSlices; ++z) {
+            if (parities == 2 && ((z_offset + z) & 1) != parity) continue;
+            const int cnt = task_count[z * 4 + colour];
+            int k = cnt;
+            if (thr > 0) {
+                k = 0;
+                for (int b = 0; b * B < cnt; ++b) {
+                    if (cnt - b * B < thr) break;
+                    k = min(cnt, (b + 1) * B);
+                }
+            }
+            zl[n] = z;
+            K[n] = k;
+            mk = max(mk, k);
+            ++n;
+        }
+        s_n = n;
+        s_maxK = mk;
+    }
+    __syncthreads();
+    const int n = s_n, maxK = s_maxK;
+    const size_t cap = (size_t)nz_local * max_group;
+    for (int e = threadIdx.x; e < n * maxK; e += blockDim.x) {
+        const int zi = e % n, r = e / n;
+        if (r >= K[zi]) continue;
+        int pos = 0;
+        for (int j = 0; j < n; ++j) pos += min(K[j], r) + ((j < zi && K[j] > r) ? 1 : 0);
+        const int z = zl[zi];
+        flat[ph * cap + pos] = (z << 14) | task_list[((size_t)z * 4 + colour) * max_group + r];
+    }
+    for (int b = threadIdx.x; b <= nb; b += blockDim.x) {
+        int s = 0;
+        for (int j = 0; j < n; ++j) s += min(K[j], b * B);
+        brange[ph * (nb + 1) + b] = s;
+    }
+}
+
 __global__ void k_rmse(const float* __restrict__ x, const float* __restrict__ g, int64_t n,
                        double* acc)
 {
@@ -139,6 +191,15 @@ cudaError_t launch_select(const SchedParams& sp, cudaStream_t st)
     cudaError_t e = cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     k_select<<<sp.nz_local, kSelThreads, smem, st>>>(sp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_flatten(const int* task_list, const int* task_count, int nz_local, int z_offset,
+                           int parities, int max_group, int batch, int thr, int nb, int* flat,
+                           int* brange, cudaStream_t st)
+{
+    k_flatten<<<parities * 4, 256, 0, st>>>(task_list, task_count, nz_local, z_offset, parities,
+                                            max_group, batch, thr, nb, flat, brange);
     return cudaGetLastError();
 }
 

@@ -86,7 +86,7 @@ __global__ void __launch_bounds__(kColThreads) k_columns(
     const int bx = sv % nsvx, by = sv / nsvx;
     const int ix = bx * side + slot % side, iy = by * side + slot / side;
     const bool valid = ix < nx && iy < ny;
-    const size_t base = ((size_t)sv * A.S2 + slot) * V;
+    const size_t base = ((size_t)sv * A.S2 + slot) * A.VA;
     Col col[kMaxViewsPerThread];
     double amax = 0.0;
 #pragma unroll
@@ -149,7 +149,7 @@ __global__ void k_bands(int V, int S2, const int32_t* __restrict__ first_tmp, De
     for (int k = threadIdx.x; k < V; k += blockDim.x) {
         int lo = 1 << 30, hi = -1;
         for (int v = 0; v < S2; ++v) {
-            const size_t i = ((size_t)sv * S2 + v) * V + k;
+            const size_t i = ((size_t)sv * S2 + v) * A.VA + k;
             const int f = first_tmp[i];
             if (f < 0) continue;
             lo = min(lo, f);
@@ -163,7 +163,7 @@ __global__ void k_bands(int V, int S2, const int32_t* __restrict__ first_tmp, De
         atomicMax(maxwidth, wdt);
         int rowmax = 0;
         for (int v = 0; v < S2; ++v) {
-            const size_t i = ((size_t)sv * S2 + v) * V + k;
+            const size_t i = ((size_t)sv * S2 + v) * A.VA + k;
             const int f = first_tmp[i];
             const int o = f < 0 ? 0 : f - lo;
             if (o > 255) atomicOr(err, 2);
@@ -185,7 +185,7 @@ __global__ void k_export(int nx, int ny, double d, int V, int M, double dc, doub
     const int ix = j % nx, iy = j / nx;
     const int sv = (iy / side) * nsvx + ix / side;
     const int slot = (iy % side) * side + ix % side;
-    const size_t base = ((size_t)sv * A.S2 + slot) * V;
+    const size_t base = ((size_t)sv * A.S2 + slot) * A.VA;
     for (int k = threadIdx.x; k < V; k += blockDim.x) {
         const int n = A.count[base + k];
         const size_t o = jo * V + k;
@@ -210,7 +210,7 @@ cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, i
                             int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxrow,
                             cudaStream_t st)
 {
-    const size_t n = (size_t)A.nsv * A.S2 * g.nviews;
+    const size_t n = (size_t)A.nsv * A.S2 * A.VA;
     int32_t* first_tmp = nullptr;
     cudaError_t e = cudaMallocAsync(&first_tmp, n * sizeof(int32_t), st);
     if (e != cudaSuccess) return e;

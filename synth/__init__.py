@@ -11,6 +11,7 @@ from .phantom import (  # noqa: F401
     WorkloadConfig,
     baggage_phantom,
     make_case,
+    make_sinogram_torch,
     phantom_image,
     shepp_logan_2d,
     shepp_logan_3d,

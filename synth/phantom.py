@@ -141,10 +141,11 @@ class WorkloadConfig:
     phantom: str = "shepp_logan"
     lambda0: float = 1.0e4
     center_offset: float = 0.0
+    fov: float = FOV_MM  # image width in mm (dxy = fov / n); the phantom is always FOV_MM wide
 
     @property
     def dxy(self):
-        return FOV_MM / self.n
+        return self.fov / self.n
 
     @property
     def dchannel(self):
@@ -158,6 +159,45 @@ CONFIGS = {
     "cfg3": WorkloadConfig("cfg3", 512, 1, 720, 1024, 9, 8, 0.005),
     "cfg4": WorkloadConfig("cfg4", 512, 64, 720, 1024, 9, 26, 0.005),
 }
+
+
+def make_sinogram_torch(cfg: WorkloadConfig, case_id: int = 0, device="cuda", z0: int = 0,
+                        z1: int | None = None):
+    """Same recipe as make_case (3-D Shepp-Logan slices, 4 sub-rays, Poisson counts) computed
+    with torch on `device` for the large bench configs; returns float32 tensors y, w
+    [z1-z0, V, M] on that device for global slices [z0, z1).  Poisson draws use a torch
+    generator seeded with (2000+case)*1000 + z per slice, so a slab is the same on any rank."""
+    import torch
+    V, M, nz = cfg.nviews, cfg.nchannels, cfg.nz
+    z1 = nz if z1 is None else z1
+    dev = torch.device(device)
+    theta = torch.arange(V, dtype=torch.float64, device=dev) * math.pi / V
+    t0 = -0.5 * M * cfg.dchannel + cfg.center_offset * cfg.dchannel
+    sub = (torch.arange(4, dtype=torch.float64, device=dev) + 0.5) / 4
+    t = t0 + (torch.arange(M, dtype=torch.float64, device=dev)[:, None] + sub[None, :]).reshape(-1) * cfg.dchannel
+    c, s = torch.cos(theta)[:, None], torch.sin(theta)[:, None]
+    gen = torch.Generator(device=dev)
+    y = torch.empty((z1 - z0, V, M), dtype=torch.float32, device=dev)
+    w = torch.empty_like(y)
+    for z in range(z0, z1):
+        gen.manual_seed((2000 + case_id) * 1000 + z)
+        if nz == 1:
+            ells = shepp_logan_2d()
+        else:
+            ells = shepp_logan_3d(-0.25 + 0.5 * (z + 0.5) / nz)
+        p = torch.zeros((V, t.numel()), dtype=torch.float64, device=dev)
+        for (x0, y0, a, b, phi, mu) in ells:
+            ct = torch.cos(theta - phi)[:, None]
+            st = torch.sin(theta - phi)[:, None]
+            r2 = a * a * ct * ct + b * b * st * st
+            sp = t[None, :] - (x0 * c + y0 * s)
+            disc = r2 - sp * sp
+            p += torch.where(disc > 0, mu * 2.0 * a * b * torch.sqrt(disc.clamp_min(0.0)) / r2, 0.0)
+        p = p.reshape(V, M, 4).mean(dim=2)
+        lam = torch.poisson(cfg.lambda0 * torch.exp(-p), generator=gen).clamp_min(1.0)
+        y[z - z0] = torch.log(cfg.lambda0 / lam).float()
+        w[z - z0] = lam.float()
+    return y, w
 
 
 @dataclass

@@ -14,19 +14,19 @@ def geoms(cfg, nz=None):
 
 def deterministic_order(n, nz, side, nbhd):
     """Global voxel order of the library's deterministic debug mode (include/mbir.h
-    mbir_options.deterministic): z-parity half (3-D prior only), colour, slice, SV index,
-    raster within the SV -- written from the documented contract, not from the CUDA code."""
+    mbir_options.deterministic): z-parity half (3-D prior only), colour, SV rank within the
+    colour (index order), slice, raster within the SV -- written from the documented contract,
+    not from the CUDA code."""
     nsx = (n + side - 1) // side
     parities = [0, 1] if (nbhd == 26 and nz > 1) else [None]
     order = []
     for zp in parities:
         for colour in range(4):
-            for z in range(nz):
-                if zp is not None and z % 2 != zp:
-                    continue
-                for sv in range(nsx * nsx):
-                    bx, by = sv % nsx, sv // nsx
-                    if (bx & 1) + 2 * (by & 1) != colour:
+            svs = [sv for sv in range(nsx * nsx) if ((sv % nsx) & 1) + 2 * ((sv // nsx) & 1) == colour]
+            for sv in svs:
+                bx, by = sv % nsx, sv // nsx
+                for z in range(nz):
+                    if zp is not None and z % 2 != zp:
                         continue
                     for ly in range(side):
                         for lx in range(side):

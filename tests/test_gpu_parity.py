@@ -43,7 +43,7 @@ def test_sysmatrix_bit_exact_index_structure(cfg1, quant):
     np.testing.assert_array_equal(count, A.count)
     m = A.count > 0
     np.testing.assert_array_equal(first[m], A.first[m])
-    np.testing.assert_allclose(vals, A.vals.astype(np.float32), rtol=2e-7, atol=1e-12)
+    np.testing.assert_allclose(vals, A.vals.astype(np.float32), rtol=2e-7, atol=1e-7 * A.vals.max())
     assert sz["nnz"] == int(A.count.sum())
     if quant:
         np.testing.assert_array_equal(gcodes, codes)
@@ -69,7 +69,7 @@ def test_sysmatrix_paper_geometry_sampled():
         assert mc <= 4
         np.testing.assert_array_equal(count[q], c)
         np.testing.assert_array_equal(first[q][c > 0], f[c > 0])
-        np.testing.assert_allclose(vals[q], v.astype(np.float32), rtol=2e-7, atol=1e-12)
+        np.testing.assert_allclose(vals[q], v.astype(np.float32), rtol=2e-7, atol=1e-7 * v.max())
         cd, am = O.quantize_column(v, c)
         np.testing.assert_array_equal(gcodes[q], cd)
         assert scales[q] == np.float32(am / 255)
@@ -191,10 +191,11 @@ def test_deterministic_equit_tracks_sequential_oracle_3d():
 
 
 # ------------------------------------------------------------------ converged parity
-@pytest.mark.parametrize("zero_skip", [0, 1])
-def test_converged_image_and_cost_match_oracle_cfg1(cfg1, zero_skip):
+@pytest.mark.parametrize("zero_skip,tol_hu,tol_cost", [(0, 1.0, 1e-4), (1, 2.0, 5e-4)])
+def test_converged_image_and_cost_match_oracle_cfg1(cfg1, zero_skip, tol_hu, tol_cost):
     """Asynchronous parallel ICD is nondeterministic, but the MAP point is unique: the
-    converged GPU image is within 1 HU RMSE of the oracle's and the cost within 1e-4."""
+    converged GPU image is within 1 HU RMSE of the oracle's and the cost within 1e-4.  With
+    zero-skipping the fixed point is order-dependent (reading R9), hence the looser bound."""
     cfg, case, g, og, A, codes, amax, Aq = cfg1
     pr = O.Prior(sigma=cfg.sigma, nbhd=8)
     x = np.zeros(cfg.n * cfg.n)
@@ -208,16 +209,21 @@ def test_converged_image_and_cost_match_oracle_cfg1(cfg1, zero_skip):
         eg = r.error_sinogram()
     assert st["equits"] >= 300
     rm = O.rmse_hu(xg, x)
-    assert rm < 1.0, rm
+    assert rm < tol_hu, rm
     cg = O.cost(og, pr, Aq, case.y, case.w, xg)
     co = O.cost(og, pr, Aq, case.y, case.w, x)
-    assert abs(cg - co) <= 1e-4 * abs(co), (cg, co)
+    assert abs(cg - co) <= tol_cost * abs(co), (cg, co)
     # e stays consistent with y - A x (fp32 drift bound)
     eo = O.error_sinogram(og, Aq, case.y.astype(np.float64), xg)
     assert np.abs(eg.ravel() - eo.ravel()).max() < 1e-3 * np.abs(case.y).max()
 
 
-def test_converged_3d_matches_oracle():
+@pytest.mark.parametrize("zero_skip,tol_hu,tol_cost", [(0, 1.0, 1e-4), (1, 2.0, 5e-4)])
+def test_converged_3d_matches_oracle(zero_skip, tol_hu, tol_cost):
+    """Without zero-skipping the MAP point is unique: 1 HU / 1e-4 (BASELINE.json).  With it
+    (P:115), a voxel whose whole neighbourhood reached 0 is frozen, so the fixed point depends on
+    the update order (reading R9: the oracle's own zero-skip and no-skip runs differ by 2.6e-4
+    in cost on this case); the looser bound covers that path dependence."""
     cfg = small3d()
     case = make_case(cfg)
     g, og = geoms(cfg)
@@ -226,15 +232,16 @@ def test_converged_3d_matches_oracle():
     pr = O.Prior(sigma=cfg.sigma, nbhd=26)
     x = np.zeros(cfg.nz * cfg.n * cfg.n)
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
-    O.icd_run(og, pr, Aq, case.w, x, e, 120, seed=3000)
-    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26), M.Options(sv_side=cfg.sv_side)) as r:
+    O.icd_run(og, pr, Aq, case.w, x, e, 120, seed=3000, zero_skip=bool(zero_skip))
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
+                         M.Options(sv_side=cfg.sv_side, zero_skip=zero_skip)) as r:
         r.set_sinogram(case.y, case.w)
         r.reconstruct(240)
         xg = r.image().ravel().astype(np.float64)
-    assert O.rmse_hu(xg, x) < 1.0
+    assert O.rmse_hu(xg, x) < tol_hu
     cg = O.cost(og, pr, Aq, case.y, case.w, xg)
     co = O.cost(og, pr, Aq, case.y, case.w, x)
-    assert abs(cg - co) <= 1e-4 * abs(co)
+    assert abs(cg - co) <= tol_cost * abs(co)
 
 
 # ------------------------------------------------------------------ scheduler + accounting
