@@ -549,9 +549,9 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     // ---- update-kernel shape
     h->vpt = G.nviews > 384 ? 2 : 1;
     h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
-    if (h->nvw > 15) return (fail(h, MBIR_EINVAL, "too many views"), bail(MBIR_EINVAL));
+    if (h->nvw > 14) return (fail(h, MBIR_EINVAL, "too many views"), bail(MBIR_EINVAL));
     h->Vs = h->nvw * 32 * h->vpt;
-    h->threads = 32 * (h->nvw + 1);
+    h->threads = 32 * (h->nvw + 2);  // view warps + prior warp + TMA producer warp
     if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
     {
         IcdParams p = make_params(h);

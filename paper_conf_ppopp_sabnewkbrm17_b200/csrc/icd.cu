@@ -48,7 +48,7 @@ __device__ __forceinline__ float phi_f(float d)
     else
         u = (ad == 0.f) ? 0.f : exp2f(c_prior.qmp * __log2f(ad * c_prior.inv_Ts));
     const float opu = 1.f + u;
-    return c_prior.c_phi * (c_prior.pq + u) / (opu * opu);
+    return __fdividef(c_prior.c_phi * (c_prior.pq + u), opu * opu);
 }
 
 // uint8 code i of a packed word -> float, via the 2^23 magic (PRMT + FADD, no I2F)
@@ -349,7 +349,7 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                 for (int c = 0; c < 32; ++c)
                     if (c < P.rows) sb_e[c * Vs + kk] = r[c];
             }
-        } else if (lane == 0) {
+        } else if (warp == nvw + 1 && lane == 0) {
             mbar_wait(mbar + gseq % R, (gseq / R) & 1);  // A records of the first voxel landed
         }
         __syncthreads();
@@ -395,7 +395,7 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
 #pragma unroll
                 for (int o = 16; o > 0; o >>= 1) t1 += __shfl_xor_sync(kFull, t1, o);
                 if (lane == 0) red[buf * 16 + warp] = t1;
-            } else {
+            } else if (warp == nvw) {
                 // prior warp: surrogate terms of Alg1:7 over the neighbourhood (reading R1-R2)
                 __syncwarp();  // lane 0's x-tile write of the previous voxel is visible
                 const int slot = list[idx];
@@ -424,9 +424,10 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                     ps.v = v;
                     ps.pad = 0.f;
                     pri[buf] = ps;
-                    // the next voxel's A records must have landed before the barrier releases
-                    if (idx + 1 < nact) mbar_wait(mbar + (g + 1) % R, ((g + 1) / R) & 1);
                 }
+            } else if (lane == 0) {
+                // producer warp: the next voxel's A records must have landed before the barrier
+                if (idx + 1 < nact) mbar_wait(mbar + (g + 1) % R, ((g + 1) / R) & 1);
             }
             __syncthreads();
             // every warp derives the same delta (identical inputs, identical order)
@@ -440,7 +441,7 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             const float theta2 = vth2[idx];     // Alg1:6, precomputed sum w A^2
             const float num = theta2 * ps.v - theta1 + 2.f * ps.sbx;
             const float den = theta2 + 2.f * ps.sb;
-            float unew = den > 0.f ? num / den : ps.v;
+            float unew = den > 0.f ? __fdividef(num, den) : ps.v;
             if (c_prior.positivity) unew = fmaxf(unew, 0.f);
             const float delta = unew - ps.v;  // Alg1:7-8
             if (warp < nvw) {
@@ -454,11 +455,14 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                             for (int i = 0; i < 4; ++i) pe[i * Vs] = fmaf(-av[t][i], sd, ev[t][i]);
                         }
                 }
+            } else if (warp == nvw) {
+                if (lane == 0) {
+                    const int slot = list[idx];
+                    xt[cslot + (slot / side) * TW + slot % side] = unew;
+                    amount += fabsf(delta);
+                }
             } else if (lane == 0) {
-                const int slot = list[idx];
-                xt[cslot + (slot / side) * TW + slot % side] = unew;
-                amount += fabsf(delta);
-                // this voxel's stage was read by every view warp before the barrier: refill it
+                // producer warp.  This voxel's stage was read by every view warp before the barrier: refill it
                 // with the A records of voxel idx + R (async proxy after generic reads)
                 if (idx + R < nact) {
                     const uint32_t s = g % R;
@@ -687,7 +691,7 @@ static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t
     const int smem = smem_layout(p.rows, p.Vs, p.side, p.S2, NNB, p.A.VA, U8, R).total;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    kern<<<dim3(gx, gy), 32 * (p.nvw + 1), smem, st>>>(p);
+    kern<<<dim3(gx, gy), 32 * (p.nvw + 2), smem, st>>>(p);  // view warps + prior + producer
     return cudaGetLastError();
 }
 
