@@ -84,6 +84,8 @@ struct mbir_handle {
     double* d_cs = nullptr;
     float *d_y = nullptr, *d_w = nullptr, *d_e = nullptr, *d_x = nullptr;
     float *d_theta2 = nullptr, *d_amount = nullptr, *d_scratch = nullptr;
+    uint8_t* d_perm = nullptr;  // [kNPerm][S2] voxel visiting orders
+    static constexpr int kNPerm = 64;
     int *d_task_list = nullptr, *d_task_count = nullptr;
     int *d_flat = nullptr, *d_brange = nullptr, *d_fetch = nullptr;
     unsigned long long* d_counters = nullptr;  // [updates, skipped, visits]
@@ -97,6 +99,7 @@ struct mbir_handle {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     std::vector<cudaEvent_t> kev;  // per-launch event pairs of the update kernel (one iteration)
     int kev_used = 0;
+    unsigned long long* d_tprof = nullptr;  // phase cycle counters (env MBIR_PHASE_PROFILE)
     std::string err;
 };
 
@@ -147,12 +150,15 @@ IcdParams make_params(mbir_handle* h)
     p.x = h->d_x;
     p.theta2 = h->d_theta2;
     p.scratch = h->d_scratch;
+    p.perm = h->d_perm;
+    p.nperm = mbir_handle::kNPerm;
     p.sv_amount = h->d_amount;
     p.counters = h->d_counters;
     p.sum_delta = h->d_sum_delta;
     p.seed = h->o.seed;
     p.iter = h->iter;
     p.deterministic = h->o.deterministic;
+    p.tprof = h->d_tprof;
     return p;
 }
 
@@ -335,6 +341,18 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         st->kernel_seconds = ksec;
         st->kernel_launches = klaunches;
     }
+    if (h->d_tprof) {  // development aid: per-phase cycles of the update kernel (thread 0 of each CTA)
+        unsigned long long t[16];
+        cudaMemcpy(t, h->d_tprof, sizeof(t), cudaMemcpyDeviceToHost);
+        cudaMemset(h->d_tprof, 0, sizeof(t));
+        const double v = (double)(t[5] ? t[5] : 1);
+        fprintf(stderr,
+                "[mbir phase] visits %llu voxels %llu | cycles/visit: order %.0f pack %.0f loop %.0f "
+                "writeback %.0f | loop cycles/voxel %.1f | warp0 own pack %.0f (tile0: issue %.0f "
+                "land %.0f stage %.0f)\n",
+                t[5], t[4], t[0] / v, t[1] / v, t[2] / v, t[3] / v, t[2] / (double)(t[4] ? t[4] : 1),
+                t[6] / v, t[7] / v, t[8] / v, t[9] / v);
+    }
     return MBIR_OK;
 }
 
@@ -410,8 +428,8 @@ void mbir_destroy(mbir_handle* h)
     void* ptrs[] = {h->A.codes, h->A.vals, h->A.off, h->A.count, h->A.scale, h->A.band_start,
                     h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
                     h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count,
-                    h->d_flat, h->d_brange, h->d_fetch, h->d_counters, h->d_sum_delta,
-                    h->d_flag, h->d_acc};
+                    h->d_flat, h->d_brange, h->d_fetch, h->d_perm, h->d_counters, h->d_sum_delta,
+                    h->d_flag, h->d_acc, h->d_tprof};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     if (h->h_counters) cudaFreeHost(h->h_counters);
@@ -456,7 +474,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if (G.nx < 1 || G.ny < 1 || G.nz_local < 1 || G.nviews < 1 || G.nchannels < 1 || !(G.dxy > 0) ||
         !(G.dchannel > 0) || G.z_offset < 0 || G.z_offset + G.nz_local > h->g.nz_total)
         return bail(MBIR_EINVAL);
-    if (G.nviews > 960) return (fail(h, MBIR_EINVAL, "nviews > 960 not supported"), bail(MBIR_EINVAL));
+    if (G.nviews > 768) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
     if (G.nchannels > (1 << 24)) return bail(MBIR_EINVAL);
     const mbir_prior& P = h->pr;
     if (!(P.p >= 1.0 && P.p <= 2.0) || P.q != 2.0 || !(P.T > 0) || !(P.sigma > 0) ||
@@ -542,14 +560,19 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if (info[0] & 2) return (fail(h, MBIR_EINVAL, "SV band wider than 255 channels"), bail(MBIR_EINVAL));
     h->rows = info[1];
     h->band_max = info[2];
-    if (h->rows > kMaxSvbRows)
-        return (fail(h, MBIR_EINVAL, "SV band needs " + std::to_string(h->rows) + " > 32 buffer rows: reduce sv_side"), bail(MBIR_EINVAL));
+    // a band row plus its misalignment (<= 3 floats) must fit one aligned 32-float window
+    if (h->rows > kMaxSvbRows - 3)
+        return (fail(h, MBIR_EINVAL, "SV band needs " + std::to_string(h->rows) + " > 29 buffer rows: reduce sv_side"), bail(MBIR_EINVAL));
+    if (((size_t)G.nviews * G.nchannels) % 4 != 0)
+        return (fail(h, MBIR_EINVAL, "nviews * nchannels must be a multiple of 4"), bail(MBIR_EINVAL));
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
     // ---- update-kernel shape
-    h->vpt = G.nviews > 384 ? 2 : 1;
+    // views per thread: fat view warps (4 views per lane, <= 8 warps) keep the per-voxel
+    // per-warp overhead (reduction, barrier, delta) small; tiny view counts use 1
+    h->vpt = G.nviews > 128 ? 4 : 1;
     h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
-    if (h->nvw > 14) return (fail(h, MBIR_EINVAL, "too many views"), bail(MBIR_EINVAL));
+    if (h->nvw > 6) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
     h->Vs = h->nvw * 32 * h->vpt;
     h->threads = 32 * (h->nvw + 2);  // view warps + prior warp + TMA producer warp
     if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
@@ -577,10 +600,33 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_flat, (size_t)8 * G.nz_local * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_brange, (size_t)8 * (h->max_group + 1)))) return bail(r);
     if ((r = dalloc(h, &h->d_fetch, (size_t)8 * h->max_group))) return bail(r);
+    {
+        // random voxel visiting orders within an SV ("randomized order"; reading R10):
+        // kNPerm Fisher-Yates permutations from a seeded splitmix64, one picked per SV visit
+        std::vector<uint8_t> perm((size_t)mbir_handle::kNPerm * h->S2);
+        uint64_t s = h->o.seed ^ 0xA0761D6478BD642FULL;
+        auto next = [&s]() {
+            uint64_t z = (s += 0x9E3779B97F4A7C15ULL);
+            z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+            z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+            return z ^ (z >> 31);
+        };
+        for (int q = 0; q < mbir_handle::kNPerm; ++q) {
+            uint8_t* pq = perm.data() + (size_t)q * h->S2;
+            for (int i = 0; i < h->S2; ++i) pq[i] = (uint8_t)i;
+            for (int i = h->S2 - 1; i > 0; --i) std::swap(pq[i], pq[next() % (uint64_t)(i + 1)]);
+        }
+        if ((r = dalloc(h, &h->d_perm, perm.size()))) return bail(r);
+        if (cudaMemcpy(h->d_perm, perm.data(), perm.size(), cudaMemcpyHostToDevice) != cudaSuccess) return bail(MBIR_ECUDA);
+    }
     if ((r = dalloc(h, &h->d_counters, 3))) return bail(r);
     if ((r = dalloc(h, &h->d_sum_delta, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_flag, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_acc, 1))) return bail(r);
+    if (getenv("MBIR_PHASE_PROFILE")) {
+        if ((r = dalloc(h, &h->d_tprof, 16))) return bail(r);
+        cudaMemset(h->d_tprof, 0, 16 * sizeof(unsigned long long));
+    }
     if (cudaMallocHost((void**)&h->h_counters, 4 * sizeof(unsigned long long)) != cudaSuccess) return bail(MBIR_ENOMEM);
     cudaMemsetAsync(h->d_x, 0, sizeof(float) * pl * (G.nz_local + 2), h->st);
     cudaMemsetAsync(h->d_amount, 0, sizeof(float) * G.nz_local * h->nsv, h->st);

@@ -86,6 +86,13 @@ __device__ __forceinline__ void red_add_f32(float* p, float v)
     asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v));
 }
 
+// vector atomic add of 4 consecutive floats (16-byte aligned), sm_90+
+__device__ __forceinline__ void red_add_v4(float* p, float a, float b, float c, float d)
+{
+    asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(a), "f"(b), "f"(c), "f"(d)
+                 : "memory");
+}
+
 __device__ __forceinline__ uint64_t mix64(uint64_t z)
 {
     z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
@@ -96,6 +103,35 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z)
 struct PriSlot {
     float sb, sbx, v, pad;
 };
+
+// q-GGMRF surrogate sums of Alg1:7 for the voxel at packed tile coordinate tofv (ly << 8 | lx):
+// lane r < nnb owns neighbour r (offset ndx/ndy/ndz, weight nbw); returns the warp-reduced
+// sums sbv = sum b_r phi(v - x_r) and sbx = sum b_r phi(v - x_r) x_r, plus this lane's own
+// (bt, xr) and the voxel's value v.  Free boundary: off-image neighbours contribute nothing.
+__device__ __forceinline__ void prior_terms(int tofv, const float* xt, int cslot, int TW, int gx0,
+                                            int gy0, int zg, const IcdParams& P, int ndx, int ndy,
+                                            int ndz, float nbw, int lane, int nnb, float& sbv,
+                                            float& sbx, float& bt, float& xr, float& v)
+{
+    const int lx = tofv & 255, ly = tofv >> 8;
+    v = xt[cslot + ly * TW + lx];
+    bt = 0.f;
+    xr = 0.f;
+    if (lane < nnb) {
+        const int gx = gx0 + lx + ndx, gy = gy0 + ly + ndy, gz = zg + ndz;
+        if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
+            xr = xt[cslot + (ndz * TW + ly + ndy) * TW + lx + ndx];
+            bt = nbw * phi_f(v - xr);
+        }
+    }
+    sbv = bt;
+    sbx = bt * xr;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        sbv += __shfl_xor_sync(kFull, sbv, o);
+        sbx += __shfl_xor_sync(kFull, sbx, o);
+    }
+}
 
 // ---- TMA (cp.async.bulk) + mbarrier helpers for the A-record ring ----
 __device__ __forceinline__ uint32_t smem_u32(const void* p)
@@ -131,15 +167,15 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
 }
 
 struct SmemLayout {
-    int sb_e, sb_w, xt, list, flags, red, pri, vscale, vth2, misc, astage, stage_bytes, off_in_stage,
-        mbar, total;
+    int sb_e, sb_w, xt, list, flags, tof, red, pri, vscale, vth2, misc, astage, stage_bytes,
+        off_in_stage, mbar, staging, total;
 };
 
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
 
 // A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
 __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, int S2, int nnb,
-                                                  int VA, bool u8, int nstage)
+                                                  int VA, bool u8, int nstage, int nvw)
 {
     SmemLayout L;
     const int TW = side + 2;
@@ -150,6 +186,7 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.xt = o;    o = align16(o + nzt * TW * TW * 4);
     L.list = o;  o = align16(o + S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
+    L.tof = o;   o = align16(o + S2 * 4);
     L.red = o;   o = align16(o + 2 * 16 * 4);
     L.pri = o;   o = align16(o + 2 * (int)sizeof(PriSlot));
     L.vscale = o; o = align16(o + S2 * 4);
@@ -159,29 +196,32 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.stage_bytes = align16(L.off_in_stage + VA);
     L.astage = o; o = align16(o + nstage * L.stage_bytes);
     L.mbar = o;  o = align16(o + nstage * 8);
+    L.staging = o; o = align16(o + nvw * 32 * 32 * 4);  // one 32x32 transpose tile per view warp
     L.total = o;
     return L;
 }
 
 template <int VPT, bool U8, int NNB, int R>
-__global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
+__global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 view + 2 warps
 {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int nvw = P.nvw;
     const int V = P.V, M = P.M, Vs = P.Vs, S2 = P.S2, side = P.side, VA = P.A.VA;
-    const SmemLayout L = smem_layout(P.rows, Vs, side, S2, NNB, VA, U8, R);
+    const SmemLayout L = smem_layout(P.rows, Vs, side, S2, NNB, VA, U8, R, nvw);
     float* sb_e = (float*)(smem + L.sb_e);
     float* sb_w = (float*)(smem + L.sb_w);
     float* xt = (float*)(smem + L.xt);
     int* list = (int*)(smem + L.list);
     int* flags = (int*)(smem + L.flags);
+    int* tof = (int*)(smem + L.tof);  // visiting order as packed (ly << 8 | lx)
     float* red = (float*)(smem + L.red);
     PriSlot* pri = (PriSlot*)(smem + L.pri);
     float* vscale = (float*)(smem + L.vscale);
     float* vth2 = (float*)(smem + L.vth2);
     uint64_t* mbar = (uint64_t*)(smem + L.mbar);
     unsigned char* astage = smem + L.astage;
+    float* stg_w = (float*)(smem + L.staging) + (warp < nvw ? warp : 0) * 32 * 32;
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
     const size_t plane = (size_t)P.nx * P.ny;
@@ -202,15 +242,25 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
         kval[t] = warp < nvw && kv[t] < V;
     }
     uint32_t gseq = 0;  // running voxel sequence number of this CTA: A stage = gseq % R
+    // prior-warp lane r owns neighbour r: its offset and weight live in registers (a per-lane
+    // __constant__ index would serialise in the constant cache on every voxel)
+    int ndx = 0, ndy = 0, ndz = 0;
+    float nbw = 0.f;
+    if (lane < c_prior.nnb) {
+        ndx = c_prior.dx[lane];
+        ndy = c_prior.dy[lane];
+        ndz = c_prior.dz[lane];
+        nbw = c_prior.b[lane];
+    }
 
     // this launch's batch: flat tasks [start, end) of the phase list (sched.cu k_flatten),
     // pulled one at a time by the persistent CTAs (dynamic distribution, Alg3:4 / T3)
     const int tstart = P.brange[0], tend = P.brange[1];
-    int* s_task = (int*)(smem + L.misc);
-    for (;;) {
-        if (threadIdx.x == 0) s_task[0] = tstart + atomicAdd(P.fetch, 1);
-        __syncthreads();
-        const int q = s_task[0];
+    int* s_task = (int*)(smem + L.misc);  // [0] first task, [1] next task (fetched one ahead)
+    if (threadIdx.x == 0) s_task[0] = tstart + atomicAdd(P.fetch, 1);
+    __syncthreads();
+    int q = s_task[0];
+    for (;; q = s_task[1]) {
         if (q >= tend) break;
         const int tk = P.flat[q];
         const int z = tk >> 14, sv = tk & 16383;  // local slice, SV
@@ -219,6 +269,8 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
         const int gx0 = bx * side, gy0 = by * side;
         const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
 
+        long long tp0 = 0, tp1 = 0, tp1b = 0, tp2 = 0, tp3 = 0, tpa = 0, tpb = 0, tpc = 0;
+        if (P.tprof && threadIdx.x == 0) tp0 = clock64();
         // ---- 1. x tile (+1 halo ring, +-1 slice in 3-D) into shared memory
         for (int i = threadIdx.x; i < (NNB == 26 ? 3 : 1) * TW * TW; i += blockDim.x) {
             const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
@@ -251,11 +303,12 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             flags[v0] = keep;
         }
         const int nact = __syncthreads_count(keep);
-        if (nact == 0) {
+        if (nact == 0) {  // the whole SV is zero-skipped: account for it and take the next task
             if (threadIdx.x == 0) {
                 P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
                 atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
                 atomicAdd(P.counters + 2, 1ull);
+                s_task[1] = tstart + atomicAdd(P.fetch, 1);
             }
             __syncthreads();
             continue;
@@ -266,32 +319,24 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
         //         prior warp's lane 0 then starts the TMA ring of A records (R voxels ahead)
         const size_t arec = (size_t)sv * S2;  // first A record of this SV
         if (is_prior) {
+            // one of NPERM host-drawn random permutations of the tile, chosen per
+            // (seed, iteration, slice, SV) visit; identity (raster order) in deterministic mode
             const uint64_t h = mix64(P.seed ^ mix64(((uint64_t)P.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)sv));
-            if (lane == 0) {
-                for (int i = 0; i < S2; ++i) list[i] = i;
-                if (!P.deterministic) {
-                    uint64_t st = h;
-                    for (int i = S2 - 1; i > 0; --i) {
-                        st += 0x9E3779B97F4A7C15ULL;
-                        const int r = (int)(((uint64_t)(uint32_t)mix64(st) * (uint32_t)(i + 1)) >> 32);
-                        const int t = list[i];
-                        list[i] = list[r];
-                        list[r] = t;
-                    }
-                }
-            }
-            __syncwarp();
+            const uint8_t* perm = P.perm + (size_t)(h % (uint64_t)P.nperm) * S2;
             int n = 0;
             for (int base = 0; base < S2; base += 32) {
                 const int i = base + lane;
-                const int v = i < S2 ? list[i] : 0;
+                const int v = i < S2 ? (P.deterministic ? i : (int)perm[i]) : 0;
                 const bool k = i < S2 && flags[v];
                 const unsigned m = __ballot_sync(kFull, k);
-                __syncwarp();
-                if (k) list[n + __popc(m & ((1u << lane) - 1))] = v;
+                if (k) {
+                    const int p = n + __popc(m & ((1u << lane) - 1));
+                    list[p] = v;
+                    tof[p] = ((v / side) << 8) | (v % side);  // packed (ly, lx): no div in the loop
+                }
                 n += __popc(m);
-                __syncwarp();
             }
+            __syncwarp();
             for (int i = lane; i < nact; i += 32) {
                 const int v = list[i];
                 vscale[i] = P.A.scale[arec + v];
@@ -314,46 +359,105 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             }
         }
 
+        if (P.tprof && threadIdx.x == 0) tp1 = clock64();
         // ---- 4. view threads: SVB pack (coalesced 128-byte band rows, transposed by shuffles);
         //         e_init rows go to this CTA's L2-resident scratch tile for the write-back
         float* scr = P.scratch + (size_t)blockIdx.x * (size_t)Vs * 32;
         if (warp < nvw) {
             const float* wz = P.w + (size_t)z * V * M;
             float* ez = P.e + (size_t)z * V * M;
+            // Each band row is read as the 16-byte-aligned 32-float window that contains it (the
+            // slice base is 16-byte aligned, V*M % 4 == 0): 8 lanes x float4 per row, 4 rows per
+            // LDG.128, so a 32-view tile of w and e is 16 vector loads (few requests in flight).
+            // The window is stored rotated in the warp's staging tile -- band column c of row i at
+            // column (c + i) % 32 -- so that lane k then reads row k's column c at (c + k) % 32
+            // (banks distinct over k) and writes sb[c][k] (banks distinct over k): conflict-free.
+            // e_init windows go to this CTA's L2-resident scratch tile for the write-back.
+            int bwv[VPT], rov[VPT];
+#pragma unroll
+            for (int t = 0; t < VPT; ++t) {
+                const int kk = (warp * VPT + t) * 32 + lane;
+                bwv[t] = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
+                rov[t] = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
+            }
+            const int sub = lane >> 3, ch = lane & 7;  // row-in-quad and float4 chunk of this lane
 #pragma unroll 1
             for (int t = 0; t < VPT; ++t) {
                 const int k0 = (warp * VPT + t) * 32;
                 const int kk = k0 + lane;
-                const int bw = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
-                // 32-bit element offset of this lane's band row; rows are broadcast by shuffle
-                const int roff = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
-                float r[32];
+                float4 w4[8], e4[8];
+                int so[8];
 #pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                    const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
-                    r[i] = lane < wi ? __ldg(wz + oi + lane) : 0.f;
+                for (int m = 0; m < 8; ++m) {
+                    const int i = 4 * m + sub;
+                    const int oi = __shfl_sync(kFull, rov[t], i), wi = __shfl_sync(kFull, bwv[t], i);
+                    const int s = oi & 3;
+                    so[m] = s;
+                    const bool ok = k0 + i < V && 4 * ch < s + wi;
+                    const size_t a4 = (size_t)(oi - s) + 4 * ch;
+                    w4[m] = ok ? __ldg((const float4*)(wz + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    e4[m] = ok ? __ldcg((const float4*)(ez + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
                 }
-                transpose32(r, lane);
+                if (P.tprof && threadIdx.x == 0 && t == 0) tpa = clock64();
+#pragma unroll
+                for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), e4[m]);
+                if (P.tprof && threadIdx.x == 0 && t == 0) tpb = clock64();
+                auto put = [&](const float4 (&v)[8]) {
+#pragma unroll
+                    for (int m = 0; m < 8; ++m) {
+                        const int i = 4 * m + sub;
+                        const float vv[4] = {v[m].x, v[m].y, v[m].z, v[m].w};
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const int c = 4 * ch + j - so[m];  // band column
+                            if (c >= 0) stg_w[i * 32 + ((c + i) & 31)] = vv[j];
+                        }
+                    }
+                    __syncwarp();
+                };
+                const int bwk = bwv[t];
+                put(w4);
 #pragma unroll
                 for (int c = 0; c < 32; ++c)
-                    if (c < P.rows) sb_w[c * Vs + kk] = r[c];
-                asm volatile("" ::: "memory");  // keep the e loads after the w tile is retired
-#pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                    const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
-                    r[i] = lane < wi ? __ldcg(ez + oi + lane) : 0.f;
-                    __stcg(scr + (k0 + i) * 32 + lane, r[i]);
-                }
-                transpose32(r, lane);
+                    if (c < P.rows) sb_w[c * Vs + kk] = c < bwk ? stg_w[lane * 32 + ((c + lane) & 31)] : 0.f;
+                __syncwarp();
+                put(e4);
 #pragma unroll
                 for (int c = 0; c < 32; ++c)
-                    if (c < P.rows) sb_e[c * Vs + kk] = r[c];
+                    if (c < P.rows) sb_e[c * Vs + kk] = c < bwk ? stg_w[lane * 32 + ((c + lane) & 31)] : 0.f;
+                __syncwarp();
+                if (P.tprof && threadIdx.x == 0 && t == 0) tpc = clock64();
             }
-        } else if (warp == nvw + 1 && lane == 0) {
-            mbar_wait(mbar + gseq % R, (gseq / R) & 1);  // A records of the first voxel landed
+            if (P.tprof && threadIdx.x == 0) tp1b = clock64();
+        } else if (warp == nvw + 1) {
+            // producer warp: fetch the next task now and warm L2 with its band rows, so the
+            // next pack reads L2 instead of HBM (the x tile, scratch and A ring are separate)
+            int nq = 0;
+            if (lane == 0) {
+                nq = tstart + atomicAdd(P.fetch, 1);
+                s_task[1] = nq;
+            }
+            nq = __shfl_sync(kFull, nq, 0);
+            if (nq < tend) {
+                const int ntk = P.flat[nq];
+                const int nz = ntk >> 14, nsv = ntk & 16383;
+                const float* nw = P.w + (size_t)nz * V * M;
+                const float* ne = P.e + (size_t)nz * V * M;
+                for (int k = lane; k < V; k += 32) {
+                    const int b = P.A.band_start[(size_t)nsv * V + k];
+                    const int wd = max((int)P.A.band_width[(size_t)nsv * V + k], 1);
+                    const size_t o0 = (size_t)k * M + b, o1 = o0 + wd - 1;
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(nw + o0));
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(nw + o1));
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(ne + o0));
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(ne + o1));
+                }
+            }
+            if (lane == 0) mbar_wait(mbar + gseq % R, (gseq / R) & 1);  // first voxel's A landed
         }
         __syncthreads();
 
+        if (P.tprof && threadIdx.x == 0) tp2 = clock64();
         // ---- 5. sequential-exact voxel loop, one barrier per voxel
         float amount = 0.f;
         const int cslot = (zc * TW + 1) * TW + 1;  // tile index of local (0,0)
@@ -361,7 +465,11 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             const int buf = idx & 1;
             const uint32_t g = gseq + idx;
             const unsigned char* stg = astage + (g % R) * L.stage_bytes;
-            float ev[VPT][4], av[VPT][4];
+            // live across the barrier per view: e values, band offset and the A record (the raw
+            // 32-bit code word in u8 mode -- re-dequantised for the scatter, saving registers)
+            float ev[VPT][4];
+            uint32_t cwv[VPT];
+            float4 a4v[VPT];
             int oo[VPT];
             if (warp < nvw) {
                 float t1 = 0.f;
@@ -370,16 +478,17 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                     if (kval[t]) {
                         const int o = stg[L.off_in_stage + kv[t]];
                         oo[t] = o;
+                        float av[4];
                         if (U8) {
-                            const uint32_t cw = ((const uint32_t*)stg)[kv[t]];
+                            cwv[t] = ((const uint32_t*)stg)[kv[t]];
 #pragma unroll
-                            for (int i = 0; i < 4; ++i) av[t][i] = dq(cw, i);
+                            for (int i = 0; i < 4; ++i) av[i] = dq(cwv[t], i);
                         } else {
-                            const float4 a4 = ((const float4*)stg)[kv[t]];
-                            av[t][0] = a4.x;
-                            av[t][1] = a4.y;
-                            av[t][2] = a4.z;
-                            av[t][3] = a4.w;
+                            a4v[t] = ((const float4*)stg)[kv[t]];
+                            av[0] = a4v[t].x;
+                            av[1] = a4v[t].y;
+                            av[2] = a4v[t].z;
+                            av[3] = a4v[t].w;
                         }
                         const float* pe = sb_e + o * Vs + kv[t];
                         const float* pw = sb_w + o * Vs + kv[t];
@@ -387,7 +496,7 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
 #pragma unroll
                         for (int i = 0; i < 4; ++i) {
                             ev[t][i] = pe[i * Vs];
-                            acc = fmaf(pw[i * Vs] * ev[t][i], av[t][i], acc);
+                            acc = fmaf(pw[i * Vs] * ev[t][i], av[i], acc);
                         }
                         t1 += acc;
                     }
@@ -396,34 +505,13 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                 for (int o = 16; o > 0; o >>= 1) t1 += __shfl_xor_sync(kFull, t1, o);
                 if (lane == 0) red[buf * 16 + warp] = t1;
             } else if (warp == nvw) {
-                // prior warp: surrogate terms of Alg1:7 over the neighbourhood (reading R1-R2)
-                __syncwarp();  // lane 0's x-tile write of the previous voxel is visible
-                const int slot = list[idx];
-                const int lx = slot % side, ly = slot / side;
-                const float v = xt[cslot + ly * TW + lx];
-                float sbv = 0.f, sbx = 0.f;
-                if (lane < NNB) {
-                    const int dx = c_prior.dx[lane], dy = c_prior.dy[lane], dz = c_prior.dz[lane];
-                    const int gx = gx0 + lx + dx, gy = gy0 + ly + dy, gz = zg + dz;
-                    if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
-                        const float xr = xt[cslot + (dz * TW + ly + dy) * TW + lx + dx];
-                        const float bt = c_prior.b[lane] * phi_f(v - xr);
-                        sbv = bt;
-                        sbx = bt * xr;
-                    }
-                }
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) {
-                    sbv += __shfl_xor_sync(kFull, sbv, o);
-                    sbx += __shfl_xor_sync(kFull, sbx, o);
-                }
-                if (lane == 0) {
-                    PriSlot ps;
-                    ps.sb = sbv;
-                    ps.sbx = sbx;
-                    ps.v = v;
-                    ps.pad = 0.f;
-                    pri[buf] = ps;
+                // prior warp: the surrogate terms of voxel idx were published after barrier idx-1
+                // (speculatively, then corrected); only voxel 0 is computed here
+                if (idx == 0) {
+                    float sbv, sbx, bt, xr, v;
+                    prior_terms(tof[0], xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
+                                sbv, sbx, bt, xr, v);
+                    if (lane == 0) pri[0] = PriSlot{sbv, sbx, v, 0.f};
                 }
             } else if (lane == 0) {
                 // producer warp: the next voxel's A records must have landed before the barrier
@@ -431,10 +519,9 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             }
             __syncthreads();
             // every warp derives the same delta (identical inputs, identical order)
-            const float4* r4 = (const float4*)(red + buf * 16);
-            const float4 a0 = r4[0], a1 = r4[1], a2 = r4[2], a3 = r4[3];
-            const float s1 = ((a0.x + a0.y) + (a0.z + a0.w)) + ((a1.x + a1.y) + (a1.z + a1.w)) +
-                             (((a2.x + a2.y) + (a2.z + a2.w)) + ((a3.x + a3.y) + (a3.z + a3.w)));
+            const float4* r4 = (const float4*)(red + buf * 16);  // nvw <= 8 partials, rest 0
+            const float4 a0 = r4[0], a1 = r4[1];
+            const float s1 = ((a0.x + a0.y) + (a0.z + a0.w)) + ((a1.x + a1.y) + (a1.z + a1.w));
             const PriSlot ps = pri[buf];
             const float scale = vscale[idx];
             const float theta1 = -scale * s1;   // Alg1:5, theta1 = -sum w A e
@@ -452,15 +539,44 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
                         if (kval[t]) {
                             float* pe = sb_e + oo[t] * Vs + kv[t];
 #pragma unroll
-                            for (int i = 0; i < 4; ++i) pe[i * Vs] = fmaf(-av[t][i], sd, ev[t][i]);
+                            for (int i = 0; i < 4; ++i) {
+                                const float a = U8 ? dq(cwv[t], i)
+                                                   : (i == 0 ? a4v[t].x : i == 1 ? a4v[t].y : i == 2 ? a4v[t].z : a4v[t].w);
+                                pe[i * Vs] = fmaf(-a, sd, ev[t][i]);
+                            }
                         }
                 }
             } else if (warp == nvw) {
-                if (lane == 0) {
-                    const int slot = list[idx];
-                    xt[cslot + (slot / side) * TW + slot % side] = unew;
-                    amount += fabsf(delta);
+                // prior warp: surrogate terms of voxel idx+1, computed from the x tile BEFORE
+                // voxel idx's new value is stored (concurrently with delta above), then corrected
+                // for that one neighbour if voxel idx is adjacent to voxel idx+1
+                const int tcur = tof[idx];
+                const int ccur = cslot + (tcur >> 8) * TW + (tcur & 255);
+                if (idx + 1 < nact) {
+                    const int tnext = tof[idx + 1];
+                    float sbv, sbx, bt, xr, v1;
+                    prior_terms(tnext, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
+                                sbv, sbx, bt, xr, v1);
+                    __syncwarp();
+                    if (lane == 0) xt[ccur] = unew;
+                    const int dx = (tcur & 255) - (tnext & 255), dy = (tcur >> 8) - (tnext >> 8);
+                    if (dx >= -1 && dx <= 1 && dy >= -1 && dy <= 1) {
+                        const bool mine = lane < NNB && ndx == dx && ndy == dy && ndz == 0;
+                        float c0 = 0.f, c1 = 0.f;
+                        if (mine) {
+                            const float bn = nbw * phi_f(v1 - unew);
+                            c0 = bn - bt;
+                            c1 = bn * unew - bt * xr;
+                        }
+                        const int src = __ffs(__ballot_sync(kFull, mine)) - 1;
+                        sbv += __shfl_sync(kFull, c0, src);
+                        sbx += __shfl_sync(kFull, c1, src);
+                    }
+                    if (lane == 0) pri[(idx + 1) & 1] = PriSlot{sbv, sbx, v1, 0.f};
+                } else if (lane == 0) {
+                    xt[ccur] = unew;
                 }
+                if (lane == 0) amount += fabsf(delta);
             } else if (lane == 0) {
                 // producer warp.  This voxel's stage was read by every view warp before the barrier: refill it
                 // with the A records of voxel idx + R (async proxy after generic reads)
@@ -479,33 +595,46 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             }
         }
         gseq += nact;
+        if (P.tprof && threadIdx.x == 0) tp3 = clock64();
         __syncthreads();
 
         // ---- 6. write-back: delta e of the band, atomically, and the SV's voxels
         if (warp < nvw) {
             float* ez = P.e + (size_t)z * V * M;
+            // the final band goes back through the rotated staging tile (see the pack), then each
+            // aligned 32-float row window gets delta = final - e_init with red.global.add.v4.f32
+            const int sub = lane >> 3, ch = lane & 7;
 #pragma unroll 1
             for (int t = 0; t < VPT; ++t) {
                 const int k0 = (warp * VPT + t) * 32;
                 const int kk = k0 + lane;
                 const int bw = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
                 const int roff = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
-                float s0[32];  // e_init rows (lane = channel), loads in flight during the transpose
+                float4 s4[8];  // e_init windows, in flight during the staging below
 #pragma unroll
-                for (int i = 0; i < 32; ++i) s0[i] = __ldcg(scr + (k0 + i) * 32 + lane);
-                float r[32];
+                for (int m = 0; m < 8; ++m) s4[m] = __ldcg((const float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch));
 #pragma unroll
                 for (int c = 0; c < 32; ++c)
-                    r[c] = (kk < V && c < P.rows) ? sb_e[c * Vs + kk] : 0.f;
-                transpose32(r, lane);
+                    if (c < P.rows) stg_w[lane * 32 + ((c + lane) & 31)] = sb_e[c * Vs + kk];
+                __syncwarp();
 #pragma unroll
-                for (int i = 0; i < 32; ++i) {
+                for (int m = 0; m < 8; ++m) {
+                    const int i = 4 * m + sub;
                     const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
-                    const float d = r[i] - s0[i];
-                    if (lane < wi && d != 0.f) red_add_f32(ez + oi + lane, d);
+                    const int s = oi & 3;
+                    float d[4];
+                    const float e0[4] = {s4[m].x, s4[m].y, s4[m].z, s4[m].w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int c = 4 * ch + j - s;
+                        d[j] = (c >= 0 && c < wi) ? stg_w[i * 32 + ((c + i) & 31)] - e0[j] : 0.f;
+                    }
+                    if (k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
+                        red_add_v4(ez + (oi - s) + 4 * ch, d[0], d[1], d[2], d[3]);
                 }
+                __syncwarp();
             }
-        } else {
+        } else if (warp == nvw) {
             for (int i = lane; i < tw * th; i += 32) {
                 const int lx = i % tw, ly = i / tw;
                 P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] =
@@ -520,6 +649,19 @@ __global__ void __launch_bounds__(512, 1) k_icd_sv(const IcdParams P)
             }
         }
         __syncthreads();
+        if (P.tprof && threadIdx.x == 0) {
+            const long long tp4 = clock64();
+            atomicAdd(P.tprof + 0, (unsigned long long)(tp1 - tp0));  // x tile, zero-skip, order
+            atomicAdd(P.tprof + 1, (unsigned long long)(tp2 - tp1));  // SVB pack (+ first A stage)
+            atomicAdd(P.tprof + 2, (unsigned long long)(tp3 - tp2));  // voxel loop
+            atomicAdd(P.tprof + 3, (unsigned long long)(tp4 - tp3));  // write-back
+            atomicAdd(P.tprof + 4, (unsigned long long)nact);
+            atomicAdd(P.tprof + 5, 1ull);
+            atomicAdd(P.tprof + 6, (unsigned long long)(tp1b - tp1));  // view-warp 0's own pack
+            atomicAdd(P.tprof + 7, (unsigned long long)(tpa - tp1));   // tile 0: issue of loads
+            atomicAdd(P.tprof + 8, (unsigned long long)(tpb - tpa));   // tile 0: loads landed
+            atomicAdd(P.tprof + 9, (unsigned long long)(tpc - tpb));   // tile 0: staging/transposes
+        }
     }
 }
 
@@ -680,7 +822,7 @@ constexpr int ring_depth(bool u8) { return u8 ? 8 : 3; }
 int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
 {
     (void)vpt;
-    return smem_layout(p.rows, p.Vs, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize)).total;
+    return smem_layout(p.rows, p.Vs, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw).total;
 }
 
 template <int VPT, bool U8, int NNB>
@@ -688,7 +830,7 @@ static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t
 {
     constexpr int R = ring_depth(U8);
     auto kern = k_icd_sv<VPT, U8, NNB, R>;
-    const int smem = smem_layout(p.rows, p.Vs, p.side, p.S2, NNB, p.A.VA, U8, R).total;
+    const int smem = smem_layout(p.rows, p.Vs, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw).total;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     kern<<<dim3(gx, gy), 32 * (p.nvw + 2), smem, st>>>(p);  // view warps + prior + producer
@@ -702,8 +844,8 @@ cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int 
         if (quantize) return nnb == 26 ? launch_icd_t<1, true, 26>(p, gx, gy, st) : launch_icd_t<1, true, 8>(p, gx, gy, st);
         return nnb == 26 ? launch_icd_t<1, false, 26>(p, gx, gy, st) : launch_icd_t<1, false, 8>(p, gx, gy, st);
     }
-    if (quantize) return nnb == 26 ? launch_icd_t<2, true, 26>(p, gx, gy, st) : launch_icd_t<2, true, 8>(p, gx, gy, st);
-    return nnb == 26 ? launch_icd_t<2, false, 26>(p, gx, gy, st) : launch_icd_t<2, false, 8>(p, gx, gy, st);
+    if (quantize) return nnb == 26 ? launch_icd_t<4, true, 26>(p, gx, gy, st) : launch_icd_t<4, true, 8>(p, gx, gy, st);
+    return nnb == 26 ? launch_icd_t<4, false, 26>(p, gx, gy, st) : launch_icd_t<4, false, 8>(p, gx, gy, st);
 }
 
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st)

@@ -58,6 +58,8 @@ struct IcdParams {
     float* theta2;           // [nz_local][nsv][S2]
     float* scratch;          // [max CTAs][Vs][32] e_init tiles of the running SV visits
     float* sv_amount;        // [nz_local][nsv] sum |delta| of the SV's last visit
+    const uint8_t* perm;     // [nperm][S2] random permutations of an SV's voxel slots
+    int nperm;
     const int* flat;         // phase task list, entries (local slice << 14) | SV
     const int* brange;       // [2]: this launch's batch = flat[brange[0] .. brange[1])
     int* fetch;              // task counter of this launch (zeroed per iteration)
@@ -67,6 +69,7 @@ struct IcdParams {
     int iter;
     int zero_skip_active;
     int deterministic;
+    unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
 };
 
 struct SchedParams {
