@@ -526,7 +526,14 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     h->A.nsv = h->nsv;
     h->A.S2 = h->S2;
     h->A.V = G.nviews;
-    h->A.VA = (G.nviews + 15) & ~15;  // record stride: TMA bulk copies need 16-byte multiples
+    // ---- update-kernel shape: fat view warps (4 views per lane, <= 6 warps) keep the per-voxel
+    // per-warp overhead (reduction, barrier, delta) small; tiny view counts use 1 per lane
+    h->vpt = G.nviews > 128 ? 4 : 1;
+    h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
+    if (h->nvw > 6) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
+    h->Vs = h->nvw * 32 * h->vpt;
+    h->A.vpt = h->vpt;
+    h->A.VA = h->Vs;  // thread-major record positions (apos); a multiple of 32 -> TMA-sized
     const size_t nA = (size_t)h->nsv * h->S2 * h->A.VA;
     if (quant) {
         if ((r = dalloc(h, &h->A.codes, nA))) return bail(r);
@@ -567,13 +574,6 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         return (fail(h, MBIR_EINVAL, "nviews * nchannels must be a multiple of 4"), bail(MBIR_EINVAL));
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
-    // ---- update-kernel shape
-    // views per thread: fat view warps (4 views per lane, <= 8 warps) keep the per-voxel
-    // per-warp overhead (reduction, barrier, delta) small; tiny view counts use 1
-    h->vpt = G.nviews > 128 ? 4 : 1;
-    h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
-    if (h->nvw > 6) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
-    h->Vs = h->nvw * 32 * h->vpt;
     h->threads = 32 * (h->nvw + 2);  // view warps + prior warp + TMA producer warp
     if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
     {

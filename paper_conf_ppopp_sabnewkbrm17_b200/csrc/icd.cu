@@ -468,28 +468,40 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
             // live across the barrier per view: e values, band offset and the A record (the raw
             // 32-bit code word in u8 mode -- re-dequantised for the scatter, saving registers)
             float ev[VPT][4];
-            uint32_t cwv[VPT];
-            float4 a4v[VPT];
+            float4 a4v[VPT];  // dequantised A values of this voxel's 4 channels per view
             int oo[VPT];
             if (warp < nvw) {
                 float t1 = 0.f;
+                // this thread's VPT A records are adjacent (apos): one vector load of codes
+                // and one of band offsets
+                const int tp = warp * 32 + lane;
+                uint32_t cwa[VPT], oba = 0;
+                if (U8) {
+                    if (VPT == 4) {
+                        const uint4 c4 = ((const uint4*)stg)[tp];
+                        cwa[0] = c4.x;
+                        cwa[VPT > 1 ? 1 : 0] = c4.y;
+                        cwa[VPT > 2 ? 2 : 0] = c4.z;
+                        cwa[VPT > 3 ? 3 : 0] = c4.w;
+                    } else {
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t) cwa[t] = ((const uint32_t*)stg)[tp * VPT + t];
+                    }
+                }
+                if (VPT == 4)
+                    oba = ((const uint32_t*)(stg + L.off_in_stage))[tp];
 #pragma unroll
                 for (int t = 0; t < VPT; ++t) {
                     if (kval[t]) {
-                        const int o = stg[L.off_in_stage + kv[t]];
+                        const int o = VPT == 4 ? (int)((oba >> (8 * t)) & 255u) : (int)stg[L.off_in_stage + tp * VPT + t];
                         oo[t] = o;
-                        float av[4];
                         if (U8) {
-                            cwv[t] = ((const uint32_t*)stg)[kv[t]];
-#pragma unroll
-                            for (int i = 0; i < 4; ++i) av[i] = dq(cwv[t], i);
+                            const uint32_t cw = cwa[t];
+                            a4v[t] = make_float4(dq(cw, 0), dq(cw, 1), dq(cw, 2), dq(cw, 3));
                         } else {
-                            a4v[t] = ((const float4*)stg)[kv[t]];
-                            av[0] = a4v[t].x;
-                            av[1] = a4v[t].y;
-                            av[2] = a4v[t].z;
-                            av[3] = a4v[t].w;
+                            a4v[t] = ((const float4*)stg)[tp * VPT + t];
                         }
+                        const float av[4] = {a4v[t].x, a4v[t].y, a4v[t].z, a4v[t].w};
                         const float* pe = sb_e + o * Vs + kv[t];
                         const float* pw = sb_w + o * Vs + kv[t];
                         float acc = 0.f;
@@ -540,8 +552,7 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                             float* pe = sb_e + oo[t] * Vs + kv[t];
 #pragma unroll
                             for (int i = 0; i < 4; ++i) {
-                                const float a = U8 ? dq(cwv[t], i)
-                                                   : (i == 0 ? a4v[t].x : i == 1 ? a4v[t].y : i == 2 ? a4v[t].z : a4v[t].w);
+                                const float a = i == 0 ? a4v[t].x : i == 1 ? a4v[t].y : i == 2 ? a4v[t].z : a4v[t].w;
                                 pe[i * Vs] = fmaf(-a, sd, ev[t][i]);
                             }
                         }
@@ -680,14 +691,14 @@ __global__ void k_theta2(const IcdParams P)
     const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
     float acc = 0.f;
     for (int k = lane; k < P.V; k += 32) {
-        const int f = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + k];
-        const int n = P.A.count[ab + k];
+        const int f = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + apos(k, P.A.vpt)];
+        const int n = P.A.count[ab + apos(k, P.A.vpt)];
         float a[4];
         if (U8) {
-            const uint32_t c = P.A.codes[ab + k];
+            const uint32_t c = P.A.codes[ab + apos(k, P.A.vpt)];
             for (int i = 0; i < 4; ++i) a[i] = dq(c, i) * sc;
         } else {
-            const float4 q = P.A.vals[ab + k];
+            const float4 q = P.A.vals[ab + apos(k, P.A.vpt)];
             a[0] = q.x; a[1] = q.y; a[2] = q.z; a[3] = q.w;
         }
         for (int i = 0; i < 4; ++i)
@@ -719,7 +730,7 @@ __global__ void k_forward(const IcdParams P)
             const float xv = P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx];
             if (xv == 0.f) continue;
             any = true;
-            const size_t ai = ((size_t)sv * P.S2 + slot) * P.A.VA + k;
+            const size_t ai = ((size_t)sv * P.S2 + slot) * P.A.VA + apos(k, P.A.vpt);
             const int o = P.A.off[ai];
             const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
             for (int i = 0; i < 4; ++i) {
@@ -763,14 +774,14 @@ __global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
     const float* ez = P.e + (size_t)z * P.V * P.M;
     float t1 = 0.f, t2 = 0.f;
     for (int k = threadIdx.x; k < P.V; k += blockDim.x) {
-        const int f = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + k];
-        const int n = P.A.count[ab + k];
+        const int f = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + apos(k, P.A.vpt)];
+        const int n = P.A.count[ab + apos(k, P.A.vpt)];
         for (int i = 0; i < 4 && i < n; ++i) {
             float a;
             if (U8) {
-                a = dq(P.A.codes[ab + k], i) * sc;
+                a = dq(P.A.codes[ab + apos(k, P.A.vpt)], i) * sc;
             } else {
-                const float4 v4 = P.A.vals[ab + k];
+                const float4 v4 = P.A.vals[ab + apos(k, P.A.vpt)];
                 a = i == 0 ? v4.x : i == 1 ? v4.y : i == 2 ? v4.z : v4.w;
             }
             const float ww = wz[(size_t)k * P.M + f + i];

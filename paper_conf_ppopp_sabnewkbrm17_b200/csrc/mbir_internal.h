@@ -33,7 +33,9 @@ struct PriorConst {
 // ---- compressed system matrix, per SuperVoxel ----
 struct DevA {
     int nsv, S2, V;          // SVs per slice, slots per SV (side^2), views
-    int VA;                  // per-voxel record stride in views, V rounded up to 16 (TMA-sized)
+    int VA;                  // per-voxel record stride (positions) = 32 * view warps * vpt
+    int vpt;                 // views per update-kernel thread; records are stored thread-major:
+                             // view k sits at position apos(k) so a thread's views are adjacent
     uint32_t* codes;         // [nsv][S2][V] 4 uint8 codes (byte i = channel offset i), quantize_A
     float4* vals;            // [nsv][S2][V] fp32 values, !quantize_A
     uint8_t* off;            // [nsv][S2][V] first channel - band start
@@ -42,6 +44,14 @@ struct DevA {
     int32_t* band_start;     // [nsv][V] first channel of the SV band
     uint8_t* band_width;     // [nsv][V] band width (channels)
 };
+
+// Record position of view k: thread (warp w, lane l) of the update kernel owns views
+// (w*vpt + t)*32 + l, t < vpt, stored at positions (w*32 + l)*vpt + t (one vector load each).
+__host__ __device__ __forceinline__ int apos(int k, int vpt)
+{
+    const int blk = k >> 5;  // = w*vpt + t
+    return ((blk / vpt) * 32 + (k & 31)) * vpt + blk % vpt;
+}
 
 // ---- parameters of the fused SuperVoxel update kernel ----
 struct IcdParams {

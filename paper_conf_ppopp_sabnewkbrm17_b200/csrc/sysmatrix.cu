@@ -121,8 +121,8 @@ __global__ void __launch_bounds__(kColThreads) k_columns(
         const int k = threadIdx.x + t * kColThreads;
         if (k >= V) continue;
         const int n = col[t].count < kK ? col[t].count : kK;
-        first_tmp[base + k] = n > 0 ? col[t].first : -1;
-        A.count[base + k] = (uint8_t)n;
+        first_tmp[base + apos(k, A.vpt)] = n > 0 ? col[t].first : -1;
+        A.count[base + apos(k, A.vpt)] = (uint8_t)n;
         if (quantize) {
             uint32_t word = 0;
 #pragma unroll
@@ -133,9 +133,9 @@ __global__ void __launch_bounds__(kColThreads) k_columns(
                                     : 0u;
                 word |= code << (8 * i);
             }
-            A.codes[base + k] = word;
+            A.codes[base + apos(k, A.vpt)] = word;
         } else {
-            A.vals[base + k] = make_float4((float)col[t].v[0], (float)col[t].v[1],
+            A.vals[base + apos(k, A.vpt)] = make_float4((float)col[t].v[0], (float)col[t].v[1],
                                            (float)col[t].v[2], (float)col[t].v[3]);
         }
     }
@@ -149,7 +149,7 @@ __global__ void k_bands(int V, int S2, const int32_t* __restrict__ first_tmp, De
     for (int k = threadIdx.x; k < V; k += blockDim.x) {
         int lo = 1 << 30, hi = -1;
         for (int v = 0; v < S2; ++v) {
-            const size_t i = ((size_t)sv * S2 + v) * A.VA + k;
+            const size_t i = ((size_t)sv * S2 + v) * A.VA + apos(k, A.vpt);
             const int f = first_tmp[i];
             if (f < 0) continue;
             lo = min(lo, f);
@@ -163,7 +163,7 @@ __global__ void k_bands(int V, int S2, const int32_t* __restrict__ first_tmp, De
         atomicMax(maxwidth, wdt);
         int rowmax = 0;
         for (int v = 0; v < S2; ++v) {
-            const size_t i = ((size_t)sv * S2 + v) * A.VA + k;
+            const size_t i = ((size_t)sv * S2 + v) * A.VA + apos(k, A.vpt);
             const int f = first_tmp[i];
             const int o = f < 0 ? 0 : f - lo;
             if (o > 255) atomicOr(err, 2);
@@ -187,12 +187,12 @@ __global__ void k_export(int nx, int ny, double d, int V, int M, double dc, doub
     const int slot = (iy % side) * side + ix % side;
     const size_t base = ((size_t)sv * A.S2 + slot) * A.VA;
     for (int k = threadIdx.x; k < V; k += blockDim.x) {
-        const int n = A.count[base + k];
+        const int n = A.count[base + apos(k, A.vpt)];
         const size_t o = jo * V + k;
-        if (first) first[o] = n > 0 ? A.band_start[(size_t)sv * V + k] + A.off[base + k] : 0;
+        if (first) first[o] = n > 0 ? A.band_start[(size_t)sv * V + k] + A.off[base + apos(k, A.vpt)] : 0;
         if (count) count[o] = n;
         if (codes) {
-            const uint32_t wd = quantize ? A.codes[base + k] : 0u;
+            const uint32_t wd = quantize ? A.codes[base + apos(k, A.vpt)] : 0u;
             for (int i = 0; i < kK; ++i) codes[o * kK + i] = (uint8_t)(wd >> (8 * i));
         }
         if (vals) {
