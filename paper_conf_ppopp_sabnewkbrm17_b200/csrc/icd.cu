@@ -133,6 +133,93 @@ __device__ __forceinline__ void prior_terms(int tofv, const float* xt, int cslot
     }
 }
 
+// surrogate terms of a pair of consecutive voxels (a, b): a's sums, b's sums computed with a's
+// OLD value, and -- if a is b's neighbour -- that neighbour's term (btab) and weight (bab)
+struct PriPair {
+    float sa, sxa, va, sb, sxb, vb, btab, bab;
+};
+
+__device__ __forceinline__ float sum8(const float* r)
+{
+    const float4 a = ((const float4*)r)[0], b = ((const float4*)r)[1];
+    return ((a.x + a.y) + (a.z + a.w)) + ((b.x + b.y) + (b.z + b.w));
+}
+
+// A values of a voxel re-indexed to another voxel's channels: result[i] = A[i + d] (0 outside)
+template <bool U8>
+__device__ __forceinline__ float4 shifted(uint32_t cw, float4 a, int d)
+{
+    if (U8) {
+        const uint32_t s = (d >= 4 || d <= -4) ? 0u : (d >= 0 ? (cw >> (8 * d)) : (cw << (-8 * d)));
+        return make_float4(dq(s, 0), dq(s, 1), dq(s, 2), dq(s, 3));
+    }
+    const float v[4] = {a.x, a.y, a.z, a.w};
+    float r[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int j = i + d;
+        r[i] = j == 0 ? v[0] : j == 1 ? v[1] : j == 2 ? v[2] : j == 3 ? v[3] : 0.f;
+    }
+    return make_float4(r[0], r[1], r[2], r[3]);
+}
+
+// this thread's VPT adjacent A records (apos) from a stage: code words + dequantised values,
+// and (VPT == 4) the 4 band offsets packed in one word
+template <int VPT, bool U8>
+__device__ __forceinline__ void load_records(const unsigned char* stg, int off_in_stage, int tp,
+                                             uint32_t (&cw)[VPT], float4 (&f)[VPT], uint32_t& ob)
+{
+    if (U8) {
+        if (VPT == 4) {
+            const uint4 c4 = ((const uint4*)stg)[tp];
+            cw[0] = c4.x;
+            cw[VPT > 1 ? 1 : 0] = c4.y;
+            cw[VPT > 2 ? 2 : 0] = c4.z;
+            cw[VPT > 3 ? 3 : 0] = c4.w;
+        } else {
+#pragma unroll
+            for (int t = 0; t < VPT; ++t) cw[t] = ((const uint32_t*)stg)[tp * VPT + t];
+        }
+#pragma unroll
+        for (int t = 0; t < VPT; ++t) f[t] = make_float4(dq(cw[t], 0), dq(cw[t], 1), dq(cw[t], 2), dq(cw[t], 3));
+    } else {
+#pragma unroll
+        for (int t = 0; t < VPT; ++t) {
+            f[t] = ((const float4*)stg)[tp * VPT + t];
+            cw[t] = 0u;
+        }
+    }
+    if (VPT == 4) ob = ((const uint32_t*)(stg + off_in_stage))[tp];
+}
+
+// prior warp: PriPair for voxels (i0, i0+1) of the visiting order from the current x tile
+__device__ __forceinline__ void prior_pair(const int* tof, int i0, int nact, const float* xt, int cslot,
+                                           int TW, int gx0, int gy0, int zg, const IcdParams& P,
+                                           int ndx, int ndy, int ndz, float nbw, int lane, int nnb,
+                                           PriPair* out)
+{
+    const int ta = tof[i0];
+    float s0, x0, bt0, xr0, v0;
+    prior_terms(ta, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, nnb, s0, x0, bt0, xr0, v0);
+    PriPair pp{s0, x0, v0, 0.f, 0.f, 0.f, 0.f, 0.f};
+    if (i0 + 1 < nact) {
+        const int tb = tof[i0 + 1];
+        float s1, x1, bt1, xr1, v1;
+        prior_terms(tb, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, nnb, s1, x1, bt1, xr1, v1);
+        pp.sb = s1;
+        pp.sxb = x1;
+        pp.vb = v1;
+        const int dx = (ta & 255) - (tb & 255), dy = (ta >> 8) - (tb >> 8);
+        if (dx >= -1 && dx <= 1 && dy >= -1 && dy <= 1) {
+            const bool mine = lane < nnb && ndx == dx && ndy == dy && ndz == 0;
+            const int src = __ffs(__ballot_sync(0xffffffffu, mine)) - 1;
+            pp.btab = __shfl_sync(0xffffffffu, bt1, src);
+            pp.bab = __shfl_sync(0xffffffffu, nbw, src);
+        }
+    }
+    if (lane == 0) *out = pp;
+}
+
 // ---- TMA (cp.async.bulk) + mbarrier helpers for the A-record ring ----
 __device__ __forceinline__ uint32_t smem_u32(const void* p)
 {
@@ -187,8 +274,8 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.list = o;  o = align16(o + S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
     L.tof = o;   o = align16(o + S2 * 4);
-    L.red = o;   o = align16(o + 2 * 16 * 4);
-    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriSlot));
+    L.red = o;   o = align16(o + 2 * 24 * 4);  // [2 bufs][3 quantities][8 warps]
+    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriPair));
     L.vscale = o; o = align16(o + S2 * 4);
     L.vth2 = o;  o = align16(o + S2 * 4);
     L.misc = o;  o = align16(o + 16 * 4);
@@ -216,7 +303,7 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     int* flags = (int*)(smem + L.flags);
     int* tof = (int*)(smem + L.tof);  // visiting order as packed (ly << 8 | lx)
     float* red = (float*)(smem + L.red);
-    PriSlot* pri = (PriSlot*)(smem + L.pri);
+    PriPair* pri = (PriPair*)(smem + L.pri);
     float* vscale = (float*)(smem + L.vscale);
     float* vth2 = (float*)(smem + L.vth2);
     uint64_t* mbar = (uint64_t*)(smem + L.mbar);
@@ -228,7 +315,7 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     const bool is_prior = warp == nvw;
     const uint32_t stage_tx = (uint32_t)(VA * (U8 ? 4 : 16) + VA);
 
-    if (threadIdx.x < 32) red[threadIdx.x] = 0.f;  // slots >= nvw stay zero
+    if (threadIdx.x < 48) red[threadIdx.x] = 0.f;  // slots >= nvw stay zero
     if (threadIdx.x == 0) {
         for (int s = 0; s < R; ++s) mbar_init(mbar + s, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -458,150 +545,172 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
         __syncthreads();
 
         if (P.tprof && threadIdx.x == 0) tp2 = clock64();
-        // ---- 5. sequential-exact voxel loop, one barrier per voxel
+        // ---- 5. sequential-exact voxel loop, TWO voxels (a, b) per barrier.  Both are gathered
+        //         from the same state of e, together with the overlap H = sum w A_b A_a over their
+        //         shared sinogram entries; after the barrier every warp computes delta_a, then
+        //         theta1_b corrected for a's update (theta1_b' = theta1_b + s_b s_a delta_a H, the
+        //         exact change of e between them), the prior of b corrected if a is b's
+        //         neighbour, then delta_b -- exactly sequential ICD in the visiting order.
         float amount = 0.f;
         const int cslot = (zc * TW + 1) * TW + 1;  // tile index of local (0,0)
-        for (int idx = 0; idx < nact; ++idx) {
-            const int buf = idx & 1;
+        for (int idx = 0; idx < nact; idx += 2) {
+            const int buf = (idx >> 1) & 1;
+            const bool hasb = idx + 1 < nact;
             const uint32_t g = gseq + idx;
-            const unsigned char* stg = astage + (g % R) * L.stage_bytes;
-            // live across the barrier per view: e values, band offset and the A record (the raw
-            // 32-bit code word in u8 mode -- re-dequantised for the scatter, saving registers)
-            float ev[VPT][4];
-            float4 a4v[VPT];  // dequantised A values of this voxel's 4 channels per view
-            int oo[VPT];
+            const unsigned char* sta = astage + (g % R) * L.stage_bytes;
+            const unsigned char* stb = astage + ((g + 1) % R) * L.stage_bytes;
+            float ea[VPT][4], eb[VPT][4];
+            float4 fa[VPT], fb[VPT];  // dequantised A of voxel a / b on its own 4 channels
+            float4 fab[VPT];          // A of voxel a on b's 4 channels
+            uint32_t ca[VPT], cb[VPT];
+            int oa[VPT], ob[VPT];
             if (warp < nvw) {
-                float t1 = 0.f;
-                // this thread's VPT A records are adjacent (apos): one vector load of codes
-                // and one of band offsets
+                float ga = 0.f, gb = 0.f, hh = 0.f;
                 const int tp = warp * 32 + lane;
-                uint32_t cwa[VPT], oba = 0;
-                if (U8) {
-                    if (VPT == 4) {
-                        const uint4 c4 = ((const uint4*)stg)[tp];
-                        cwa[0] = c4.x;
-                        cwa[VPT > 1 ? 1 : 0] = c4.y;
-                        cwa[VPT > 2 ? 2 : 0] = c4.z;
-                        cwa[VPT > 3 ? 3 : 0] = c4.w;
-                    } else {
-#pragma unroll
-                        for (int t = 0; t < VPT; ++t) cwa[t] = ((const uint32_t*)stg)[tp * VPT + t];
-                    }
-                }
-                if (VPT == 4)
-                    oba = ((const uint32_t*)(stg + L.off_in_stage))[tp];
+                uint32_t oba = 0, obb = 0;
+                load_records<VPT, U8>(sta, L.off_in_stage, tp, ca, fa, oba);
+                if (hasb) load_records<VPT, U8>(stb, L.off_in_stage, tp, cb, fb, obb);
 #pragma unroll
                 for (int t = 0; t < VPT; ++t) {
-                    if (kval[t]) {
-                        const int o = VPT == 4 ? (int)((oba >> (8 * t)) & 255u) : (int)stg[L.off_in_stage + tp * VPT + t];
-                        oo[t] = o;
-                        if (U8) {
-                            const uint32_t cw = cwa[t];
-                            a4v[t] = make_float4(dq(cw, 0), dq(cw, 1), dq(cw, 2), dq(cw, 3));
-                        } else {
-                            a4v[t] = ((const float4*)stg)[tp * VPT + t];
-                        }
-                        const float av[4] = {a4v[t].x, a4v[t].y, a4v[t].z, a4v[t].w};
-                        const float* pe = sb_e + o * Vs + kv[t];
-                        const float* pw = sb_w + o * Vs + kv[t];
-                        float acc = 0.f;
+                    // padded views (k >= V) have zero A and zero-filled SVB columns: harmless,
+                    // so there is no per-view branch
+                    oa[t] = VPT == 4 ? (int)((oba >> (8 * t)) & 255u) : (int)sta[L.off_in_stage + tp * VPT + t];
+                    const float va[4] = {fa[t].x, fa[t].y, fa[t].z, fa[t].w};
+                    const float* pe = sb_e + oa[t] * Vs + kv[t];
+                    const float* pw = sb_w + oa[t] * Vs + kv[t];
+                    float acc = 0.f;
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        ea[t][i] = pe[i * Vs];
+                        acc = fmaf(pw[i * Vs] * ea[t][i], va[i], acc);
+                    }
+                    ga += acc;
+                    if (hasb) {
+                        ob[t] = VPT == 4 ? (int)((obb >> (8 * t)) & 255u) : (int)stb[L.off_in_stage + tp * VPT + t];
+                        const float vb[4] = {fb[t].x, fb[t].y, fb[t].z, fb[t].w};
+                        fab[t] = shifted<U8>(ca[t], fa[t], ob[t] - oa[t]);  // A_a on b's channels
+                        const float vab[4] = {fab[t].x, fab[t].y, fab[t].z, fab[t].w};
+                        const float* qe = sb_e + ob[t] * Vs + kv[t];
+                        const float* qw = sb_w + ob[t] * Vs + kv[t];
+                        float accb = 0.f, acch = 0.f;
 #pragma unroll
                         for (int i = 0; i < 4; ++i) {
-                            ev[t][i] = pe[i * Vs];
-                            acc = fmaf(pw[i * Vs] * ev[t][i], av[i], acc);
+                            eb[t][i] = qe[i * Vs];
+                            const float wab = qw[i * Vs] * vb[i];
+                            accb = fmaf(wab, eb[t][i], accb);
+                            acch = fmaf(wab, vab[i], acch);
                         }
-                        t1 += acc;
+                        gb += accb;
+                        hh += acch;
                     }
                 }
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) t1 += __shfl_xor_sync(kFull, t1, o);
-                if (lane == 0) red[buf * 16 + warp] = t1;
-            } else if (warp == nvw) {
-                // prior warp: the surrogate terms of voxel idx were published after barrier idx-1
-                // (speculatively, then corrected); only voxel 0 is computed here
-                if (idx == 0) {
-                    float sbv, sbx, bt, xr, v;
-                    prior_terms(tof[0], xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
-                                sbv, sbx, bt, xr, v);
-                    if (lane == 0) pri[0] = PriSlot{sbv, sbx, v, 0.f};
+                for (int o = 16; o > 0; o >>= 1) {
+                    ga += __shfl_xor_sync(kFull, ga, o);
+                    gb += __shfl_xor_sync(kFull, gb, o);
+                    hh += __shfl_xor_sync(kFull, hh, o);
                 }
+                if (lane == 0) {
+                    red[buf * 24 + warp] = ga;
+                    red[buf * 24 + 8 + warp] = gb;
+                    red[buf * 24 + 16 + warp] = hh;
+                }
+            } else if (warp == nvw) {
+                // prior warp: the surrogate terms of this pair were published after the previous
+                // barrier; only the first pair is computed here
+                if (idx == 0) prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB, pri);
             } else if (lane == 0) {
-                // producer warp: the next voxel's A records must have landed before the barrier
-                if (idx + 1 < nact) mbar_wait(mbar + (g + 1) % R, ((g + 1) / R) & 1);
+                // producer warp: the next pair's A records must have landed before the barrier
+                if (idx + 2 < nact) mbar_wait(mbar + (g + 2) % R, ((g + 2) / R) & 1);
+                if (idx + 3 < nact) mbar_wait(mbar + (g + 3) % R, ((g + 3) / R) & 1);
             }
             __syncthreads();
-            // every warp derives the same delta (identical inputs, identical order)
-            const float4* r4 = (const float4*)(red + buf * 16);  // nvw <= 8 partials, rest 0
-            const float4 a0 = r4[0], a1 = r4[1];
-            const float s1 = ((a0.x + a0.y) + (a0.z + a0.w)) + ((a1.x + a1.y) + (a1.z + a1.w));
-            const PriSlot ps = pri[buf];
-            const float scale = vscale[idx];
-            const float theta1 = -scale * s1;   // Alg1:5, theta1 = -sum w A e
-            const float theta2 = vth2[idx];     // Alg1:6, precomputed sum w A^2
-            const float num = theta2 * ps.v - theta1 + 2.f * ps.sbx;
-            const float den = theta2 + 2.f * ps.sb;
-            float unew = den > 0.f ? __fdividef(num, den) : ps.v;
-            if (c_prior.positivity) unew = fmaxf(unew, 0.f);
-            const float delta = unew - ps.v;  // Alg1:7-8
+            // every warp derives the same two deltas (identical inputs, identical order)
+            const float* rb = red + buf * 24;  // nvw <= 8 partials per quantity, rest 0
+            const float sa = sum8(rb), sbs = sum8(rb + 8), sh = sum8(rb + 16);
+            const PriPair pp = pri[buf];
+            const float scale_a = vscale[idx];
+            float ua = pp.va;
+            {
+                const float theta1 = -scale_a * sa;  // Alg1:5
+                const float theta2 = vth2[idx];      // Alg1:6 (precomputed)
+                const float num = theta2 * pp.va - theta1 + 2.f * pp.sxa;
+                const float den = theta2 + 2.f * pp.sa;
+                if (den > 0.f) ua = __fdividef(num, den);
+                if (c_prior.positivity) ua = fmaxf(ua, 0.f);
+            }
+            const float da = ua - pp.va;  // Alg1:7-8
+            float ub = pp.vb, db = 0.f, scale_b = 0.f;
+            if (hasb) {
+                scale_b = vscale[idx + 1];
+                // e after a's update: sum w A_b e' = s_b (S_b - s_a delta_a H)
+                const float theta1 = -scale_b * fmaf(-scale_a * da, sh, sbs);
+                const float theta2 = vth2[idx + 1];
+                float psb = pp.sb, psx = pp.sxb;
+                if (pp.bab != 0.f) {  // a is b's neighbour: its term with a's new value
+                    const float bn = pp.bab * phi_f(pp.vb - ua);
+                    psb += bn - pp.btab;
+                    psx += bn * ua - pp.btab * pp.va;
+                }
+                const float num = theta2 * pp.vb - theta1 + 2.f * psx;
+                const float den = theta2 + 2.f * psb;
+                if (den > 0.f) ub = __fdividef(num, den);
+                if (c_prior.positivity) ub = fmaxf(ub, 0.f);
+                db = ub - pp.vb;
+            }
             if (warp < nvw) {
-                if (delta != 0.f) {  // Alg1:9-11: e -= A delta on this thread's views
-                    const float sd = scale * delta;
+                // Alg1:9-11 for both voxels on this thread's views: a's channels first with a's
+                // update, then b's channels with both updates -- b's path rewrites the entries the
+                // two voxels share with the full value, so A_b is never needed on a's channels
+                const float sda = scale_a * da, sdb = scale_b * db;
+                if (sda != 0.f || sdb != 0.f) {
 #pragma unroll
-                    for (int t = 0; t < VPT; ++t)
-                        if (kval[t]) {
-                            float* pe = sb_e + oo[t] * Vs + kv[t];
+                    for (int t = 0; t < VPT; ++t) {
+                        const float va[4] = {fa[t].x, fa[t].y, fa[t].z, fa[t].w};
+                        float* pe = sb_e + oa[t] * Vs + kv[t];
 #pragma unroll
-                            for (int i = 0; i < 4; ++i) {
-                                const float a = i == 0 ? a4v[t].x : i == 1 ? a4v[t].y : i == 2 ? a4v[t].z : a4v[t].w;
-                                pe[i * Vs] = fmaf(-a, sd, ev[t][i]);
-                            }
+                        for (int i = 0; i < 4; ++i) pe[i * Vs] = fmaf(-va[i], sda, ea[t][i]);
+                        if (hasb) {
+                            const float vb[4] = {fb[t].x, fb[t].y, fb[t].z, fb[t].w};
+                            const float vab[4] = {fab[t].x, fab[t].y, fab[t].z, fab[t].w};
+                            float* qe = sb_e + ob[t] * Vs + kv[t];
+#pragma unroll
+                            for (int i = 0; i < 4; ++i) qe[i * Vs] = fmaf(-vb[i], sdb, fmaf(-vab[i], sda, eb[t][i]));
                         }
+                    }
                 }
             } else if (warp == nvw) {
-                // prior warp: surrogate terms of voxel idx+1, computed from the x tile BEFORE
-                // voxel idx's new value is stored (concurrently with delta above), then corrected
-                // for that one neighbour if voxel idx is adjacent to voxel idx+1
-                const int tcur = tof[idx];
-                const int ccur = cslot + (tcur >> 8) * TW + (tcur & 255);
-                if (idx + 1 < nact) {
-                    const int tnext = tof[idx + 1];
-                    float sbv, sbx, bt, xr, v1;
-                    prior_terms(tnext, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
-                                sbv, sbx, bt, xr, v1);
-                    __syncwarp();
-                    if (lane == 0) xt[ccur] = unew;
-                    const int dx = (tcur & 255) - (tnext & 255), dy = (tcur >> 8) - (tnext >> 8);
-                    if (dx >= -1 && dx <= 1 && dy >= -1 && dy <= 1) {
-                        const bool mine = lane < NNB && ndx == dx && ndy == dy && ndz == 0;
-                        float c0 = 0.f, c1 = 0.f;
-                        if (mine) {
-                            const float bn = nbw * phi_f(v1 - unew);
-                            c0 = bn - bt;
-                            c1 = bn * unew - bt * xr;
-                        }
-                        const int src = __ffs(__ballot_sync(kFull, mine)) - 1;
-                        sbv += __shfl_sync(kFull, c0, src);
-                        sbx += __shfl_sync(kFull, c1, src);
+                // prior warp: store the pair's new values, then the next pair's surrogate terms
+                if (lane == 0) {
+                    const int ta = tof[idx];
+                    xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
+                    if (hasb) {
+                        const int tb = tof[idx + 1];
+                        xt[cslot + (tb >> 8) * TW + (tb & 255)] = ub;
                     }
-                    if (lane == 0) pri[(idx + 1) & 1] = PriSlot{sbv, sbx, v1, 0.f};
-                } else if (lane == 0) {
-                    xt[ccur] = unew;
+                    amount += fabsf(da) + fabsf(db);
                 }
-                if (lane == 0) amount += fabsf(delta);
+                __syncwarp();
+                if (idx + 2 < nact)
+                    prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
+                               pri + (buf ^ 1));
             } else if (lane == 0) {
-                // producer warp.  This voxel's stage was read by every view warp before the barrier: refill it
-                // with the A records of voxel idx + R (async proxy after generic reads)
-                if (idx + R < nact) {
-                    const uint32_t s = g % R;
-                    unsigned char* dst = astage + s * L.stage_bytes;
-                    const size_t rec = (arec + list[idx + R]) * (size_t)VA;
-                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                    mbar_expect_tx(mbar + s, stage_tx);
-                    if (U8)
-                        tma_load_1d(dst, P.A.codes + rec, VA * 4, mbar + s);
-                    else
-                        tma_load_1d(dst, P.A.vals + rec, VA * 16, mbar + s);
-                    tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, mbar + s);
+                // producer warp: the pair's stages were read by every view warp before the
+                // barrier: refill them with the A records of voxels idx + R, idx + 1 + R
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    if (idx + u + R < nact) {
+                        const uint32_t s = (g + u) % R;
+                        unsigned char* dst = astage + s * L.stage_bytes;
+                        const size_t rec = (arec + list[idx + u + R]) * (size_t)VA;
+                        mbar_expect_tx(mbar + s, stage_tx);
+                        if (U8)
+                            tma_load_1d(dst, P.A.codes + rec, VA * 4, mbar + s);
+                        else
+                            tma_load_1d(dst, P.A.vals + rec, VA * 16, mbar + s);
+                        tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, mbar + s);
+                    }
                 }
             }
         }
@@ -828,7 +937,8 @@ __global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
 }  // namespace
 
 // A-record ring depth (voxels of TMA lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
-constexpr int ring_depth(bool u8) { return u8 ? 8 : 3; }
+// (the pair loop needs >= 4: the current pair's two stages plus the next pair's two)
+constexpr int ring_depth(bool u8) { return u8 ? 8 : 4; }
 
 int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
 {
