@@ -94,6 +94,7 @@ struct mbir_handle {
     double* d_acc = nullptr;
     unsigned long long* h_counters = nullptr;  // pinned [4] (3 counters + sum_delta bits)
     bool have_sino = false;
+    bool x_zero = true;  // the image is known to be all zero (then e = y needs no projection)
     int iter = 0;
     int64_t nnz = 0, a_bytes = 0, band_entries = 0;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -216,7 +217,10 @@ int refresh_error(mbir_handle* h, bool theta2)
 {
     IcdParams p = make_params(h);
     const bool q = h->o.quantize_A != 0;
-    CK(launch_forward(p, q, h->d_y, h->st));
+    if (h->x_zero)  // e = y - A 0
+        CK(cudaMemcpyAsync(h->d_e, h->d_y, sino_elems(h) * 4, cudaMemcpyDeviceToDevice, h->st));
+    else
+        CK(launch_forward(p, q, h->d_y, h->st));
     if (theta2) CK(launch_theta2(p, q, h->st));
     return MBIR_OK;
 }
@@ -237,6 +241,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         if (n_iter >= 0 && it >= n_iter) break;
         if (n_iter < 0 && (double)updates >= target_equits * nvox_total) break;
         h->iter += 1;
+        h->x_zero = false;
         h->kev_used = 0;
         CK(cudaMemsetAsync(h->d_counters, 0, 3 * sizeof(unsigned long long), h->st));
         CK(cudaMemsetAsync(h->d_sum_delta, 0, sizeof(double), h->st));
@@ -727,6 +732,7 @@ int mbir_set_image(mbir_handle* h, const float* x0, int where)
     } else {
         CK(cudaMemsetAsync(h->d_x + pl, 0, pl * h->g.nz_local * 4, h->st));
     }
+    h->x_zero = (x0 == nullptr);
     int r = exchange_halo(h, -1);
     if (r) return r;
     if (h->have_sino) {

@@ -785,36 +785,40 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     }
 }
 
-// theta2[z][sv][slot] = sum_k sum_i w * A^2 (Alg1:6), fixed for a given sinogram.
-// One warp per voxel, lanes over views; reads w straight from HBM (setup-time kernel).
+// theta2[z][sv][slot] = sum_k sum_i w * A^2 (Alg1:6), fixed for a given sinogram.  One block per
+// (SV, slice), one warp per voxel; lanes walk the voxel's A record positions (coalesced) and
+// read w through the read-only path (the SV's band is L1/L2-resident).  Setup-time kernel.
 template <bool U8>
 __global__ void k_theta2(const IcdParams P)
 {
-    const int lane = threadIdx.x & 31;
-    const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-    const int z = blockIdx.y;
-    if (gw >= P.nsv * P.S2) return;
-    const int sv = gw / P.S2, slot = gw % P.S2;
-    const size_t ab = ((size_t)sv * P.S2 + slot) * P.A.VA;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int sv = blockIdx.x, z = blockIdx.y;
     const float* wz = P.w + (size_t)z * P.V * P.M;
-    const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
-    float acc = 0.f;
-    for (int k = lane; k < P.V; k += 32) {
-        const int f = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + apos(k, P.A.vpt)];
-        const int n = P.A.count[ab + apos(k, P.A.vpt)];
-        float a[4];
-        if (U8) {
-            const uint32_t c = P.A.codes[ab + apos(k, P.A.vpt)];
-            for (int i = 0; i < 4; ++i) a[i] = dq(c, i) * sc;
-        } else {
-            const float4 q = P.A.vals[ab + apos(k, P.A.vpt)];
-            a[0] = q.x; a[1] = q.y; a[2] = q.z; a[3] = q.w;
+    const int vpt = P.A.vpt;
+    for (int slot = warp; slot < P.S2; slot += nw) {
+        const size_t ab = ((size_t)sv * P.S2 + slot) * P.A.VA;
+        const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
+        float acc = 0.f;
+        for (int pk = lane; pk < P.A.VA; pk += 32) {  // record positions, coalesced
+            const int qq = pk / vpt, t = pk % vpt;     // inverse of apos()
+            const int k = ((qq >> 5) * vpt + t) * 32 + (qq & 31);
+            if (k >= P.V) continue;
+            const int n = P.A.count[ab + pk];
+            const int o = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + pk];
+            float a[4];
+            if (U8) {
+                const uint32_t c = P.A.codes[ab + pk];
+                for (int i = 0; i < 4; ++i) a[i] = dq(c, i) * sc;
+            } else {
+                const float4 q = P.A.vals[ab + pk];
+                a[0] = q.x; a[1] = q.y; a[2] = q.z; a[3] = q.w;
+            }
+            for (int i = 0; i < 4; ++i)
+                if (i < n) acc += __ldg(wz + (size_t)k * P.M + o + i) * a[i] * a[i];
         }
-        for (int i = 0; i < 4; ++i)
-            if (i < n) acc += wz[(size_t)k * P.M + f + i] * a[i] * a[i];
+        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(kFull, acc, o);
+        if (lane == 0) P.theta2[((size_t)z * P.nsv + sv) * P.S2 + slot] = acc;
     }
-    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(kFull, acc, o);
-    if (lane == 0) P.theta2[((size_t)z * P.nsv + sv) * P.S2 + slot] = acc;
 }
 
 // e[z] += -A x[z] for one (slice, SV) per block (e must hold y on entry).  Threads own views;
@@ -829,14 +833,21 @@ __global__ void k_forward(const IcdParams P)
     const int gx0 = bx * P.side, gy0 = by * P.side;
     const int tw = min(P.side, P.nx - gx0), th = min(P.side, P.ny - gy0);
     const size_t plane = (size_t)P.nx * P.ny;
+    float* xs = acc + P.rows * P.Vs;  // [S2] the SV's voxel values
+    bool nz = false;
+    for (int slot = threadIdx.x; slot < P.S2; slot += blockDim.x) {
+        const int lx = slot % P.side, ly = slot / P.side;
+        const float xv = (lx < tw && ly < th) ? P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] : 0.f;
+        xs[slot] = xv;
+        nz |= xv != 0.f;
+    }
+    if (!__syncthreads_or(nz)) return;  // all-zero SV contributes nothing
     for (int i = threadIdx.x; i < P.rows * P.Vs; i += blockDim.x) acc[i] = 0.f;
     __syncthreads();
     bool any = false;
     for (int k = threadIdx.x; k < P.V; k += blockDim.x) {
         for (int slot = 0; slot < P.S2; ++slot) {
-            const int lx = slot % P.side, ly = slot / P.side;
-            if (lx >= tw || ly >= th) continue;
-            const float xv = P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx];
+            const float xv = xs[slot];
             if (xv == 0.f) continue;
             any = true;
             const size_t ai = ((size_t)sv * P.S2 + slot) * P.A.VA + apos(k, P.A.vpt);
@@ -971,12 +982,8 @@ cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int 
 
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st)
 {
-    const int wpb = 8;
-    dim3 grid((p.nsv * p.S2 + wpb - 1) / wpb, p.nz_local);
-    if (quantize)
-        k_theta2<true><<<grid, 32 * wpb, 0, st>>>(p);
-    else
-        k_theta2<false><<<grid, 32 * wpb, 0, st>>>(p);
+    auto k = quantize ? k_theta2<true> : k_theta2<false>;
+    k<<<dim3(p.nsv, p.nz_local), 512, 0, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -985,7 +992,7 @@ cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cu
     cudaError_t e = cudaMemcpyAsync(p.e, y, sizeof(float) * (size_t)p.nz_local * p.V * p.M,
                                     cudaMemcpyDeviceToDevice, st);
     if (e != cudaSuccess) return e;
-    const int smem = p.rows * p.Vs * 4;
+    const int smem = (p.rows * p.Vs + p.S2) * 4;
     auto k = quantize ? k_forward<true> : k_forward<false>;
     e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
