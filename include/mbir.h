@@ -198,8 +198,17 @@ int mbir_probe_update(mbir_handle* h, const int64_t* voxels, int n, float* theta
                       float* theta2, float* delta);
 
 /* Multi-GPU bootstrap: write a fresh 128-byte ncclUniqueId into id (call on rank 0 only).
- * Returns ENOTSUP if the library was built without NCCL. */
+ * Returns ENOTSUP if libnccl.so.2 cannot be loaded. */
 int mbir_nccl_unique_id(void* id128);
+
+/* z-slab halo schedule (host-only, no GPU).  After the half-iteration
+ * that updated the slices of global parity `parity` (0 or 1; -1 = both boundary slices, as after
+ * mbir_set_image), rank `rank` of `nranks` owning global slices [z_offset, z_offset + nz_local)
+ * exchanges boundary slices with its neighbours.  Writes up to 4 operations to ops (int32[4][3]:
+ * peer rank, 1 = send / 0 = receive, local storage slice where 0 is the lower halo, 1..nz_local
+ * the owned slices and nz_local + 1 the upper halo) in the order they are posted inside one NCCL
+ * group, and returns how many (>= 0), or MBIR_EINVAL.  mbir_reconstruct uses exactly this plan. */
+int mbir_halo_plan(int z_offset, int nz_local, int rank, int nranks, int parity, int32_t* ops);
 
 void mbir_destroy(mbir_handle* h);
 const char* mbir_strerror(int code);

@@ -26,8 +26,8 @@ EXPORTS = (
     "mbir_set_image", "mbir_reconstruct", "mbir_iterate", "mbir_get_image",
     "mbir_get_error_sinogram", "mbir_rmse_hu", "mbir_query_sizes", "mbir_get_sysmatrix",
     "mbir_get_sysmatrix_columns",
-    "mbir_probe_update", "mbir_nccl_unique_id", "mbir_destroy", "mbir_strerror",
-    "mbir_last_error",
+    "mbir_probe_update", "mbir_nccl_unique_id", "mbir_halo_plan", "mbir_destroy",
+    "mbir_strerror", "mbir_last_error",
 )
 
 
@@ -128,6 +128,8 @@ def load(path: str = LIB_PATH):
     L.mbir_probe_update.argtypes = [H, vp, C.c_int, vp, vp, vp]
     L.mbir_nccl_unique_id.restype = C.c_int
     L.mbir_nccl_unique_id.argtypes = [vp]
+    L.mbir_halo_plan.restype = C.c_int
+    L.mbir_halo_plan.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, C.c_int, vp]
     L.mbir_destroy.restype = None
     L.mbir_destroy.argtypes = [H]
     L.mbir_strerror.restype = C.c_char_p

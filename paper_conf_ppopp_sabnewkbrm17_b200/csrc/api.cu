@@ -177,19 +177,17 @@ int exchange_halo(mbir_handle* h, int parity)
 {
     if (h->nranks <= 1) return MBIR_OK;
     const size_t pl = plane_elems(h);
-    const int z0 = h->g.z_offset, z1 = h->g.z_offset + h->g.nz_local - 1;
+    int32_t ops[4][3];
+    const int n = mbir_halo_plan(h->g.z_offset, h->g.nz_local, h->rank, h->nranks, parity, &ops[0][0]);
+    if (n < 0) return fail(h, MBIR_EINVAL, "bad halo plan");
     NcclApi& N = nccl();
     CKN(N.GroupStart());
-    // my first slice -> rank-1 (its top halo); my last slice -> rank+1 (its bottom halo)
-    if (h->rank > 0) {
-        if (parity < 0 || (z0 & 1) == parity) CKN(N.Send(h->d_x + 1 * pl, pl, ncclFloat, h->rank - 1, h->comm, h->st));
-        if (parity < 0 || ((z0 - 1) & 1) == parity) CKN(N.Recv(h->d_x, pl, ncclFloat, h->rank - 1, h->comm, h->st));
-    }
-    if (h->rank < h->nranks - 1) {
-        if (parity < 0 || (z1 & 1) == parity)
-            CKN(N.Send(h->d_x + (size_t)h->g.nz_local * pl, pl, ncclFloat, h->rank + 1, h->comm, h->st));
-        if (parity < 0 || ((z1 + 1) & 1) == parity)
-            CKN(N.Recv(h->d_x + (size_t)(h->g.nz_local + 1) * pl, pl, ncclFloat, h->rank + 1, h->comm, h->st));
+    for (int i = 0; i < n; ++i) {
+        float* buf = h->d_x + (size_t)ops[i][2] * pl;
+        if (ops[i][1])
+            CKN(N.Send(buf, pl, ncclFloat, ops[i][0], h->comm, h->st));
+        else
+            CKN(N.Recv(buf, pl, ncclFloat, ops[i][0], h->comm, h->st));
     }
     CKN(N.GroupEnd());
     return MBIR_OK;
@@ -424,6 +422,32 @@ int mbir_nccl_unique_id(void* id128)
     if (N.GetUniqueId(&id) != ncclSuccess) return MBIR_ENCCL;
     memcpy(id128, &id, sizeof(id));
     return MBIR_OK;
+}
+
+int mbir_halo_plan(int z_offset, int nz_local, int rank, int nranks, int parity, int32_t* ops)
+{
+    if (!ops || nz_local < 1 || z_offset < 0 || nranks < 1 || rank < 0 || rank >= nranks || parity < -1 ||
+        parity > 1)
+        return MBIR_EINVAL;
+    const int z0 = z_offset, z1 = z_offset + nz_local - 1;  // my first / last global slice
+    int n = 0;
+    auto add = [&](int peer, int send, int slice) {
+        ops[3 * n] = peer;
+        ops[3 * n + 1] = send;
+        ops[3 * n + 2] = slice;
+        ++n;
+    };
+    // my first slice -> rank-1 (its upper halo), my lower halo <- rank-1's last slice (z0 - 1)
+    if (rank > 0) {
+        if (parity < 0 || (z0 & 1) == parity) add(rank - 1, 1, 1);
+        if (parity < 0 || ((z0 - 1) & 1) == parity) add(rank - 1, 0, 0);
+    }
+    // my last slice -> rank+1 (its lower halo), my upper halo <- rank+1's first slice (z1 + 1)
+    if (rank < nranks - 1) {
+        if (parity < 0 || (z1 & 1) == parity) add(rank + 1, 1, nz_local);
+        if (parity < 0 || ((z1 + 1) & 1) == parity) add(rank + 1, 0, nz_local + 1);
+    }
+    return n;
 }
 
 void mbir_destroy(mbir_handle* h)
