@@ -146,9 +146,22 @@ def cpu_baseline(budget_s=12.0):
                       f"{int(Aq.count.sum() / (cfg.n * cfg.n))} nnz/voxel), {upd} updates in {el:.1f} s"}
 
 
+def workload_config(cfg, side, args, world):
+    """The `config` object of both arms (the reference arm times a bounded sample of it)."""
+    sino_gb = 3 * cfg.nz * cfg.nviews * cfg.nchannels * 4 / 1e9
+    return {"workload": f"{cfg.name}: {cfg.n}x{cfg.n}x{cfg.nz} volume, {cfg.nviews} views x "
+                        f"{cfg.nchannels} channels parallel-beam 3-D Shepp-Logan, Poisson "
+                        f"(lambda0=1e4), q-GGMRF {cfg.nbhd}-nbhd, SV side {side}",
+            "equits_per_step": args.equits, "slab_slices_per_gpu": cfg.nz // world,
+            "parallelism": f"z-slab x{world}", "batch_svs": args.batch_svs,
+            "l2": "inputs larger than L2 (uint8 A ~1 GB + y, w, e %.2f GB, no flush needed)" % sino_gb}
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return
+    from synth import CONFIGS
+    cfg_full = CONFIGS[args.config]
     O, og, Aq, pr, case, cfg = oracle_sample_setup()
     for _ in range(args.warmup):
         oracle_time(O, og, Aq, pr, case, 0.5)
@@ -162,10 +175,11 @@ def run_reference(args, rank, world):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot_t / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "impl": "reference",
-            "config": {"workload": "cfg4 per-update work, bounded sample (128x128 slice at config-4 "
-                                   "pitch, 720 views x 256 channels)"},
+            "config": workload_config(cfg_full, args.sv_side or cfg_full.sv_side, args, world),
             "cpu_baseline": {"value": v, "unit": "voxel updates/s", "cores": 1, "kind": "oracle",
-                             "sample": "each step: >= 3 s of sequential-oracle equits on the sample"},
+                             "sample": "each step: >= 3 s of sequential-oracle equits on a bounded "
+                                       "sample of the workload's per-update work: a 128x128 slice "
+                                       "at config-4 pitch (0.5 mm), 720 views x 256 channels"},
             "e2e": {"value": v, "unit": "voxel updates/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -185,6 +199,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_ppopp_sabnewkbrm17_b200 as M
+    from paper_conf_ppopp_sabnewkbrm17_b200 import dist as D
     from synth import CONFIGS, make_sinogram_torch
 
     torch.cuda.set_device(local)
@@ -194,9 +209,7 @@ def main():
     cfg = CONFIGS[args.config]
     side = args.sv_side or cfg.sv_side
     nz = cfg.nz
-    assert nz % world == 0, "slices must divide evenly across ranks"
-    nzl = nz // world
-    z0 = rank * nzl
+    z0, nzl = D.slab(nz, world, rank)
     stream = torch.cuda.current_stream(dev)
 
     t_setup = time.perf_counter()
@@ -205,13 +218,7 @@ def main():
                    z_offset=z0, nz_total=nz)
     pr = M.Prior(sigma=cfg.sigma, neighborhood=cfg.nbhd)
     opt = M.Options(sv_side=side, batch_svs=args.batch_svs)
-    nccl_id = None
-    if world > 1:
-        buf = torch.zeros(128, dtype=torch.uint8, device=dev)
-        if rank == 0:
-            buf.copy_(torch.frombuffer(bytearray(M.mbir_nccl_unique_id()), dtype=torch.uint8))
-        dist.broadcast(buf, 0)
-        nccl_id = bytes(buf.cpu().numpy().tobytes())
+    nccl_id = D.broadcast_nccl_id() if world > 1 else None
     r = M.Reconstructor(g, pr, opt, device=local, stream=stream.cuda_stream, rank=rank,
                         nranks=world, nccl_id=nccl_id)
     r.set_sinogram(y, w)
@@ -334,13 +341,7 @@ def main():
             "ms_per_step": 1000 * el / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32 (A uint8)",
             "data": "synthetic",
-            "config": {"workload": f"{cfg.name}: {cfg.n}x{cfg.n}x{cfg.nz} volume, {cfg.nviews} views x "
-                                   f"{cfg.nchannels} channels parallel-beam 3-D Shepp-Logan, Poisson "
-                                   f"(lambda0=1e4), q-GGMRF 26-nbhd, SV side {side}",
-                       "equits_per_step": args.equits, "slab_slices_per_gpu": nzl,
-                       "parallelism": f"z-slab x{world}", "batch_svs": args.batch_svs,
-                       "l2": "inputs larger than L2 (A %.2f GB + sinograms %.2f GB)" % (
-                           sizes["a_bytes"] / 1e9, 3 * y.numel() * 4 * world / 1e9)},
+            "config": workload_config(cfg, side, args, world),
             "updates_per_step": updates / args.steps,
             "time_to_converge": conv,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,

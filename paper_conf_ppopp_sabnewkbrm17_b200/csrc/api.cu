@@ -345,7 +345,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         st->kernel_launches = klaunches;
     }
     if (h->d_tprof) {  // development aid: per-phase cycles of the update kernel (thread 0 of each CTA)
-        unsigned long long t[16];
+        unsigned long long t[32];
         cudaMemcpy(t, h->d_tprof, sizeof(t), cudaMemcpyDeviceToHost);
         cudaMemset(h->d_tprof, 0, sizeof(t));
         const double v = (double)(t[5] ? t[5] : 1);
@@ -355,6 +355,11 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
                 "land %.0f stage %.0f)\n",
                 t[5], t[4], t[0] / v, t[1] / v, t[2] / v, t[3] / v, t[2] / (double)(t[4] ? t[4] : 1),
                 t[6] / v, t[7] / v, t[8] / v, t[9] / v);
+        fprintf(stderr, "[mbir phase] barrier wait cycles/visit by warp:");
+        for (int i = 0; i < 8; ++i) fprintf(stderr, " %.0f", t[10 + i] / v);
+        fprintf(stderr, " | producer loop %.0f | view full-wait (records < R, >= R) %.0f %.0f | prior_pair %.0f",
+                t[21] / v, t[22] / v, t[23] / v, t[24] / v);
+        fprintf(stderr, "\n");
     }
     return MBIR_OK;
 }
@@ -601,6 +606,8 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         return (fail(h, MBIR_EINVAL, "SV band needs " + std::to_string(h->rows) + " > 29 buffer rows: reduce sv_side"), bail(MBIR_EINVAL));
     if (((size_t)G.nviews * G.nchannels) % 4 != 0)
         return (fail(h, MBIR_EINVAL, "nviews * nchannels must be a multiple of 4"), bail(MBIR_EINVAL));
+    if ((size_t)G.nviews * G.nchannels >= (size_t(1) << 27))  // band row offsets are packed << 5
+        return (fail(h, MBIR_EINVAL, "nviews * nchannels must be < 2^27"), bail(MBIR_EINVAL));
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
     h->threads = 32 * (h->nvw + 2);  // view warps + prior warp + TMA producer warp
@@ -653,8 +660,8 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_flag, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_acc, 1))) return bail(r);
     if (getenv("MBIR_PHASE_PROFILE")) {
-        if ((r = dalloc(h, &h->d_tprof, 16))) return bail(r);
-        cudaMemset(h->d_tprof, 0, 16 * sizeof(unsigned long long));
+        if ((r = dalloc(h, &h->d_tprof, 32))) return bail(r);
+        cudaMemset(h->d_tprof, 0, 32 * sizeof(unsigned long long));
     }
     if (cudaMallocHost((void**)&h->h_counters, 4 * sizeof(unsigned long long)) != cudaSuccess) return bail(MBIR_ENOMEM);
     cudaMemsetAsync(h->d_x, 0, sizeof(float) * pl * (G.nz_local + 2), h->st);

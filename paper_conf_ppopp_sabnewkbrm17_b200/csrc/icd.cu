@@ -108,10 +108,15 @@ struct PriSlot {
 // lane r < nnb owns neighbour r (offset ndx/ndy/ndz, weight nbw); returns the warp-reduced
 // sums sbv = sum b_r phi(v - x_r) and sbx = sum b_r phi(v - x_r) x_r, plus this lane's own
 // (bt, xr) and the voxel's value v.  Free boundary: off-image neighbours contribute nothing.
+// Neighbours at packed tile positions ov0 / ov1 (same slice) take the values xv0 / xv1 instead
+// of the tile's: the voxels just updated, whose new values the calling warp holds in registers
+// before they are stored to the tile.
 __device__ __forceinline__ void prior_terms(int tofv, const float* xt, int cslot, int TW, int gx0,
                                             int gy0, int zg, const IcdParams& P, int ndx, int ndy,
                                             int ndz, float nbw, int lane, int nnb, float& sbv,
-                                            float& sbx, float& bt, float& xr, float& v)
+                                            float& sbx, float& bt, float& xr, float& v,
+                                            int ov0 = -1 << 20, float xv0 = 0.f, int ov1 = -1 << 20,
+                                            float xv1 = 0.f)
 {
     const int lx = tofv & 255, ly = tofv >> 8;
     v = xt[cslot + ly * TW + lx];
@@ -121,6 +126,9 @@ __device__ __forceinline__ void prior_terms(int tofv, const float* xt, int cslot
         const int gx = gx0 + lx + ndx, gy = gy0 + ly + ndy, gz = zg + ndz;
         if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
             xr = xt[cslot + (ndz * TW + ly + ndy) * TW + lx + ndx];
+            const int pos = ndz == 0 ? ((ly + ndy) << 8) + lx + ndx : -2 << 20;
+            if (pos == ov0) xr = xv0;
+            if (pos == ov1) xr = xv1;
             bt = nbw * phi_f(v - xr);
         }
     }
@@ -139,35 +147,59 @@ struct PriPair {
     float sa, sxa, va, sb, sxb, vb, btab, bab;
 };
 
+// sum of 8 consecutive floats (16-byte aligned) with paired-fp32 adds
 __device__ __forceinline__ float sum8(const float* r)
 {
     const float4 a = ((const float4*)r)[0], b = ((const float4*)r)[1];
-    return ((a.x + a.y) + (a.z + a.w)) + ((b.x + b.y) + (b.z + b.w));
+    const float2 s = __fadd2_rn(__fadd2_rn(make_float2(a.x, a.y), make_float2(a.z, a.w)),
+                                __fadd2_rn(make_float2(b.x, b.y), make_float2(b.z, b.w)));
+    return s.x + s.y;
 }
 
-// A values of a voxel re-indexed to another voxel's channels: result[i] = A[i + d] (0 outside)
+template <bool B>
+struct BoolTag {
+    static constexpr bool value = B;
+};
+
+// dequantised codes i, i + 1 of a packed word as a channel pair: 2 PRMT + 1 FADD2
+__device__ __forceinline__ float2 dq2(uint32_t word, int i)
+{
+    const float2 m = make_float2(__uint_as_float(__byte_perm(word, 0x4B000000u, 0x7440u | (uint32_t)i)),
+                                 __uint_as_float(__byte_perm(word, 0x4B000000u, 0x7441u + (uint32_t)i)));
+    return __fadd2_rn(m, make_float2(-8388608.f, -8388608.f));
+}
+
+// A values of a voxel re-indexed to another voxel's channels: r[i] = A[i + d] (0 outside), as
+// channel pairs
 template <bool U8>
-__device__ __forceinline__ float4 shifted(uint32_t cw, float4 a, int d)
+__device__ __forceinline__ void shifted(uint32_t cw, const float2 (&a)[2], int d, float2 (&r)[2])
 {
     if (U8) {
-        const uint32_t s = (d >= 4 || d <= -4) ? 0u : (d >= 0 ? (cw >> (8 * d)) : (cw << (-8 * d)));
-        return make_float4(dq(s, 0), dq(s, 1), dq(s, 2), dq(s, 3));
+        // one PRMT: byte i of s = byte i + d of cw, or 0 (selector nibble 4 = byte 0 of the zero
+        // operand); the selector nibbles are read out of 0x444432104444 at nibble 4 + d
+        const int dc = max(-4, min(4, d));
+        const uint32_t sel = (uint32_t)(0x444432104444ull >> (16 + 4 * dc));
+        const uint32_t s = __byte_perm(cw, 0u, sel);
+        r[0] = dq2(s, 0);
+        r[1] = dq2(s, 2);
+        return;
     }
-    const float v[4] = {a.x, a.y, a.z, a.w};
-    float r[4];
+    const float v[4] = {a[0].x, a[0].y, a[1].x, a[1].y};
+    float q[4];
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
         const int j = i + d;
-        r[i] = j == 0 ? v[0] : j == 1 ? v[1] : j == 2 ? v[2] : j == 3 ? v[3] : 0.f;
+        q[i] = j == 0 ? v[0] : j == 1 ? v[1] : j == 2 ? v[2] : j == 3 ? v[3] : 0.f;
     }
-    return make_float4(r[0], r[1], r[2], r[3]);
+    r[0] = make_float2(q[0], q[1]);
+    r[1] = make_float2(q[2], q[3]);
 }
 
-// this thread's VPT adjacent A records (apos) from a stage: code words + dequantised values,
-// and (VPT == 4) the 4 band offsets packed in one word
+// this thread's VPT adjacent A records (apos) from a stage: code words + dequantised values as
+// channel pairs, and (VPT == 4) the 4 band offsets packed in one word
 template <int VPT, bool U8>
 __device__ __forceinline__ void load_records(const unsigned char* stg, int off_in_stage, int tp,
-                                             uint32_t (&cw)[VPT], float4 (&f)[VPT], uint32_t& ob)
+                                             uint32_t (&cw)[VPT], float2 (&f)[VPT][2], uint32_t& ob)
 {
     if (U8) {
         if (VPT == 4) {
@@ -181,11 +213,16 @@ __device__ __forceinline__ void load_records(const unsigned char* stg, int off_i
             for (int t = 0; t < VPT; ++t) cw[t] = ((const uint32_t*)stg)[tp * VPT + t];
         }
 #pragma unroll
-        for (int t = 0; t < VPT; ++t) f[t] = make_float4(dq(cw[t], 0), dq(cw[t], 1), dq(cw[t], 2), dq(cw[t], 3));
+        for (int t = 0; t < VPT; ++t) {
+            f[t][0] = dq2(cw[t], 0);
+            f[t][1] = dq2(cw[t], 2);
+        }
     } else {
 #pragma unroll
         for (int t = 0; t < VPT; ++t) {
-            f[t] = ((const float4*)stg)[tp * VPT + t];
+            const float4 v = ((const float4*)stg)[tp * VPT + t];
+            f[t][0] = make_float2(v.x, v.y);
+            f[t][1] = make_float2(v.z, v.w);
             cw[t] = 0u;
         }
     }
@@ -234,6 +271,10 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes)
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
                  : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar)
+{
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
 {
     asm volatile(
@@ -244,6 +285,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
         "r"(parity)
         : "memory");
 }
+// warm L2 with a global block (bulk prefetch; no completion tracking)
+__device__ __forceinline__ void l2_prefetch_bulk(const void* src, uint32_t bytes)
+{
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar)
 {
     asm volatile(
@@ -253,12 +299,11 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
         : "memory");
 }
 
-struct SmemLayout {
-    int sb_e, sb_w, xt, list, flags, tof, red, pri, vscale, vth2, misc, astage, stage_bytes,
-        off_in_stage, mbar, staging, total;
-};
-
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
+
+// the update kernel's SVB column stride: the most views a launch configuration can hold (6 view
+// warps x 32 lanes x VPT views), fixed at compile time whatever the actual view count
+__host__ __device__ constexpr int svb_stride(int vpt) { return 6 * 32 * vpt; }
 
 // A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
 __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, int S2, int nnb,
@@ -282,10 +327,33 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.off_in_stage = VA * (u8 ? 4 : 16);
     L.stage_bytes = align16(L.off_in_stage + VA);
     L.astage = o; o = align16(o + nstage * L.stage_bytes);
-    L.mbar = o;  o = align16(o + nstage * 8);
-    L.staging = o; o = align16(o + nvw * 32 * 32 * 4);  // one 32x32 transpose tile per view warp
+    L.mbar = o;  o = align16(o + 2 * nstage * 8);  // full[nstage], then empty[nstage]
+    L.staging = o; o = align16(o + nvw * 32 * 33 * 4);  // one 32x33 transpose tile per view warp
+    L.binfo = o; o = align16(o + 2 * VA * 4);           // band (row offset << 5 | width), 2 tasks
     L.total = o;
     return L;
+}
+
+// band of task tk for views k0, k0 + stride, ... < k1 into dst[k] = (k*M + start) << 5 | width;
+// optionally warms L2 with the band's w and e lines (the next task's pack then reads L2)
+__device__ __forceinline__ void band_info(const IcdParams& P, int tk, uint32_t* dst, int k0, int k1,
+                                          int stride, bool prefetch)
+{
+    const int z = tk >> 14, sv = tk & 16383;
+    const float* wz = P.w + (size_t)z * P.V * P.M;
+    const float* ez = P.e + (size_t)z * P.V * P.M;
+    for (int k = k0; k < k1; k += stride) {
+        const int r = k * P.M + P.A.band_start[(size_t)sv * P.V + k];
+        const int wd = P.A.band_width[(size_t)sv * P.V + k];
+        dst[k] = ((uint32_t)r << 5) | (uint32_t)wd;
+        if (prefetch) {
+            const int r1 = r + max(wd, 1) - 1;
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
+        }
+    }
 }
 
 template <int VPT, bool U8, int NNB, int R>
@@ -294,8 +362,16 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int nvw = P.nvw;
-    const int V = P.V, M = P.M, Vs = P.Vs, S2 = P.S2, side = P.side, VA = P.A.VA;
-    const SmemLayout L = smem_layout(P.rows, Vs, side, S2, NNB, VA, U8, R, nvw);
+    // warp roles: nvw view warps, the prior warp and the TMA producer warp.  Warps w and w + 4
+    // share a scheduler (SMSP); with >= 3 view warps the prior warp is warp 3, so it shares
+    // SMSP 3 only with the producer (which mostly sleeps on mbarriers) and the view warps spread
+    // evenly over SMSPs 0-2 (and 3 when nvw is small).
+    const int prior_w = nvw >= 3 ? 3 : nvw, prod_w = nvw + 1;
+    const bool is_prior = warp == prior_w, is_prod = warp == prod_w, is_view = !is_prior && !is_prod;
+    const int vw = is_view ? (warp < prior_w ? warp : warp - 1) : 0;  // view-warp index
+    const int V = P.V, M = P.M, S2 = P.S2, side = P.side, VA = P.A.VA;
+    constexpr int VS = svb_stride(VPT);  // SVB view stride: compile-time, so row offsets are immediates
+    const SmemLayout& L = P.lay;
     float* sb_e = (float*)(smem + L.sb_e);
     float* sb_w = (float*)(smem + L.sb_w);
     float* xt = (float*)(smem + L.xt);
@@ -308,16 +384,23 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     float* vth2 = (float*)(smem + L.vth2);
     uint64_t* mbar = (uint64_t*)(smem + L.mbar);
     unsigned char* astage = smem + L.astage;
-    float* stg_w = (float*)(smem + L.staging) + (warp < nvw ? warp : 0) * 32 * 32;
+    float* stg_w = (float*)(smem + L.staging) + vw * 32 * 33;
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
     const size_t plane = (size_t)P.nx * P.ny;
-    const bool is_prior = warp == nvw;
     const uint32_t stage_tx = (uint32_t)(VA * (U8 ? 4 : 16) + VA);
 
     if (threadIdx.x < 48) red[threadIdx.x] = 0.f;  // slots >= nvw stay zero
+    // SVB rows outside a visit's band are never packed: start them finite (zero)
+    for (int i = threadIdx.x; i < (L.sb_w - L.sb_e) / 16; i += blockDim.x) {
+        ((float4*)(smem + L.sb_e))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        ((float4*)(smem + L.sb_w))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    }
     if (threadIdx.x == 0) {
-        for (int s = 0; s < R; ++s) mbar_init(mbar + s, 1);
+        for (int s = 0; s < R; ++s) {
+            mbar_init(mbar + s, 1);          // full: the producer's arrive + the TMA bytes
+            mbar_init(mbar + R + s, nvw);    // empty: one arrive per view warp
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     // per-thread view ownership: warp w, lane l owns views (w*VPT + t)*32 + l
@@ -325,8 +408,8 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     bool kval[VPT];
 #pragma unroll
     for (int t = 0; t < VPT; ++t) {
-        kv[t] = (warp * VPT + t) * 32 + lane;
-        kval[t] = warp < nvw && kv[t] < V;
+        kv[t] = (vw * VPT + t) * 32 + lane;
+        kval[t] = is_view && kv[t] < V;
     }
     uint32_t gseq = 0;  // running voxel sequence number of this CTA: A stage = gseq % R
     // prior-warp lane r owns neighbour r: its offset and weight live in registers (a per-lane
@@ -344,10 +427,13 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     // pulled one at a time by the persistent CTAs (dynamic distribution, Alg3:4 / T3)
     const int tstart = P.brange[0], tend = P.brange[1];
     int* s_task = (int*)(smem + L.misc);  // [0] first task, [1] next task (fetched one ahead)
+    uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA]: this task's / the next task's band
     if (threadIdx.x == 0) s_task[0] = tstart + atomicAdd(P.fetch, 1);
     __syncthreads();
     int q = s_task[0];
-    for (;; q = s_task[1]) {
+    if (q < tend) band_info(P, P.flat[q], binfo, threadIdx.x, V, blockDim.x, false);
+    int tb = 0;  // binfo buffer of the current task
+    for (;; q = s_task[1], tb ^= 1) {
         if (q >= tend) break;
         const int tk = P.flat[q];
         const int z = tk >> 14, sv = tk & 16383;  // local slice, SV
@@ -398,7 +484,8 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                 s_task[1] = tstart + atomicAdd(P.fetch, 1);
             }
             __syncthreads();
-            continue;
+            if (s_task[1] < tend) band_info(P, P.flat[s_task[1]], binfo + (tb ^ 1) * VA, threadIdx.x, V, blockDim.x, false);
+            continue;  // the next task's x-tile barrier orders these writes before its pack
         }
 
         // ---- 3. visiting order: random permutation of the tile, compacted to the kept
@@ -443,104 +530,103 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                         tma_load_1d(dst, P.A.vals + rec, VA * 16, mbar + s);
                     tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, mbar + s);
                 }
+                // and warm L2 with the next R records: every record is L2-prefetched R voxels
+                // before its TMA (the producer continues this R ahead during the loop)
+                for (int i = R; i < 2 * R && i < nact; ++i) {
+                    const size_t rec = (arec + list[i]) * (size_t)VA;
+                    l2_prefetch_bulk(U8 ? (const void*)(P.A.codes + rec) : (const void*)(P.A.vals + rec), VA * (U8 ? 4 : 16));
+                    l2_prefetch_bulk(P.A.off + rec, VA);
+                }
             }
         }
 
         if (P.tprof && threadIdx.x == 0) tp1 = clock64();
         // ---- 4. view threads: SVB pack (coalesced 128-byte band rows, transposed by shuffles);
         //         e_init rows go to this CTA's L2-resident scratch tile for the write-back
-        float* scr = P.scratch + (size_t)blockIdx.x * (size_t)Vs * 32;
-        if (warp < nvw) {
+        float* scr = P.scratch + (size_t)blockIdx.x * (size_t)P.Vs * 32;
+        int pf_task = -1;  // producer warp: the next task (its band info is loaded during the loop)
+        if (is_view) {
             const float* wz = P.w + (size_t)z * V * M;
             float* ez = P.e + (size_t)z * V * M;
             // Each band row is read as the 16-byte-aligned 32-float window that contains it (the
             // slice base is 16-byte aligned, V*M % 4 == 0): 8 lanes x float4 per row, 4 rows per
             // LDG.128, so a 32-view tile of w and e is 16 vector loads (few requests in flight).
-            // The window is stored rotated in the warp's staging tile -- band column c of row i at
-            // column (c + i) % 32 -- so that lane k then reads row k's column c at (c + k) % 32
-            // (banks distinct over k) and writes sb[c][k] (banks distinct over k): conflict-free.
+            // The windows go through the warp's staging tile with a row stride of 33 floats: the
+            // put (lanes span window position p = 4ch + j and row i = 4m + sub) and the read (lane
+            // k walks its own row's positions) both touch 32 distinct banks, and band column
+            // c = p - s_k goes to sb[c][k] (bank k).  Only band columns are written: the rows past
+            // a view's band keep finite stale values that only ever meet zero A entries.
             // e_init windows go to this CTA's L2-resident scratch tile for the write-back.
-            int bwv[VPT], rov[VPT];
-#pragma unroll
-            for (int t = 0; t < VPT; ++t) {
-                const int kk = (warp * VPT + t) * 32 + lane;
-                bwv[t] = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
-                rov[t] = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
-            }
+            // Two tiles are in flight: tile t + 1's loads are issued before tile t is staged.
             const int sub = lane >> 3, ch = lane & 7;  // row-in-quad and float4 chunk of this lane
-#pragma unroll 1
-            for (int t = 0; t < VPT; ++t) {
-                const int k0 = (warp * VPT + t) * 32;
+            auto issue = [&](int t, bool isw, float4 (&v4)[8]) {
+                const int k0 = (vw * VPT + t) * 32;
                 const int kk = k0 + lane;
-                float4 w4[8], e4[8];
-                int so[8];
+                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const int bwt = (int)(bi & 31u), rot = (int)(bi >> 5);
 #pragma unroll
                 for (int m = 0; m < 8; ++m) {
                     const int i = 4 * m + sub;
-                    const int oi = __shfl_sync(kFull, rov[t], i), wi = __shfl_sync(kFull, bwv[t], i);
+                    const int oi = __shfl_sync(kFull, rot, i), wi = __shfl_sync(kFull, bwt, i);
                     const int s = oi & 3;
-                    so[m] = s;
                     const bool ok = k0 + i < V && 4 * ch < s + wi;
                     const size_t a4 = (size_t)(oi - s) + 4 * ch;
-                    w4[m] = ok ? __ldg((const float4*)(wz + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
-                    e4[m] = ok ? __ldcg((const float4*)(ez + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (isw)
+                        v4[m] = ok ? __ldg((const float4*)(wz + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    else
+                        v4[m] = ok ? __ldcg((const float4*)(ez + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
                 }
+            };
+            auto put = [&](const float4 (&v)[8]) {
+#pragma unroll
+                for (int m = 0; m < 8; ++m) {
+                    const int i = 4 * m + sub;
+                    const float vv[4] = {v[m].x, v[m].y, v[m].z, v[m].w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) stg_w[i * 33 + 4 * ch + j] = vv[j];
+                }
+                __syncwarp();
+            };
+            auto finish = [&](int t, bool isw, const float4 (&v4)[8]) {
+                const int k0 = (vw * VPT + t) * 32;
+                const int kk = k0 + lane;
+                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const int bwt = (int)(bi & 31u), sk = (int)(bi >> 5) & 3;
+                const uint32_t bmask = ((1u << bwt) - 1u) << sk;  // band's window positions
+                if (!isw) {
+#pragma unroll
+                    for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), v4[m]);
+                }
+                float* d = (isw ? sb_w : sb_e) + kk - sk * VS;  // + p * VS = band column p - sk of view kk
+                const float* sr = stg_w + lane * 33;
+                put(v4);
+#pragma unroll
+                for (int p = 0; p < 32; ++p)
+                    if (bmask & (1u << p)) d[p * VS] = sr[p];
+                __syncwarp();
+            };
+#pragma unroll 1
+            for (int t = 0; t < VPT; ++t) {
+                float4 wa[8], ea[8];
+                issue(t, true, wa);
+                issue(t, false, ea);
                 if (P.tprof && threadIdx.x == 0 && t == 0) tpa = clock64();
-#pragma unroll
-                for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), e4[m]);
-                if (P.tprof && threadIdx.x == 0 && t == 0) tpb = clock64();
-                auto put = [&](const float4 (&v)[8]) {
-#pragma unroll
-                    for (int m = 0; m < 8; ++m) {
-                        const int i = 4 * m + sub;
-                        const float vv[4] = {v[m].x, v[m].y, v[m].z, v[m].w};
-#pragma unroll
-                        for (int j = 0; j < 4; ++j) {
-                            const int c = 4 * ch + j - so[m];  // band column
-                            if (c >= 0) stg_w[i * 32 + ((c + i) & 31)] = vv[j];
-                        }
-                    }
-                    __syncwarp();
-                };
-                const int bwk = bwv[t];
-                put(w4);
-#pragma unroll
-                for (int c = 0; c < 32; ++c)
-                    if (c < P.rows) sb_w[c * Vs + kk] = c < bwk ? stg_w[lane * 32 + ((c + lane) & 31)] : 0.f;
-                __syncwarp();
-                put(e4);
-#pragma unroll
-                for (int c = 0; c < 32; ++c)
-                    if (c < P.rows) sb_e[c * Vs + kk] = c < bwk ? stg_w[lane * 32 + ((c + lane) & 31)] : 0.f;
-                __syncwarp();
+                finish(t, true, wa);
+                finish(t, false, ea);
                 if (P.tprof && threadIdx.x == 0 && t == 0) tpc = clock64();
             }
             if (P.tprof && threadIdx.x == 0) tp1b = clock64();
-        } else if (warp == nvw + 1) {
-            // producer warp: fetch the next task now and warm L2 with its band rows, so the
-            // next pack reads L2 instead of HBM (the x tile, scratch and A ring are separate)
+        } else if (is_prod) {
+            // producer warp: fetch the next task now; its band info (and an L2 warm-up of its
+            // band rows) is then produced a slice per voxel pair during the voxel loop, so the
+            // prefetches do not compete with this pack's loads
             int nq = 0;
             if (lane == 0) {
                 nq = tstart + atomicAdd(P.fetch, 1);
                 s_task[1] = nq;
             }
             nq = __shfl_sync(kFull, nq, 0);
-            if (nq < tend) {
-                const int ntk = P.flat[nq];
-                const int nz = ntk >> 14, nsv = ntk & 16383;
-                const float* nw = P.w + (size_t)nz * V * M;
-                const float* ne = P.e + (size_t)nz * V * M;
-                for (int k = lane; k < V; k += 32) {
-                    const int b = P.A.band_start[(size_t)nsv * V + k];
-                    const int wd = max((int)P.A.band_width[(size_t)nsv * V + k], 1);
-                    const size_t o0 = (size_t)k * M + b, o1 = o0 + wd - 1;
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(nw + o0));
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(nw + o1));
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(ne + o0));
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(ne + o1));
-                }
-            }
-            if (lane == 0) mbar_wait(mbar + gseq % R, (gseq / R) & 1);  // first voxel's A landed
+            pf_task = nq < tend ? P.flat[nq] : -1;
         }
         __syncthreads();
 
@@ -553,164 +639,232 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
         //         neighbour, then delta_b -- exactly sequential ICD in the visiting order.
         float amount = 0.f;
         const int cslot = (zc * TW + 1) * TW + 1;  // tile index of local (0,0)
-        for (int idx = 0; idx < nact; idx += 2) {
-            const int buf = (idx >> 1) & 1;
-            const bool hasb = idx + 1 < nact;
-            const uint32_t g = gseq + idx;
-            const unsigned char* sta = astage + (g % R) * L.stage_bytes;
-            const unsigned char* stb = astage + ((g + 1) % R) * L.stage_bytes;
-            float ea[VPT][4], eb[VPT][4];
-            float4 fa[VPT], fb[VPT];  // dequantised A of voxel a / b on its own 4 channels
-            float4 fab[VPT];          // A of voxel a on b's 4 channels
-            uint32_t ca[VPT], cb[VPT];
-            int oa[VPT], ob[VPT];
-            if (warp < nvw) {
-                float ga = 0.f, gb = 0.f, hh = 0.f;
-                const int tp = warp * 32 + lane;
-                uint32_t oba = 0, obb = 0;
-                load_records<VPT, U8>(sta, L.off_in_stage, tp, ca, fa, oba);
-                if (hasb) load_records<VPT, U8>(stb, L.off_in_stage, tp, cb, fb, obb);
+        uint64_t* full = mbar;       // full[s]: stage s holds its record (TMA bytes landed)
+        uint64_t* empty = mbar + R;  // empty[s]: every view warp has read stage s
+        const int npair_threads = (nvw + 1) * 32;  // view warps + prior warp meet per pair
+        if (!is_prod) {
+            for (int idx = 0; idx < nact; idx += 2) {
+                const int buf = (idx >> 1) & 1;
+                const bool hasb = idx + 1 < nact;
+                const uint32_t g = gseq + idx;
+                const unsigned char* sta = astage + (g % R) * L.stage_bytes;
+                const unsigned char* stb = astage + ((g + 1) % R) * L.stage_bytes;
+                // per view t of this thread: e on a's / b's 4 channels, A_a, A_b on their own
+                // channels and A_a on b's channels, as channel pairs (0,1), (2,3) for the
+                // paired-fp32 FFMA2/FMUL2 of sm_100 (one instruction per two channels)
+                float2 ea[VPT][2], eb[VPT][2], fa[VPT][2], fb[VPT][2], fab[VPT][2];
+                int oa[VPT], ob[VPT];
+                if (is_view) {
+                    const int tp = vw * 32 + lane;
+                    // HB: the pair has a second voxel (all but the last step of an odd visit)
+                    auto gather = [&](auto hb) {
+                        constexpr bool HB = decltype(hb)::value;
+                        const long long tf0 = P.tprof ? clock64() : 0;
+                        mbar_wait(full + g % R, (g / R) & 1);  // the records have landed
+                        if (HB) mbar_wait(full + (g + 1) % R, ((g + 1) / R) & 1);
+                        if (P.tprof && lane == 0) atomicAdd(P.tprof + 22 + (idx >= R), (unsigned long long)(clock64() - tf0));
+                        uint32_t ca[VPT], cb[VPT], oba = 0, obb = 0;
+                        load_records<VPT, U8>(sta, L.off_in_stage, tp, ca, fa, oba);
+                        if (HB) load_records<VPT, U8>(stb, L.off_in_stage, tp, cb, fb, obb);
+                        float2 acc = make_float2(0.f, 0.f), accb = acc, acch = acc;
 #pragma unroll
-                for (int t = 0; t < VPT; ++t) {
-                    // padded views (k >= V) have zero A and zero-filled SVB columns: harmless,
-                    // so there is no per-view branch
-                    oa[t] = VPT == 4 ? (int)((oba >> (8 * t)) & 255u) : (int)sta[L.off_in_stage + tp * VPT + t];
-                    const float va[4] = {fa[t].x, fa[t].y, fa[t].z, fa[t].w};
-                    const float* pe = sb_e + oa[t] * Vs + kv[t];
-                    const float* pw = sb_w + oa[t] * Vs + kv[t];
-                    float acc = 0.f;
-#pragma unroll
-                    for (int i = 0; i < 4; ++i) {
-                        ea[t][i] = pe[i * Vs];
-                        acc = fmaf(pw[i * Vs] * ea[t][i], va[i], acc);
-                    }
-                    ga += acc;
-                    if (hasb) {
-                        ob[t] = VPT == 4 ? (int)((obb >> (8 * t)) & 255u) : (int)stb[L.off_in_stage + tp * VPT + t];
-                        const float vb[4] = {fb[t].x, fb[t].y, fb[t].z, fb[t].w};
-                        fab[t] = shifted<U8>(ca[t], fa[t], ob[t] - oa[t]);  // A_a on b's channels
-                        const float vab[4] = {fab[t].x, fab[t].y, fab[t].z, fab[t].w};
-                        const float* qe = sb_e + ob[t] * Vs + kv[t];
-                        const float* qw = sb_w + ob[t] * Vs + kv[t];
-                        float accb = 0.f, acch = 0.f;
-#pragma unroll
-                        for (int i = 0; i < 4; ++i) {
-                            eb[t][i] = qe[i * Vs];
-                            const float wab = qw[i * Vs] * vb[i];
-                            accb = fmaf(wab, eb[t][i], accb);
-                            acch = fmaf(wab, vab[i], acch);
+                        for (int t = 0; t < VPT; ++t) {
+                            // padded views (k >= V) have zero A: no per-view branch
+                            oa[t] = VPT == 4 ? (int)((oba >> (8 * t)) & 255u) : (int)sta[L.off_in_stage + tp * VPT + t];
+                            const float* pe = sb_e + oa[t] * VS + kv[t];
+                            const float* pw = sb_w + oa[t] * VS + kv[t];
+                            ea[t][0] = make_float2(pe[0], pe[VS]);
+                            ea[t][1] = make_float2(pe[2 * VS], pe[3 * VS]);
+                            const float2 w0 = make_float2(pw[0], pw[VS]), w1 = make_float2(pw[2 * VS], pw[3 * VS]);
+                            acc = __ffma2_rn(__fmul2_rn(w0, ea[t][0]), fa[t][0], acc);
+                            acc = __ffma2_rn(__fmul2_rn(w1, ea[t][1]), fa[t][1], acc);
+                            if (HB) {
+                                ob[t] = VPT == 4 ? (int)((obb >> (8 * t)) & 255u) : (int)stb[L.off_in_stage + tp * VPT + t];
+                                shifted<U8>(ca[t], fa[t], ob[t] - oa[t], fab[t]);  // A_a on b's channels
+                                const float* qe = sb_e + ob[t] * VS + kv[t];
+                                const float* qw = sb_w + ob[t] * VS + kv[t];
+                                eb[t][0] = make_float2(qe[0], qe[VS]);
+                                eb[t][1] = make_float2(qe[2 * VS], qe[3 * VS]);
+                                const float2 wb0 = __fmul2_rn(make_float2(qw[0], qw[VS]), fb[t][0]);
+                                const float2 wb1 = __fmul2_rn(make_float2(qw[2 * VS], qw[3 * VS]), fb[t][1]);
+                                accb = __ffma2_rn(wb0, eb[t][0], accb);
+                                accb = __ffma2_rn(wb1, eb[t][1], accb);
+                                acch = __ffma2_rn(wb0, fab[t][0], acch);
+                                acch = __ffma2_rn(wb1, fab[t][1], acch);
+                            }
                         }
-                        gb += accb;
-                        hh += acch;
+                        // the stages are consumed (their values are in registers): release them
+                        // to the producer warp
+                        __syncwarp();
+                        if (lane == 0) {
+                            mbar_arrive(empty + g % R);
+                            if (HB) mbar_arrive(empty + (g + 1) % R);
+                        }
+                        float2 gab = make_float2(acc.x + acc.y, accb.x + accb.y);
+                        float hh = acch.x + acch.y;
+#pragma unroll
+                        for (int o = 16; o > 0; o >>= 1) {
+                            const float2 r = make_float2(__shfl_xor_sync(kFull, gab.x, o), __shfl_xor_sync(kFull, gab.y, o));
+                            gab = __fadd2_rn(gab, r);
+                            if (HB) hh += __shfl_xor_sync(kFull, hh, o);
+                        }
+                        if (lane == 0) {
+                            red[buf * 24 + vw] = gab.x;
+                            red[buf * 24 + 8 + vw] = gab.y;
+                            red[buf * 24 + 16 + vw] = hh;
+                        }
+                    };
+                    if (hasb)
+                        gather(BoolTag<true>{});
+                    else
+                        gather(BoolTag<false>{});
+                } else if (idx == 0) {
+                    // prior warp: the surrogate terms of a pair are published after the previous
+                    // pair's barrier; only the first pair's are computed here
+                    prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB, pri);
+                }
+                {
+                    // the view warps and the prior warp meet (named barrier 1; the producer warp
+                    // runs decoupled on the full/empty mbarriers)
+                    const long long tw0 = P.tprof ? clock64() : 0;
+                    asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
+                    if (P.tprof && lane == 0)  // development aid: per-warp wait at the pair barrier
+                        atomicAdd(P.tprof + 10 + warp, (unsigned long long)(clock64() - tw0));
+                }
+                // every warp derives the same two deltas (identical inputs, identical order)
+                const float* rb = red + buf * 24;  // nvw <= 8 partials per quantity, rest 0
+                const float sa = sum8(rb), sbs = sum8(rb + 8), sh = sum8(rb + 16);
+                const PriPair pp = pri[buf];
+                const float scale_a = vscale[idx];
+                float ua = pp.va;
+                {
+                    const float theta1 = -scale_a * sa;  // Alg1:5
+                    const float theta2 = vth2[idx];      // Alg1:6 (precomputed)
+                    const float num = theta2 * pp.va - theta1 + 2.f * pp.sxa;
+                    const float den = theta2 + 2.f * pp.sa;
+                    if (den > 0.f) ua = __fdividef(num, den);
+                    if (c_prior.positivity) ua = fmaxf(ua, 0.f);
+                }
+                const float da = ua - pp.va;  // Alg1:7-8
+                float ub = pp.vb, db = 0.f, scale_b = 0.f;
+                if (hasb) {
+                    scale_b = vscale[idx + 1];
+                    // e after a's update: sum w A_b e' = s_b (S_b - s_a delta_a H)
+                    const float theta1 = -scale_b * fmaf(-scale_a * da, sh, sbs);
+                    const float theta2 = vth2[idx + 1];
+                    float psb = pp.sb, psx = pp.sxb;
+                    if (pp.bab != 0.f) {  // a is b's neighbour: its term with a's new value
+                        const float bn = pp.bab * phi_f(pp.vb - ua);
+                        psb += bn - pp.btab;
+                        psx += bn * ua - pp.btab * pp.va;
                     }
+                    const float num = theta2 * pp.vb - theta1 + 2.f * psx;
+                    const float den = theta2 + 2.f * psb;
+                    if (den > 0.f) ub = __fdividef(num, den);
+                    if (c_prior.positivity) ub = fmaxf(ub, 0.f);
+                    db = ub - pp.vb;
                 }
+                if (is_view) {
+                    // Alg1:9-11 for both voxels on this thread's views: a's channels first with
+                    // a's update, then b's channels with both updates -- b's path rewrites the
+                    // entries the two voxels share with the full value, so A_b is never needed on
+                    // a's channels
+                    const float sda = scale_a * da, sdb = scale_b * db;
+                    if (sda != 0.f || sdb != 0.f) {
+                        const float2 na = make_float2(-sda, -sda), nb = make_float2(-sdb, -sdb);
+                        auto put2 = [&](float* p, float2 v0, float2 v1) {
+                            p[0] = v0.x;
+                            p[VS] = v0.y;
+                            p[2 * VS] = v1.x;
+                            p[3 * VS] = v1.y;
+                        };
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) {
-                    ga += __shfl_xor_sync(kFull, ga, o);
-                    gb += __shfl_xor_sync(kFull, gb, o);
-                    hh += __shfl_xor_sync(kFull, hh, o);
-                }
-                if (lane == 0) {
-                    red[buf * 24 + warp] = ga;
-                    red[buf * 24 + 8 + warp] = gb;
-                    red[buf * 24 + 16 + warp] = hh;
-                }
-            } else if (warp == nvw) {
-                // prior warp: the surrogate terms of this pair were published after the previous
-                // barrier; only the first pair is computed here
-                if (idx == 0) prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB, pri);
-            } else if (lane == 0) {
-                // producer warp: the next pair's A records must have landed before the barrier
-                if (idx + 2 < nact) mbar_wait(mbar + (g + 2) % R, ((g + 2) / R) & 1);
-                if (idx + 3 < nact) mbar_wait(mbar + (g + 3) % R, ((g + 3) / R) & 1);
-            }
-            __syncthreads();
-            // every warp derives the same two deltas (identical inputs, identical order)
-            const float* rb = red + buf * 24;  // nvw <= 8 partials per quantity, rest 0
-            const float sa = sum8(rb), sbs = sum8(rb + 8), sh = sum8(rb + 16);
-            const PriPair pp = pri[buf];
-            const float scale_a = vscale[idx];
-            float ua = pp.va;
-            {
-                const float theta1 = -scale_a * sa;  // Alg1:5
-                const float theta2 = vth2[idx];      // Alg1:6 (precomputed)
-                const float num = theta2 * pp.va - theta1 + 2.f * pp.sxa;
-                const float den = theta2 + 2.f * pp.sa;
-                if (den > 0.f) ua = __fdividef(num, den);
-                if (c_prior.positivity) ua = fmaxf(ua, 0.f);
-            }
-            const float da = ua - pp.va;  // Alg1:7-8
-            float ub = pp.vb, db = 0.f, scale_b = 0.f;
-            if (hasb) {
-                scale_b = vscale[idx + 1];
-                // e after a's update: sum w A_b e' = s_b (S_b - s_a delta_a H)
-                const float theta1 = -scale_b * fmaf(-scale_a * da, sh, sbs);
-                const float theta2 = vth2[idx + 1];
-                float psb = pp.sb, psx = pp.sxb;
-                if (pp.bab != 0.f) {  // a is b's neighbour: its term with a's new value
-                    const float bn = pp.bab * phi_f(pp.vb - ua);
-                    psb += bn - pp.btab;
-                    psx += bn * ua - pp.btab * pp.va;
-                }
-                const float num = theta2 * pp.vb - theta1 + 2.f * psx;
-                const float den = theta2 + 2.f * psb;
-                if (den > 0.f) ub = __fdividef(num, den);
-                if (c_prior.positivity) ub = fmaxf(ub, 0.f);
-                db = ub - pp.vb;
-            }
-            if (warp < nvw) {
-                // Alg1:9-11 for both voxels on this thread's views: a's channels first with a's
-                // update, then b's channels with both updates -- b's path rewrites the entries the
-                // two voxels share with the full value, so A_b is never needed on a's channels
-                const float sda = scale_a * da, sdb = scale_b * db;
-                if (sda != 0.f || sdb != 0.f) {
-#pragma unroll
-                    for (int t = 0; t < VPT; ++t) {
-                        const float va[4] = {fa[t].x, fa[t].y, fa[t].z, fa[t].w};
-                        float* pe = sb_e + oa[t] * Vs + kv[t];
-#pragma unroll
-                        for (int i = 0; i < 4; ++i) pe[i * Vs] = fmaf(-va[i], sda, ea[t][i]);
+                        for (int t = 0; t < VPT; ++t) {
+                            put2(sb_e + oa[t] * VS + kv[t], __ffma2_rn(fa[t][0], na, ea[t][0]),
+                                 __ffma2_rn(fa[t][1], na, ea[t][1]));
+                            if (hasb)
+                                put2(sb_e + ob[t] * VS + kv[t],
+                                     __ffma2_rn(fb[t][0], nb, __ffma2_rn(fab[t][0], na, eb[t][0])),
+                                     __ffma2_rn(fb[t][1], nb, __ffma2_rn(fab[t][1], na, eb[t][1])));
+                        }
+                    }
+                } else {
+                    // prior warp: store the pair's new values, then the next pair's surrogate
+                    // terms (published for the view warps before the next barrier)
+                    if (lane == 0) {
+                        const int ta = tof[idx];
+                        xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
                         if (hasb) {
-                            const float vb[4] = {fb[t].x, fb[t].y, fb[t].z, fb[t].w};
-                            const float vab[4] = {fab[t].x, fab[t].y, fab[t].z, fab[t].w};
-                            float* qe = sb_e + ob[t] * Vs + kv[t];
-#pragma unroll
-                            for (int i = 0; i < 4; ++i) qe[i * Vs] = fmaf(-vb[i], sdb, fmaf(-vab[i], sda, eb[t][i]));
+                            const int tbv = tof[idx + 1];
+                            xt[cslot + (tbv >> 8) * TW + (tbv & 255)] = ub;
                         }
+                        amount += fabsf(da) + fabsf(db);
                     }
+                    __syncwarp();
+                    const long long tr0 = P.tprof ? clock64() : 0;
+                    if (idx + 2 < nact)
+                        prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
+                                   pri + (buf ^ 1));
+                    if (P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
                 }
-            } else if (warp == nvw) {
-                // prior warp: store the pair's new values, then the next pair's surrogate terms
-                if (lane == 0) {
-                    const int ta = tof[idx];
-                    xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
-                    if (hasb) {
-                        const int tb = tof[idx + 1];
-                        xt[cslot + (tb >> 8) * TW + (tb & 255)] = ub;
+            }
+        } else if (is_prod) {
+            // producer warp, decoupled from the pair loop: first the next task's band info (and
+            // an L2 warm-up of its band rows), then the A records of voxels R .. nact-1, each as
+            // soon as the view warps have released the stage it goes to
+            if (lane == 0) {
+                const long long tq0 = P.tprof ? clock64() : 0;
+                for (int j = R; j < nact; ++j) {
+                    if (j + R < nact) {  // L2 warm-up R records ahead
+                        const size_t rp = (arec + list[j + R]) * (size_t)VA;
+                        l2_prefetch_bulk(U8 ? (const void*)(P.A.codes + rp) : (const void*)(P.A.vals + rp), VA * (U8 ? 4 : 16));
+                        l2_prefetch_bulk(P.A.off + rp, VA);
                     }
-                    amount += fabsf(da) + fabsf(db);
+                    const uint32_t n = gseq + j, s = n % R;
+                    mbar_wait(empty + s, ((n / R) - 1) & 1);  // use n/R - 1 of stage s consumed
+                    unsigned char* dst = astage + s * L.stage_bytes;
+                    const size_t rec = (arec + list[j]) * (size_t)VA;
+                    mbar_expect_tx(full + s, stage_tx);
+                    if (U8)
+                        tma_load_1d(dst, P.A.codes + rec, VA * 4, full + s);
+                    else
+                        tma_load_1d(dst, P.A.vals + rec, VA * 16, full + s);
+                    tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, full + s);
                 }
-                __syncwarp();
-                if (idx + 2 < nact)
-                    prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
-                               pri + (buf ^ 1));
-            } else if (lane == 0) {
-                // producer warp: the pair's stages were read by every view warp before the
-                // barrier: refill them with the A records of voxels idx + R, idx + 1 + R
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                if (P.tprof) atomicAdd(P.tprof + 21, (unsigned long long)(clock64() - tq0));
+            }
+            __syncwarp();
+            // then the next task's band info (R voxels of loop time remain): all loads in flight
+            // at once, then the stores and the L2 warm-up of the band rows
+            if (pf_task >= 0) {
+                constexpr int KMAX = 12;  // views per lane and pass: two passes cover V <= 768
+                const int psv = pf_task & 16383, pz = pf_task >> 14;
+                uint32_t* dst = binfo + (tb ^ 1) * VA;
+#pragma unroll 1
+                for (int k0 = 0; k0 < V; k0 += 32 * KMAX) {
+                int bs[KMAX], bwd[KMAX];
 #pragma unroll
-                for (int u = 0; u < 2; ++u) {
-                    if (idx + u + R < nact) {
-                        const uint32_t s = (g + u) % R;
-                        unsigned char* dst = astage + s * L.stage_bytes;
-                        const size_t rec = (arec + list[idx + u + R]) * (size_t)VA;
-                        mbar_expect_tx(mbar + s, stage_tx);
-                        if (U8)
-                            tma_load_1d(dst, P.A.codes + rec, VA * 4, mbar + s);
-                        else
-                            tma_load_1d(dst, P.A.vals + rec, VA * 16, mbar + s);
-                        tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, mbar + s);
+                for (int i = 0; i < KMAX; ++i) {
+                    const int k = k0 + lane + 32 * i;
+                    if (k < V) {
+                        bs[i] = P.A.band_start[(size_t)psv * V + k];
+                        bwd[i] = P.A.band_width[(size_t)psv * V + k];
                     }
+                }
+                const float* wz = P.w + (size_t)pz * V * M;
+                const float* ez = P.e + (size_t)pz * V * M;
+#pragma unroll
+                for (int i = 0; i < KMAX; ++i) {
+                    const int k = k0 + lane + 32 * i;
+                    if (k < V) {
+                        const int r = k * M + bs[i], r1 = r + max(bwd[i], 1) - 1;
+                        dst[k] = ((uint32_t)r << 5) | (uint32_t)bwd[i];
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
+                    }
+                }
                 }
             }
         }
@@ -719,42 +873,44 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
         __syncthreads();
 
         // ---- 6. write-back: delta e of the band, atomically, and the SV's voxels
-        if (warp < nvw) {
+        if (is_view) {
             float* ez = P.e + (size_t)z * V * M;
-            // the final band goes back through the rotated staging tile (see the pack), then each
-            // aligned 32-float row window gets delta = final - e_init with red.global.add.v4.f32
+            // the final band goes back through the staging tile (stride 33, as in the pack), then
+            // each aligned 32-float row window gets delta = final - e_init (band positions only)
+            // with red.global.add.v4.f32
             const int sub = lane >> 3, ch = lane & 7;
 #pragma unroll 1
             for (int t = 0; t < VPT; ++t) {
-                const int k0 = (warp * VPT + t) * 32;
+                const int k0 = (vw * VPT + t) * 32;
                 const int kk = k0 + lane;
-                const int bw = kk < V ? (int)P.A.band_width[(size_t)sv * V + kk] : 0;
-                const int roff = kk < V ? kk * M + P.A.band_start[(size_t)sv * V + kk] : 0;
+                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const int bw = (int)(bi & 31u), roff = (int)(bi >> 5);
+                const uint32_t bmask = ((1u << bw) - 1u) << (roff & 3);
                 float4 s4[8];  // e_init windows, in flight during the staging below
 #pragma unroll
                 for (int m = 0; m < 8; ++m) s4[m] = __ldcg((const float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch));
+                const float* se = sb_e + kk - (roff & 3) * VS;
+                float* sr = stg_w + lane * 33;
 #pragma unroll
-                for (int c = 0; c < 32; ++c)
-                    if (c < P.rows) stg_w[lane * 32 + ((c + lane) & 31)] = sb_e[c * Vs + kk];
+                for (int p = 0; p < 32; ++p)
+                    if (bmask & (1u << p)) sr[p] = se[p * VS];
                 __syncwarp();
 #pragma unroll
                 for (int m = 0; m < 8; ++m) {
                     const int i = 4 * m + sub;
-                    const int oi = __shfl_sync(kFull, roff, i), wi = __shfl_sync(kFull, bw, i);
+                    const int oi = __shfl_sync(kFull, roff, i);
+                    const uint32_t nib = __shfl_sync(kFull, bmask, i) >> (4 * ch);
                     const int s = oi & 3;
                     float d[4];
                     const float e0[4] = {s4[m].x, s4[m].y, s4[m].z, s4[m].w};
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const int c = 4 * ch + j - s;
-                        d[j] = (c >= 0 && c < wi) ? stg_w[i * 32 + ((c + i) & 31)] - e0[j] : 0.f;
-                    }
+                    for (int j = 0; j < 4; ++j) d[j] = (nib & (1u << j)) ? stg_w[i * 33 + 4 * ch + j] - e0[j] : 0.f;
                     if (k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
                         red_add_v4(ez + (oi - s) + 4 * ch, d[0], d[1], d[2], d[3]);
                 }
                 __syncwarp();
             }
-        } else if (warp == nvw) {
+        } else if (is_prior) {
             for (int i = lane; i < tw * th; i += 32) {
                 const int lx = i % tw, ly = i / tw;
                 P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] =
@@ -954,7 +1110,7 @@ constexpr int ring_depth(bool u8) { return u8 ? 8 : 4; }
 int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
 {
     (void)vpt;
-    return smem_layout(p.rows, p.Vs, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw).total;
+    return smem_layout(p.rows, svb_stride(vpt), p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw).total;
 }
 
 template <int VPT, bool U8, int NNB>
@@ -962,10 +1118,12 @@ static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t
 {
     constexpr int R = ring_depth(U8);
     auto kern = k_icd_sv<VPT, U8, NNB, R>;
-    const int smem = smem_layout(p.rows, p.Vs, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw).total;
+    IcdParams q = p;
+    q.lay = smem_layout(p.rows, svb_stride(VPT), p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw);
+    const int smem = q.lay.total;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    kern<<<dim3(gx, gy), 32 * (p.nvw + 2), smem, st>>>(p);  // view warps + prior + producer
+    kern<<<dim3(gx, gy), 32 * (p.nvw + 2), smem, st>>>(q);  // view warps + prior + producer
     return cudaGetLastError();
 }
 

@@ -53,6 +53,14 @@ __host__ __device__ __forceinline__ int apos(int k, int vpt)
     return ((blk / vpt) * 32 + (k & 31)) * vpt + blk % vpt;
 }
 
+// byte offsets of the update kernel's shared-memory regions (computed on the host per launch
+// configuration and passed in the parameter block, so the kernel addresses them from the
+// constant bank instead of recomputing the layout in registers)
+struct SmemLayout {
+    int sb_e, sb_w, xt, list, flags, tof, red, pri, vscale, vth2, misc, astage, stage_bytes,
+        off_in_stage, mbar, staging, binfo, total;
+};
+
 // ---- parameters of the fused SuperVoxel update kernel ----
 struct IcdParams {
     int nx, ny, nz_local, z_offset, nz_total;
@@ -80,6 +88,7 @@ struct IcdParams {
     int zero_skip_active;
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
+    SmemLayout lay;          // update-kernel smem layout (filled by launch_icd)
 };
 
 struct SchedParams {
