@@ -90,6 +90,10 @@ typedef struct mbir_options {
     int deterministic;     /* debug: every iteration visits all SVs one at a time (one CTA) in
                               the order z-parity half (3-D prior only), colour, SV rank within
                               the colour (SV index order), slice; voxels in raster order        */
+    int cluster;           /* CTAs per SV task in the update kernel: 0 = auto (currently 1);
+                              1 = one CTA owns a task; 2 = a 2-CTA thread-block cluster splits
+                              the task's views (two tasks per SM; EINVAL where not possible).
+                              The arithmetic is the same either way.                             */
 } mbir_options;
 
 /* Placement and (optional) multi-GPU slab partition.  device: CUDA ordinal.  stream: a
@@ -126,6 +130,8 @@ typedef struct mbir_sizes {
     int band_max;                   /* max SV band width over (SV, view), channels        */
     int svb_rows;                   /* rows of the shared-memory SV buffer (>= band_max)  */
     int threads_per_cta;            /* update-kernel block size                            */
+    int cluster;                    /* update-kernel CTAs per SV task (1 or 2)             */
+    int resident_ctas;              /* update-kernel CTAs resident at once (occupancy)     */
     int smem_bytes;                 /* update-kernel dynamic shared memory                 */
     int64_t nnz;                    /* total non-zeros of the slice-plane system matrix    */
     int64_t a_bytes;                /* device bytes of the compressed A                   */
@@ -133,7 +139,7 @@ typedef struct mbir_sizes {
 } mbir_sizes;
 
 /* Fill defaults: sv_side 9, sv_fraction 0.25, batch_svs 0, batch_threshold -1, zero_skip 1,
- * quantize_A 1, seed 3000, deterministic 0. */
+ * quantize_A 1, seed 3000, deterministic 0, cluster 0 (auto). */
 void mbir_default_options(mbir_options* o);
 /* p 1.2, q 2, T 1, sigma 0.005, neighborhood 26, positivity 1. */
 void mbir_default_prior(mbir_prior* p);

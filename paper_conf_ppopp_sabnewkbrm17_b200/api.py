@@ -72,11 +72,12 @@ class Options:
     quantize_A: int = 1
     seed: int = 3000
     deterministic: int = 0
+    cluster: int = 0  # update-kernel CTAs per SV task: 0 auto, 1, 2 (same arithmetic)
 
     def c(self) -> L.mbir_options:
         return L.mbir_options(self.sv_side, self.sv_fraction, self.batch_svs,
                               self.batch_threshold, self.zero_skip, self.quantize_A, self.seed,
-                              self.deterministic)
+                              self.deterministic, self.cluster)
 
 
 def _buf(a, n: int | None = None, dtype=np.float32, writable=False):

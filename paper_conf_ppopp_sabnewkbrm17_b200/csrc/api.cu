@@ -79,6 +79,8 @@ struct mbir_handle {
     int side = 0, nsvx = 0, nsvy = 0, nsv = 0, S2 = 0, nsv_pad = 0;
     int rows = 0, band_max = 0;
     int vpt = 1, nvw = 0, Vs = 0, threads = 0, smem = 0, blocks_per_sm = 1, nsm = 148;
+    int cl = 1;  // update-kernel CTAs per SV task (2: thread-block cluster splitting the views)
+    int resident = 0;  // update-kernel CTAs resident on the device at once (occupancy query)
     int max_group = 0;
     DevA A{};
     double* d_cs = nullptr;
@@ -160,6 +162,7 @@ IcdParams make_params(mbir_handle* h)
     p.iter = h->iter;
     p.deterministic = h->o.deterministic;
     p.tprof = h->d_tprof;
+    p.dbg = getenv("MBIR_DBG") ? atoi(getenv("MBIR_DBG")) : 0;
     return p;
 }
 
@@ -204,7 +207,7 @@ int timed_icd(mbir_handle* h, const IcdParams& p, int nnb, bool q, int gx, int g
         }
     }
     CK(cudaEventRecord(h->kev[2 * h->kev_used], h->st));
-    CK(launch_icd(p, h->vpt, nnb, q, gx, gy, h->st));
+    CK(launch_icd(p, h->vpt, nnb, q, h->cl, gx, gy, h->st));
     CK(cudaEventRecord(h->kev[2 * h->kev_used + 1], h->st));
     h->kev_used++;
     return MBIR_OK;
@@ -281,8 +284,9 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         IcdParams p = make_params(h);
         p.zero_skip_active = (h->o.zero_skip && h->iter > 1) ? 1 : 0;
         const size_t cap = (size_t)h->g.nz_local * h->max_group;
-        // deterministic: one CTA walks the phase list in order (sequential ICD, known order)
-        const int grid = det ? 1 : target_ctas;
+        // deterministic: one CTA (or one cluster) walks the phase list in order (sequential ICD,
+        // known order)
+        const int grid = det ? h->cl : target_ctas;
         for (int zp = 0; zp < parities; ++zp) {
             for (int colour = 0; colour < 4; ++colour) {
                 const int ph = zp * 4 + colour;
@@ -359,6 +363,8 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         for (int i = 0; i < 8; ++i) fprintf(stderr, " %.0f", t[10 + i] / v);
         fprintf(stderr, " | producer loop %.0f | view full-wait (records < R, >= R) %.0f %.0f | prior_pair %.0f",
                 t[21] / v, t[22] / v, t[23] / v, t[24] / v);
+        fprintf(stderr, " | TMA issue->ready: blocked waits %llu avg latency %.0f, unblocked %llu avg lead %.0f",
+                t[26], t[25] / (double)(t[26] ? t[26] : 1), t[28], t[27] / (double)(t[28] ? t[28] : 1));
         fprintf(stderr, "\n");
     }
     return MBIR_OK;
@@ -610,15 +616,30 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         return (fail(h, MBIR_EINVAL, "nviews * nchannels must be < 2^27"), bail(MBIR_EINVAL));
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
-    h->threads = 32 * (h->nvw + 2);  // view warps + prior warp + TMA producer warp
-    if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
     {
+        // cluster variant (two tasks per SM, each split over a 2-CTA cluster): uint8 A, 4 views
+        // per lane, an even number of view warps, and two CTAs' shared memory fitting one SM
         IcdParams p = make_params(h);
-        h->smem = icd_smem_bytes(p, h->vpt, P.neighborhood, quant);
+        const int want = h->o.cluster;
+        if (want < 0 || want > 2) return (fail(h, MBIR_EINVAL, "cluster must be 0, 1 or 2"), bail(MBIR_EINVAL));
+        const int smem2 = icd_smem_bytes(p, h->vpt, P.neighborhood, quant, 2);
+        const bool ok2 = quant && h->vpt == 4 && h->nvw % 2 == 0 && h->nvw >= 2 &&
+                         h->S2 <= 32 * (h->nvw / 2 + 1) &&
+                         2 * (smem2 + 1024) <= (int)prop.sharedMemPerMultiprocessor;
+        if (want == 2 && !ok2)
+            return (fail(h, MBIR_EINVAL, "cluster = 2 needs uint8 A, > 128 views in an even number of 128-view warps and two SV buffers per SM"), bail(MBIR_EINVAL));
+        // auto = 1: measured on cfg4, the cluster variant's per-pair DSMEM exchange lengthens the
+        // voxel chain more than splitting the views shortens it
+        h->cl = want == 2 ? 2 : 1;
+        h->threads = 32 * (h->nvw / h->cl + 1);  // view warps + the prior (and A-stream producer) warp
+        if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
+        h->smem = icd_smem_bytes(p, h->vpt, P.neighborhood, quant, h->cl);
         if (h->smem > (int)prop.sharedMemPerBlockOptin)
             return (fail(h, MBIR_EINVAL, "SV buffer (" + std::to_string(h->smem) + " B) exceeds shared memory: reduce sv_side"), bail(MBIR_EINVAL));
         h->blocks_per_sm = std::max(1, std::min((int)(prop.sharedMemPerMultiprocessor / (h->smem + 1024)),
                                                 (int)(2048 / h->threads)));
+        if (h->cl == 2) h->blocks_per_sm = 2;  // two clusters' CTAs per SM (grid = 2 x 148)
+        h->resident = icd_resident_ctas(p, h->vpt, P.neighborhood, quant, h->cl);
     }
 
     // ---- state buffers
@@ -837,6 +858,8 @@ int mbir_query_sizes(const mbir_handle* h, mbir_sizes* s)
     s->band_max = h->band_max;
     s->svb_rows = h->rows;
     s->threads_per_cta = h->threads;
+    s->cluster = h->cl;
+    s->resident_ctas = h->resident;
     s->smem_bytes = h->smem;
     s->nnz = h->nnz;
     s->a_bytes = h->a_bytes;

@@ -24,6 +24,9 @@
 // share sinogram entries.
 #include "mbir_internal.h"
 
+#include <cstdio>
+#include <cstdlib>
+
 namespace mbir {
 
 __constant__ PriorConst c_prior;
@@ -285,6 +288,21 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
         "r"(parity)
         : "memory");
 }
+// per-thread asynchronous global -> shared copies (LDGSTS), tracked per thread by commit groups
+__device__ __forceinline__ void cp_async16(void* dst, const void* src)
+{
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* dst, const void* src)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait()
+{
+    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
 // warm L2 with a global block (bulk prefetch; no completion tracking)
 __device__ __forceinline__ void l2_prefetch_bulk(const void* src, uint32_t bytes)
 {
@@ -299,19 +317,69 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
         : "memory");
 }
 
+// ---- thread-block-cluster helpers (CL = 2: the two CTAs of a cluster split an SV's views) ----
+__device__ __forceinline__ uint32_t cluster_rank()
+{
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+// shared::cluster address of the same smem location in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t peer_addr(const void* p, uint32_t rank)
+{
+    uint32_t a;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(smem_u32(p)), "r"(rank));
+    return a;
+}
+__device__ __forceinline__ void st_peer_f32(uint32_t a, float v)
+{
+    asm volatile("st.shared::cluster.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
+}
+__device__ __forceinline__ void st_peer_u32(uint32_t a, uint32_t v)
+{
+    asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+// arrive on an mbarrier of the peer CTA; release at cluster scope orders this thread's earlier
+// st.shared::cluster writes before the arrival
+__device__ __forceinline__ void mbar_arrive_peer(uint32_t a)
+{
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(a) : "memory");
+}
+// wait for a phase with acquire at cluster scope (sees the peer's released writes)
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity)
+{
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAITC_%=:\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAITC_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all()
+{
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
 
-// the update kernel's SVB column stride: the most views a launch configuration can hold (6 view
-// warps x 32 lanes x VPT views), fixed at compile time whatever the actual view count
-__host__ __device__ constexpr int svb_stride(int vpt) { return 6 * 32 * vpt; }
+// the update kernel's SVB column stride: the most views one CTA can hold (6 / CL view warps x
+// 32 lanes x VPT views), fixed at compile time whatever the actual view count
+__host__ __device__ constexpr int svb_stride(int vpt, int cl = 1) { return 6 / cl * 32 * vpt; }
 
-// A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
+// pair-exchange buffers of the update kernel (red partials / prior terms): the cluster variant
+// needs 3 (a CTA can run one pair ahead of its peer), 4 keeps the index a mask
+constexpr int kPairBufs = 4;
+
+// A-record stage: U8: codes u32[VL] then offsets u8[VL]; fp32: float4[VL] then offsets u8[VL];
+// VL = VA / cl record positions (this CTA's views)
 __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, int S2, int nnb,
-                                                  int VA, bool u8, int nstage, int nvw)
+                                                  int VA, bool u8, int nstage, int nvw, int cl)
 {
     SmemLayout L;
     const int TW = side + 2;
     const int nzt = nnb == 26 ? 3 : 1;
+    const int VL = VA / cl, nvl = nvw / cl;
     int o = 0;
     L.sb_e = o;  o = align16(o + rows * Vs * 4);
     L.sb_w = o;  o = align16(o + rows * Vs * 4);
@@ -319,58 +387,63 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.list = o;  o = align16(o + S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
     L.tof = o;   o = align16(o + S2 * 4);
-    L.red = o;   o = align16(o + 2 * 24 * 4);  // [2 bufs][3 quantities][8 warps]
-    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriPair));
+    L.red = o;   o = align16(o + kPairBufs * 24 * 4);  // [bufs][3 quantities][8 view warps]
+    L.pri = o;   o = align16(o + kPairBufs * (int)sizeof(PriPair));
     L.vscale = o; o = align16(o + S2 * 4);
     L.vth2 = o;  o = align16(o + S2 * 4);
     L.misc = o;  o = align16(o + 16 * 4);
-    L.off_in_stage = VA * (u8 ? 4 : 16);
-    L.stage_bytes = align16(L.off_in_stage + VA);
+    L.off_in_stage = VL * (u8 ? 4 : 16);
+    L.stage_bytes = align16(L.off_in_stage + VL);
     L.astage = o; o = align16(o + nstage * L.stage_bytes);
-    L.mbar = o;  o = align16(o + 2 * nstage * 8);  // full[nstage], then empty[nstage]
-    L.staging = o; o = align16(o + nvw * 32 * 33 * 4);  // one 32x33 transpose tile per view warp
-    L.binfo = o; o = align16(o + 2 * VA * 4);           // band (row offset << 5 | width), 2 tasks
+    // pair[kPairBufs], task[1]
+    L.mbar = o;  o = align16(o + (kPairBufs + 1) * 8);
+    L.staging = o; o = align16(o + nvl * 32 * 33 * 4);  // one 32x33 transpose tile per view warp
+    L.binfo = o; o = align16(o + 2 * VL * 4);           // band (row offset << 5 | width), 2 tasks
     L.total = o;
     return L;
 }
 
-// band of task tk for views k0, k0 + stride, ... < k1 into dst[k] = (k*M + start) << 5 | width;
-// optionally warms L2 with the band's w and e lines (the next task's pack then reads L2)
-__device__ __forceinline__ void band_info(const IcdParams& P, int tk, uint32_t* dst, int k0, int k1,
-                                          int stride, bool prefetch)
+// band of task tk for this CTA's views vbase + k, k = k0, k0 + stride, ... < VL (and < V) into
+// dst[k] = ((vbase + k)*M + start) << 5 | width
+__device__ __forceinline__ void band_info(const IcdParams& P, int tk, uint32_t* dst, int vbase, int VL,
+                                          int k0, int stride)
 {
-    const int z = tk >> 14, sv = tk & 16383;
-    const float* wz = P.w + (size_t)z * P.V * P.M;
-    const float* ez = P.e + (size_t)z * P.V * P.M;
-    for (int k = k0; k < k1; k += stride) {
-        const int r = k * P.M + P.A.band_start[(size_t)sv * P.V + k];
-        const int wd = P.A.band_width[(size_t)sv * P.V + k];
+    const int sv = tk & 16383;
+    for (int k = k0; k < VL && vbase + k < P.V; k += stride) {
+        const int kg = vbase + k;
+        const int r = kg * P.M + P.A.band_start[(size_t)sv * P.V + kg];
+        const int wd = P.A.band_width[(size_t)sv * P.V + kg];
         dst[k] = ((uint32_t)r << 5) | (uint32_t)wd;
-        if (prefetch) {
-            const int r1 = r + max(wd, 1) - 1;
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
-        }
     }
 }
 
-template <int VPT, bool U8, int NNB, int R>
-__global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 view + 2 warps
+// CL = 1: one CTA per SM owns a whole (slice, SV) task.  CL = 2: a 2-CTA cluster owns the task,
+// each CTA holding half the views (its half of the SVB and of every A record), two clusters'
+// CTAs per SM; per voxel pair the CTAs exchange their partial sums through distributed shared
+// memory, so both derive the same deltas.  Two independent tasks per SM let one CTA's pack and
+// write-back overlap the other's voxel loop.
+// CL = 1: one CTA of <= 6 view warps + the prior warp per SM; CL = 2: two CTAs of 3 view warps +
+// the prior warp per SM (8 warps: the full register budget per thread)
+template <int VPT, bool U8, int NNB, int R, int CL>
+__global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int nvw = P.nvw;
-    // warp roles: nvw view warps, the prior warp and the TMA producer warp.  Warps w and w + 4
-    // share a scheduler (SMSP); with >= 3 view warps the prior warp is warp 3, so it shares
-    // SMSP 3 only with the producer (which mostly sleeps on mbarriers) and the view warps spread
-    // evenly over SMSPs 0-2 (and 3 when nvw is small).
-    const int prior_w = nvw >= 3 ? 3 : nvw, prod_w = nvw + 1;
-    const bool is_prior = warp == prior_w, is_prod = warp == prod_w, is_view = !is_prior && !is_prod;
-    const int vw = is_view ? (warp < prior_w ? warp : warp - 1) : 0;  // view-warp index
-    const int V = P.V, M = P.M, S2 = P.S2, side = P.side, VA = P.A.VA;
-    constexpr int VS = svb_stride(VPT);  // SVB view stride: compile-time, so row offsets are immediates
+    const int nvw = P.nvw;              // view warps of the whole task (both CTAs)
+    const int nvl = nvw / CL;           // view warps of this CTA
+    const uint32_t crank = CL == 1 ? 0u : cluster_rank();
+    // warp roles: nvl view warps and the prior warp, which also produces the A-record stream
+    // (TMA) and the next task's band info.  Warps w and w + 4 share a scheduler (SMSP); with >= 3
+    // view warps the prior warp is warp 3, so the view warps spread evenly over SMSPs 0-2 (and 3
+    // when nvl is small).
+    const int prior_w = nvl >= 3 ? 3 : nvl;
+    const bool is_prior = warp == prior_w, is_view = !is_prior;
+    const int vw = is_view ? (warp < prior_w ? warp : warp - 1) : 0;  // local view-warp index
+    const int gvw = (int)crank * nvl + vw;                             // view-warp index in the task
+    const int V = P.V, M = P.M, S2 = P.S2, side = P.side;
+    const int VL = P.A.VA / CL;          // record positions / SVB columns of this CTA
+    const int vbase = (int)crank * VL;   // first view (and record position) of this CTA
+    constexpr int VS = svb_stride(VPT, CL);  // SVB view stride: compile-time, so row offsets are immediates
     const SmemLayout& L = P.lay;
     float* sb_e = (float*)(smem + L.sb_e);
     float* sb_w = (float*)(smem + L.sb_w);
@@ -388,30 +461,32 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
     const size_t plane = (size_t)P.nx * P.ny;
-    const uint32_t stage_tx = (uint32_t)(VA * (U8 ? 4 : 16) + VA);
+    uint64_t* pairbar = mbar;              // [kPairBufs] (CL = 2): both CTAs' partials + prior terms
+    uint64_t* taskbar = pairbar + kPairBufs;  // (CL = 2, rank 1): the next task id has arrived
 
-    if (threadIdx.x < 48) red[threadIdx.x] = 0.f;  // slots >= nvw stay zero
+    if (threadIdx.x < kPairBufs * 24) red[threadIdx.x] = 0.f;  // slots >= nvw stay zero
     // SVB rows outside a visit's band are never packed: start them finite (zero)
     for (int i = threadIdx.x; i < (L.sb_w - L.sb_e) / 16; i += blockDim.x) {
         ((float4*)(smem + L.sb_e))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
         ((float4*)(smem + L.sb_w))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
     }
     if (threadIdx.x == 0) {
-        for (int s = 0; s < R; ++s) {
-            mbar_init(mbar + s, 1);          // full: the producer's arrive + the TMA bytes
-            mbar_init(mbar + R + s, nvw);    // empty: one arrive per view warp
-        }
+        for (int b = 0; b < kPairBufs; ++b) mbar_init(pairbar + b, nvw + 1);  // all view warps + prior
+        mbar_init(taskbar, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    // per-thread view ownership: warp w, lane l owns views (w*VPT + t)*32 + l
+    // per-thread view ownership: (task) view-warp g, lane l owns views (g*VPT + t)*32 + l, held in
+    // SVB column (vw*VPT + t)*32 + l of its CTA
     int kv[VPT];
     bool kval[VPT];
 #pragma unroll
     for (int t = 0; t < VPT; ++t) {
         kv[t] = (vw * VPT + t) * 32 + lane;
-        kval[t] = is_view && kv[t] < V;
+        kval[t] = is_view && vbase + kv[t] < V;
     }
     uint32_t gseq = 0;  // running voxel sequence number of this CTA: A stage = gseq % R
+    uint32_t pseq = 0;  // running voxel-pair number: exchange buffer pseq % kPairBufs
+    uint32_t ntask = 0; // tasks with a voxel loop so far (task-id handoff parity, CL = 2)
     // prior-warp lane r owns neighbour r: its offset and weight live in registers (a per-lane
     // __constant__ index would serialise in the constant cache on every voxel)
     int ndx = 0, ndy = 0, ndz = 0;
@@ -426,14 +501,24 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
     // this launch's batch: flat tasks [start, end) of the phase list (sched.cu k_flatten),
     // pulled one at a time by the persistent CTAs (dynamic distribution, Alg3:4 / T3)
     const int tstart = P.brange[0], tend = P.brange[1];
-    int* s_task = (int*)(smem + L.misc);  // [0] first task, [1] next task (fetched one ahead)
-    uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA]: this task's / the next task's band
-    if (threadIdx.x == 0) s_task[0] = tstart + atomicAdd(P.fetch, 1);
-    __syncthreads();
+    // s_task[0]: first task; s_task[1 + (n & 1)]: the task after task n (fetched one ahead by
+    // rank 0 and, CL = 2, stored into both CTAs; alternating slots so a write for task n + 1
+    // never meets a read of task n's)
+    int* s_task = (int*)(smem + L.misc);
+    uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VL]: this task's / the next task's band
+    // publish a task index (rank 0 only) into slot i of both CTAs
+    auto publish_task = [&](int i, int v) {
+        s_task[i] = v;
+        if (CL == 2) st_peer_u32(peer_addr(s_task + i, 1), (uint32_t)v);
+    };
+    if (CL == 2) cluster_sync_all();  // peer smem (mbarriers, red) initialised before any remote access
+    if (threadIdx.x == 0 && crank == 0) publish_task(0, tstart + atomicAdd(P.fetch, 1));
+    if (CL == 2) cluster_sync_all(); else __syncthreads();
     int q = s_task[0];
-    if (q < tend) band_info(P, P.flat[q], binfo, threadIdx.x, V, blockDim.x, false);
+    if (q < tend) band_info(P, P.flat[q], binfo, vbase, VL, threadIdx.x, blockDim.x);
     int tb = 0;  // binfo buffer of the current task
-    for (;; q = s_task[1], tb ^= 1) {
+    int nslot = 1;  // s_task slot of the next task
+    for (;; q = s_task[nslot], nslot ^= 3, tb ^= 1) {
         if (q >= tend) break;
         const int tk = P.flat[q];
         const int z = tk >> 14, sv = tk & 16383;  // local slice, SV
@@ -477,14 +562,15 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
         }
         const int nact = __syncthreads_count(keep);
         if (nact == 0) {  // the whole SV is zero-skipped: account for it and take the next task
-            if (threadIdx.x == 0) {
+            if (threadIdx.x == 0 && crank == 0) {
                 P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
                 atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
                 atomicAdd(P.counters + 2, 1ull);
-                s_task[1] = tstart + atomicAdd(P.fetch, 1);
+                publish_task(nslot, tstart + atomicAdd(P.fetch, 1));
             }
-            __syncthreads();
-            if (s_task[1] < tend) band_info(P, P.flat[s_task[1]], binfo + (tb ^ 1) * VA, threadIdx.x, V, blockDim.x, false);
+            if (CL == 2) cluster_sync_all(); else __syncthreads();
+            if (s_task[nslot] < tend)
+                band_info(P, P.flat[s_task[nslot]], binfo + (tb ^ 1) * VL, vbase, VL, threadIdx.x, blockDim.x);
             continue;  // the next task's x-tile barrier orders these writes before its pack
         }
 
@@ -492,6 +578,37 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
         //         voxels with a warp ballot; per-voxel scale and theta2 staged in smem; the
         //         prior warp's lane 0 then starts the TMA ring of A records (R voxels ahead)
         const size_t arec = (size_t)sv * S2;  // first A record of this SV
+        // view thread tp: asynchronous copy of its own slice of voxel j's record (this CTA's part)
+        // into stage (gseq + j) % R, one commit group per voxel (empty past the visit's end).  A
+        // thread reads back only what it copied (VPT = 1: its lane quad's offset word), so the
+        // A stream needs no cross-warp synchronisation: per-thread LDGSTS + wait_group.
+        auto copy_record = [&](int j, int tp) {
+            if (j < nact) {
+                unsigned char* st = astage + ((gseq + (uint32_t)j) % R) * L.stage_bytes;
+                const size_t rec = (arec + list[j]) * (size_t)P.A.VA + vbase;
+                if (U8) {
+                    if (VPT == 4)
+                        cp_async16(st + tp * 16, P.A.codes + rec + tp * 4);
+                    else
+                        cp_async4(st + tp * 4, P.A.codes + rec + tp);
+                } else {
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t) cp_async16(st + (tp * VPT + t) * 16, P.A.vals + rec + tp * VPT + t);
+                }
+                if (VPT == 4)
+                    cp_async4(st + L.off_in_stage + tp * 4, P.A.off + rec + tp * 4);
+                else if ((tp & 3) == 0)
+                    cp_async4(st + L.off_in_stage + tp, P.A.off + rec + tp);
+            }
+            cp_async_commit();
+        };
+        // prior warp, lane 0 (development switch MBIR_DBG bit 0): L2 warm-up of voxel j's record
+        auto prefetch_record = [&](int j) {
+            if (!(P.dbg & 1)) return;
+            const size_t rec = (arec + list[j]) * (size_t)P.A.VA + vbase;
+            l2_prefetch_bulk(U8 ? (const void*)(P.A.codes + rec) : (const void*)(P.A.vals + rec), VL * (U8 ? 4 : 16));
+            l2_prefetch_bulk(P.A.off + rec, VL);
+        };
         if (is_prior) {
             // one of NPERM host-drawn random permutations of the tile, chosen per
             // (seed, iteration, slice, SV) visit; identity (raster order) in deterministic mode
@@ -518,24 +635,12 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
             }
             __syncwarp();
             if (lane == 0) {
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                for (int i = 0; i < R && i < nact; ++i) {
-                    const uint32_t s = (gseq + i) % R;
-                    unsigned char* dst = astage + s * L.stage_bytes;
-                    const size_t rec = (arec + list[i]) * (size_t)VA;
-                    mbar_expect_tx(mbar + s, stage_tx);
-                    if (U8)
-                        tma_load_1d(dst, P.A.codes + rec, VA * 4, mbar + s);
-                    else
-                        tma_load_1d(dst, P.A.vals + rec, VA * 16, mbar + s);
-                    tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, mbar + s);
-                }
-                // and warm L2 with the next R records: every record is L2-prefetched R voxels
-                // before its TMA (the producer continues this R ahead during the loop)
-                for (int i = R; i < 2 * R && i < nact; ++i) {
-                    const size_t rec = (arec + list[i]) * (size_t)VA;
-                    l2_prefetch_bulk(U8 ? (const void*)(P.A.codes + rec) : (const void*)(P.A.vals + rec), VA * (U8 ? 4 : 16));
-                    l2_prefetch_bulk(P.A.off + rec, VA);
+                // the L2 warm-up of the records R .. 2R-1, and the next task (rank 0 fetches it;
+                // CL = 2 hands it to rank 1 through DSMEM + an mbarrier arrival)
+                for (int i = R; i < 2 * R && i < nact; ++i) prefetch_record(i);
+                if (crank == 0) {
+                    publish_task(nslot, tstart + atomicAdd(P.fetch, 1));
+                    if (CL == 2) mbar_arrive_peer(peer_addr(taskbar, 1));
                 }
             }
         }
@@ -544,7 +649,6 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
         // ---- 4. view threads: SVB pack (coalesced 128-byte band rows, transposed by shuffles);
         //         e_init rows go to this CTA's L2-resident scratch tile for the write-back
         float* scr = P.scratch + (size_t)blockIdx.x * (size_t)P.Vs * 32;
-        int pf_task = -1;  // producer warp: the next task (its band info is loaded during the loop)
         if (is_view) {
             const float* wz = P.w + (size_t)z * V * M;
             float* ez = P.e + (size_t)z * V * M;
@@ -560,16 +664,16 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
             // Two tiles are in flight: tile t + 1's loads are issued before tile t is staged.
             const int sub = lane >> 3, ch = lane & 7;  // row-in-quad and float4 chunk of this lane
             auto issue = [&](int t, bool isw, float4 (&v4)[8]) {
-                const int k0 = (vw * VPT + t) * 32;
+                const int k0 = (vw * VPT + t) * 32;  // local column of the tile's first view
                 const int kk = k0 + lane;
-                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const uint32_t bi = vbase + kk < V ? binfo[tb * VL + kk] : 0u;
                 const int bwt = (int)(bi & 31u), rot = (int)(bi >> 5);
 #pragma unroll
                 for (int m = 0; m < 8; ++m) {
                     const int i = 4 * m + sub;
                     const int oi = __shfl_sync(kFull, rot, i), wi = __shfl_sync(kFull, bwt, i);
                     const int s = oi & 3;
-                    const bool ok = k0 + i < V && 4 * ch < s + wi;
+                    const bool ok = vbase + k0 + i < V && 4 * ch < s + wi;
                     const size_t a4 = (size_t)(oi - s) + 4 * ch;
                     if (isw)
                         v4[m] = ok ? __ldg((const float4*)(wz + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
@@ -590,7 +694,7 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
             auto finish = [&](int t, bool isw, const float4 (&v4)[8]) {
                 const int k0 = (vw * VPT + t) * 32;
                 const int kk = k0 + lane;
-                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const uint32_t bi = vbase + kk < V ? binfo[tb * VL + kk] : 0u;
                 const int bwt = (int)(bi & 31u), sk = (int)(bi >> 5) & 3;
                 const uint32_t bmask = ((1u << bwt) - 1u) << sk;  // band's window positions
                 if (!isw) {
@@ -616,17 +720,6 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                 if (P.tprof && threadIdx.x == 0 && t == 0) tpc = clock64();
             }
             if (P.tprof && threadIdx.x == 0) tp1b = clock64();
-        } else if (is_prod) {
-            // producer warp: fetch the next task now; its band info (and an L2 warm-up of its
-            // band rows) is then produced a slice per voxel pair during the voxel loop, so the
-            // prefetches do not compete with this pack's loads
-            int nq = 0;
-            if (lane == 0) {
-                nq = tstart + atomicAdd(P.fetch, 1);
-                s_task[1] = nq;
-            }
-            nq = __shfl_sync(kFull, nq, 0);
-            pf_task = nq < tend ? P.flat[nq] : -1;
         }
         __syncthreads();
 
@@ -639,12 +732,15 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
         //         neighbour, then delta_b -- exactly sequential ICD in the visiting order.
         float amount = 0.f;
         const int cslot = (zc * TW + 1) * TW + 1;  // tile index of local (0,0)
-        uint64_t* full = mbar;       // full[s]: stage s holds its record (TMA bytes landed)
-        uint64_t* empty = mbar + R;  // empty[s]: every view warp has read stage s
-        const int npair_threads = (nvw + 1) * 32;  // view warps + prior warp meet per pair
-        if (!is_prod) {
+        const int npair_threads = (nvl + 1) * 32;  // view warps + prior warp meet per pair
+        {
+            // the A records of the first R voxels (every stage is free: the previous visit ended
+            // with a CTA-wide barrier)
+            if (is_view)
+                for (int i = 0; i < R; ++i) copy_record(i, vw * 32 + lane);
             for (int idx = 0; idx < nact; idx += 2) {
-                const int buf = (idx >> 1) & 1;
+                const uint32_t pn = pseq + (uint32_t)(idx >> 1);  // running pair number
+                const int buf = (int)(pn % kPairBufs);
                 const bool hasb = idx + 1 < nact;
                 const uint32_t g = gseq + idx;
                 const unsigned char* sta = astage + (g % R) * L.stage_bytes;
@@ -660,9 +756,12 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                     auto gather = [&](auto hb) {
                         constexpr bool HB = decltype(hb)::value;
                         const long long tf0 = P.tprof ? clock64() : 0;
-                        mbar_wait(full + g % R, (g / R) & 1);  // the records have landed
-                        if (HB) mbar_wait(full + (g + 1) % R, ((g + 1) / R) & 1);
-                        if (P.tprof && lane == 0) atomicAdd(P.tprof + 22 + (idx >= R), (unsigned long long)(clock64() - tf0));
+                        // this thread's copies of voxels idx, idx + 1 have landed (R voxels'
+                        // groups are in flight: idx .. idx + R - 1)
+                        cp_async_wait<R - 2>();
+                        if (VPT != 4) __syncwarp();  // offset words copied by the lane quad's first lane
+                        if (P.tprof && lane == 0)  // development aid: A-stream wait
+                            atomicAdd(P.tprof + 22 + (idx >= R), (unsigned long long)(clock64() - tf0));
                         uint32_t ca[VPT], cb[VPT], oba = 0, obb = 0;
                         load_records<VPT, U8>(sta, L.off_in_stage, tp, ca, fa, oba);
                         if (HB) load_records<VPT, U8>(stb, L.off_in_stage, tp, cb, fb, obb);
@@ -693,13 +792,6 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                                 acch = __ffma2_rn(wb1, fab[t][1], acch);
                             }
                         }
-                        // the stages are consumed (their values are in registers): release them
-                        // to the producer warp
-                        __syncwarp();
-                        if (lane == 0) {
-                            mbar_arrive(empty + g % R);
-                            if (HB) mbar_arrive(empty + (g + 1) % R);
-                        }
                         float2 gab = make_float2(acc.x + acc.y, accb.x + accb.y);
                         float hh = acch.x + acch.y;
 #pragma unroll
@@ -708,10 +800,25 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                             gab = __fadd2_rn(gab, r);
                             if (HB) hh += __shfl_xor_sync(kFull, hh, o);
                         }
+                        // the pair's stages are consumed (every lane's values are in registers and
+                        // reduced): refill them with the records R voxels ahead
+                        copy_record(idx + R, tp);
+                        copy_record(idx + 1 + R, tp);
                         if (lane == 0) {
-                            red[buf * 24 + vw] = gab.x;
-                            red[buf * 24 + 8 + vw] = gab.y;
-                            red[buf * 24 + 16 + vw] = hh;
+                            float* rs = red + buf * 24 + gvw;
+                            rs[0] = gab.x;
+                            rs[8] = gab.y;
+                            rs[16] = hh;
+                            if (CL == 2) {
+                                // the same slots of the peer CTA, then arrive on both CTAs'
+                                // pair barriers (the release orders the stores)
+                                const uint32_t pa = peer_addr(rs, crank ^ 1u);
+                                st_peer_f32(pa, gab.x);
+                                st_peer_f32(pa + 32, gab.y);
+                                st_peer_f32(pa + 64, hh);
+                                mbar_arrive_peer(peer_addr(pairbar + buf, crank ^ 1u));
+                                mbar_arrive(pairbar + buf);
+                            }
                         }
                     };
                     if (hasb)
@@ -721,13 +828,21 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                 } else if (idx == 0) {
                     // prior warp: the surrogate terms of a pair are published after the previous
                     // pair's barrier; only the first pair's are computed here
-                    prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB, pri);
+                    prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB, pri + buf);
                 }
                 {
-                    // the view warps and the prior warp meet (named barrier 1; the producer warp
-                    // runs decoupled on the full/empty mbarriers)
+                    // the view warps and the prior warp meet (CL = 1: named barrier 1; CL = 2: the
+                    // pair mbarrier, which also collects the peer CTA's view warps)
                     const long long tw0 = P.tprof ? clock64() : 0;
-                    asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
+                    if (CL == 1) {
+                        asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
+                    } else {
+                        if (is_prior) {
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive(pairbar + buf);  // pri[buf] is published
+                        }
+                        mbar_wait_cluster(pairbar + buf, (pn / kPairBufs) & 1u);
+                    }
                     if (P.tprof && lane == 0)  // development aid: per-warp wait at the pair barrier
                         atomicAdd(P.tprof + 10 + warp, (unsigned long long)(clock64() - tw0));
                 }
@@ -792,6 +907,8 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                     // prior warp: store the pair's new values, then the next pair's surrogate
                     // terms (published for the view warps before the next barrier)
                     if (lane == 0) {
+                        if (idx + 2 * R < nact) prefetch_record(idx + 2 * R);
+                        if (idx + 1 + 2 * R < nact) prefetch_record(idx + 1 + 2 * R);
                         const int ta = tof[idx];
                         xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
                         if (hasb) {
@@ -804,71 +921,14 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                     const long long tr0 = P.tprof ? clock64() : 0;
                     if (idx + 2 < nact)
                         prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
-                                   pri + (buf ^ 1));
+                                   pri + (pn + 1) % kPairBufs);
                     if (P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
-                }
-            }
-        } else if (is_prod) {
-            // producer warp, decoupled from the pair loop: first the next task's band info (and
-            // an L2 warm-up of its band rows), then the A records of voxels R .. nact-1, each as
-            // soon as the view warps have released the stage it goes to
-            if (lane == 0) {
-                const long long tq0 = P.tprof ? clock64() : 0;
-                for (int j = R; j < nact; ++j) {
-                    if (j + R < nact) {  // L2 warm-up R records ahead
-                        const size_t rp = (arec + list[j + R]) * (size_t)VA;
-                        l2_prefetch_bulk(U8 ? (const void*)(P.A.codes + rp) : (const void*)(P.A.vals + rp), VA * (U8 ? 4 : 16));
-                        l2_prefetch_bulk(P.A.off + rp, VA);
-                    }
-                    const uint32_t n = gseq + j, s = n % R;
-                    mbar_wait(empty + s, ((n / R) - 1) & 1);  // use n/R - 1 of stage s consumed
-                    unsigned char* dst = astage + s * L.stage_bytes;
-                    const size_t rec = (arec + list[j]) * (size_t)VA;
-                    mbar_expect_tx(full + s, stage_tx);
-                    if (U8)
-                        tma_load_1d(dst, P.A.codes + rec, VA * 4, full + s);
-                    else
-                        tma_load_1d(dst, P.A.vals + rec, VA * 16, full + s);
-                    tma_load_1d(dst + L.off_in_stage, P.A.off + rec, VA, full + s);
-                }
-                if (P.tprof) atomicAdd(P.tprof + 21, (unsigned long long)(clock64() - tq0));
-            }
-            __syncwarp();
-            // then the next task's band info (R voxels of loop time remain): all loads in flight
-            // at once, then the stores and the L2 warm-up of the band rows
-            if (pf_task >= 0) {
-                constexpr int KMAX = 12;  // views per lane and pass: two passes cover V <= 768
-                const int psv = pf_task & 16383, pz = pf_task >> 14;
-                uint32_t* dst = binfo + (tb ^ 1) * VA;
-#pragma unroll 1
-                for (int k0 = 0; k0 < V; k0 += 32 * KMAX) {
-                int bs[KMAX], bwd[KMAX];
-#pragma unroll
-                for (int i = 0; i < KMAX; ++i) {
-                    const int k = k0 + lane + 32 * i;
-                    if (k < V) {
-                        bs[i] = P.A.band_start[(size_t)psv * V + k];
-                        bwd[i] = P.A.band_width[(size_t)psv * V + k];
-                    }
-                }
-                const float* wz = P.w + (size_t)pz * V * M;
-                const float* ez = P.e + (size_t)pz * V * M;
-#pragma unroll
-                for (int i = 0; i < KMAX; ++i) {
-                    const int k = k0 + lane + 32 * i;
-                    if (k < V) {
-                        const int r = k * M + bs[i], r1 = r + max(bwd[i], 1) - 1;
-                        dst[k] = ((uint32_t)r << 5) | (uint32_t)bwd[i];
-                        asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
-                        asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
-                        asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
-                        asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
-                    }
-                }
                 }
             }
         }
         gseq += nact;
+        pseq += (uint32_t)(nact + 1) >> 1;
+        ++ntask;
         if (P.tprof && threadIdx.x == 0) tp3 = clock64();
         __syncthreads();
 
@@ -883,7 +943,7 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
             for (int t = 0; t < VPT; ++t) {
                 const int k0 = (vw * VPT + t) * 32;
                 const int kk = k0 + lane;
-                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const uint32_t bi = vbase + kk < V ? binfo[tb * VL + kk] : 0u;
                 const int bw = (int)(bi & 31u), roff = (int)(bi >> 5);
                 const uint32_t bmask = ((1u << bw) - 1u) << (roff & 3);
                 float4 s4[8];  // e_init windows, in flight during the staging below
@@ -905,27 +965,69 @@ __global__ void __launch_bounds__(256, 1) k_icd_sv(const IcdParams P)  // <= 6 v
                     const float e0[4] = {s4[m].x, s4[m].y, s4[m].z, s4[m].w};
 #pragma unroll
                     for (int j = 0; j < 4; ++j) d[j] = (nib & (1u << j)) ? stg_w[i * 33 + 4 * ch + j] - e0[j] : 0.f;
-                    if (k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
+                    if (vbase + k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
                         red_add_v4(ez + (oi - s) + 4 * ch, d[0], d[1], d[2], d[3]);
                 }
                 __syncwarp();
             }
-        } else if (is_prior) {
-            for (int i = lane; i < tw * th; i += 32) {
-                const int lx = i % tw, ly = i / tw;
-                P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] =
-                    xt[cslot + ly * TW + lx];
+        } else {
+            // prior warp: the image and the counters (rank 0 only), then the next task's band
+            // info with an L2 warm-up of its band rows (the next pack then reads L2)
+            if (crank == 0) {
+                for (int i = lane; i < tw * th; i += 32) {
+                    const int lx = i % tw, ly = i / tw;
+                    P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] =
+                        xt[cslot + ly * TW + lx];
+                }
+                if (lane == 0) {
+                    P.sv_amount[(size_t)z * P.nsv + sv] = amount;
+                    atomicAdd(P.counters + 0, (unsigned long long)nact);
+                    atomicAdd(P.counters + 1, (unsigned long long)(tw * th - nact));
+                    atomicAdd(P.counters + 2, 1ull);
+                    atomicAdd(P.sum_delta, (double)amount);
+                }
+            } else if (lane == 0) {
+                mbar_wait_cluster(taskbar, (ntask - 1u) & 1u);  // rank 0 published the next task
             }
-            if (lane == 0) {
-                P.sv_amount[(size_t)z * P.nsv + sv] = amount;
-                atomicAdd(P.counters + 0, (unsigned long long)nact);
-                atomicAdd(P.counters + 1, (unsigned long long)(tw * th - nact));
-                atomicAdd(P.counters + 2, 1ull);
-                atomicAdd(P.sum_delta, (double)amount);
+            __syncwarp();
+            const int nq = s_task[nslot];
+            if (nq < tend) {
+                const int nt = P.flat[nq];
+                constexpr int KMAX = 12;  // views per lane and pass: all loads in flight at once
+                const int psv = nt & 16383, pz = nt >> 14;
+                uint32_t* dst = binfo + (tb ^ 1) * VL - vbase;  // indexed by task view k
+                const int kend = min(V, vbase + VL);
+                const float* wz = P.w + (size_t)pz * V * M;
+                const float* ez = P.e + (size_t)pz * V * M;
+#pragma unroll 1
+                for (int k0 = vbase; k0 < kend; k0 += 32 * KMAX) {
+                    int bs[KMAX], bwd[KMAX];
+#pragma unroll
+                    for (int i = 0; i < KMAX; ++i) {
+                        const int k = k0 + lane + 32 * i;
+                        if (k < kend) {
+                            bs[i] = P.A.band_start[(size_t)psv * V + k];
+                            bwd[i] = P.A.band_width[(size_t)psv * V + k];
+                        }
+                    }
+#pragma unroll
+                    for (int i = 0; i < KMAX; ++i) {
+                        const int k = k0 + lane + 32 * i;
+                        if (k < kend) {
+                            const int r = k * M + bs[i], r1 = r + max(bwd[i], 1) - 1;
+                            dst[k] = ((uint32_t)r << 5) | (uint32_t)bwd[i];
+                            if (P.dbg & 2) continue;
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
+                        }
+                    }
+                }
             }
         }
-        __syncthreads();
-        if (P.tprof && threadIdx.x == 0) {
+        if (CL == 2) cluster_sync_all(); else __syncthreads();
+        if (P.tprof && threadIdx.x == 0 && crank == 0) {
             const long long tp4 = clock64();
             atomicAdd(P.tprof + 0, (unsigned long long)(tp1 - tp0));  // x tile, zero-skip, order
             atomicAdd(P.tprof + 1, (unsigned long long)(tp2 - tp1));  // SVB pack (+ first A stage)
@@ -1104,38 +1206,112 @@ __global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
 }  // namespace
 
 // A-record ring depth (voxels of TMA lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
-// (the pair loop needs >= 4: the current pair's two stages plus the next pair's two)
-constexpr int ring_depth(bool u8) { return u8 ? 8 : 4; }
+// (the pair loop needs >= 4: the current pair's two stages plus the next pair's two).  The
+// cluster variant holds half a record per stage but must fit two CTAs per SM: 6 stages.
+constexpr int ring_depth(bool u8, int cl) { return u8 ? (cl == 2 ? 6 : 8) : 4; }
 
-int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
+int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl)
 {
-    (void)vpt;
-    return smem_layout(p.rows, svb_stride(vpt), p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw).total;
+    return smem_layout(p.rows, svb_stride(vpt, cl), p.side, p.S2, nnb, p.A.VA, quantize,
+                       ring_depth(quantize, cl), p.nvw, cl).total;
 }
 
-template <int VPT, bool U8, int NNB>
+template <int VPT, bool U8, int NNB, int CL>
 static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t st)
 {
-    constexpr int R = ring_depth(U8);
-    auto kern = k_icd_sv<VPT, U8, NNB, R>;
+    constexpr int R = ring_depth(U8, CL);
+    auto kern = k_icd_sv<VPT, U8, NNB, R, CL>;
     IcdParams q = p;
-    q.lay = smem_layout(p.rows, svb_stride(VPT), p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw);
+    q.lay = smem_layout(p.rows, svb_stride(VPT, CL), p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, CL);
     const int smem = q.lay.total;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    kern<<<dim3(gx, gy), 32 * (p.nvw + 2), smem, st>>>(q);  // view warps + prior + producer
-    return cudaGetLastError();
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e != cudaSuccess) return e;
+    const int threads = 32 * (p.nvw / CL + 1);  // view warps + prior warp
+    if (CL == 1) {
+        kern<<<dim3(gx, gy), threads, smem, st>>>(q);
+        return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(gx, gy);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, q);
 }
 
-cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int gx, int gy,
+// resident CTAs of the update kernel per device (occupancy query; clusters x CL for CL = 2)
+template <int VPT, bool U8, int NNB, int CL>
+static int resident_ctas_t(const IcdParams& p)
+{
+    constexpr int R = ring_depth(U8, CL);
+    auto kern = k_icd_sv<VPT, U8, NNB, R, CL>;
+    const int smem = smem_layout(p.rows, svb_stride(VPT, CL), p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, CL).total;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
+    cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    const int threads = 32 * (p.nvw / CL + 1);
+    if (getenv("MBIR_OCC_DEBUG")) {
+        int nb = -1;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, threads, smem);
+        cudaFuncAttributes fa{};
+        cudaFuncGetAttributes(&fa, kern);
+        fprintf(stderr, "[mbir occ] CL %d threads %d smem %d blocks/SM (no cluster) %d regs %d static smem %zu local %zu\n",
+                CL, threads, smem, nb, fa.numRegs, fa.sharedSizeBytes, fa.localSizeBytes);
+    }
+    if (CL == 1) {
+        int nb = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, threads, smem) != cudaSuccess) return -1;
+        int dev = 0, nsm = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        return nb * nsm;
+    }
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(2 * 148);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int ncl = 0;
+    if (cudaOccupancyMaxActiveClusters(&ncl, kern, &cfg) != cudaSuccess) return -1;
+    return ncl * CL;
+}
+
+int icd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int cl)
+{
+    if (vpt == 1) {
+        if (quantize) return nnb == 26 ? resident_ctas_t<1, true, 26, 1>(p) : resident_ctas_t<1, true, 8, 1>(p);
+        return nnb == 26 ? resident_ctas_t<1, false, 26, 1>(p) : resident_ctas_t<1, false, 8, 1>(p);
+    }
+    if (quantize && cl == 2) return nnb == 26 ? resident_ctas_t<4, true, 26, 2>(p) : resident_ctas_t<4, true, 8, 2>(p);
+    if (quantize) return nnb == 26 ? resident_ctas_t<4, true, 26, 1>(p) : resident_ctas_t<4, true, 8, 1>(p);
+    return nnb == 26 ? resident_ctas_t<4, false, 26, 1>(p) : resident_ctas_t<4, false, 8, 1>(p);
+}
+
+cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int cl, int gx, int gy,
                        cudaStream_t st)
 {
     if (vpt == 1) {
-        if (quantize) return nnb == 26 ? launch_icd_t<1, true, 26>(p, gx, gy, st) : launch_icd_t<1, true, 8>(p, gx, gy, st);
-        return nnb == 26 ? launch_icd_t<1, false, 26>(p, gx, gy, st) : launch_icd_t<1, false, 8>(p, gx, gy, st);
+        if (quantize) return nnb == 26 ? launch_icd_t<1, true, 26, 1>(p, gx, gy, st) : launch_icd_t<1, true, 8, 1>(p, gx, gy, st);
+        return nnb == 26 ? launch_icd_t<1, false, 26, 1>(p, gx, gy, st) : launch_icd_t<1, false, 8, 1>(p, gx, gy, st);
     }
-    if (quantize) return nnb == 26 ? launch_icd_t<4, true, 26>(p, gx, gy, st) : launch_icd_t<4, true, 8>(p, gx, gy, st);
-    return nnb == 26 ? launch_icd_t<4, false, 26>(p, gx, gy, st) : launch_icd_t<4, false, 8>(p, gx, gy, st);
+    if (quantize && cl == 2)
+        return nnb == 26 ? launch_icd_t<4, true, 26, 2>(p, gx, gy, st) : launch_icd_t<4, true, 8, 2>(p, gx, gy, st);
+    if (quantize) return nnb == 26 ? launch_icd_t<4, true, 26, 1>(p, gx, gy, st) : launch_icd_t<4, true, 8, 1>(p, gx, gy, st);
+    return nnb == 26 ? launch_icd_t<4, false, 26, 1>(p, gx, gy, st) : launch_icd_t<4, false, 8, 1>(p, gx, gy, st);
 }
 
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st)

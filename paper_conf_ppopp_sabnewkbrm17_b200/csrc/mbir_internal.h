@@ -88,6 +88,8 @@ struct IcdParams {
     int zero_skip_active;
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
+    int dbg;                 // development switches (env MBIR_DBG): bit 0 no A-record L2 warm-up,
+                             // bit 1 no band-row L2 warm-up
     SmemLayout lay;          // update-kernel smem layout (filled by launch_icd)
 };
 
@@ -109,9 +111,12 @@ cudaError_t set_prior_constants(const PriorConst& pc);
 cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, int side, int nsvx,
                             int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxoff,
                             cudaStream_t st);
-int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize);
-cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid_x, int grid_y,
-                       cudaStream_t st);
+// cl: CTAs per SV task (1, or 2 = a thread-block cluster splitting the views; uint8 A, vpt 4,
+// an even number of view warps)
+int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
+int icd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
+cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int cl, int grid_x,
+                       int grid_y, cudaStream_t st);
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st);
 cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cudaStream_t st);
 cudaError_t launch_probe(const IcdParams& p, bool quantize, int nnb, const int64_t* vox, int n,

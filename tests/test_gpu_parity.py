@@ -316,3 +316,76 @@ def test_invalid_arguments_rejected():
         y[0, 0, 0] = np.nan
         with pytest.raises(M.MbirError):
             r.set_sinogram(y, np.ones_like(y))
+
+
+# ------------------------------------------------------------------ the bench's launch shape
+def mini720():
+    """The bench's kernel shape on an image the oracle handles: 720 views (4 views per lane, six
+    128-view warps), channel pitch dxy/2 as in the paper geometry (K = 4, 2.4K nnz per voxel),
+    SV side 9 with a ragged last SV column/row, two slices, 26-neighbourhood."""
+    return WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005)
+
+
+@pytest.fixture(scope="module")
+def m720():
+    cfg = mini720()
+    case = make_case(cfg)
+    g, og = geoms(cfg)
+    A = O.sysmatrix(og)
+    _, _, Aq = O.quantize(A)
+    return cfg, case, g, og, Aq
+
+
+@pytest.mark.parametrize("cluster", [1, 2])
+def test_bench_shape_deterministic_tracks_oracle(m720, cluster):
+    """The launch configuration bench.py times (uint8 A, 4 views per lane, 6 view warps, one CTA
+    or a 2-CTA cluster per task): deterministic order, 2 equits, against the sequential oracle."""
+    cfg, case, g, og, Aq = m720
+    pr = O.Prior(sigma=cfg.sigma, nbhd=26)
+    order = deterministic_order(cfg.n, cfg.nz, cfg.sv_side, 26)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
+                         M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0, cluster=cluster)) as r:
+        assert r.sizes()["cluster"] == cluster
+        r.set_sinogram(case.y, case.w)
+        x = np.zeros(cfg.nz * cfg.n * cfg.n)
+        e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+        for it in range(2):
+            st = r.iterate(1)
+            assert st["updates"] == x.size and st["skipped"] == 0
+            O.icd_run(og, pr, Aq, case.w, x, e, 1, zero_skip=False, order=order)
+            xg = r.image().ravel()
+            err = np.abs(xg - x).max() / np.abs(x).max()
+            assert err < 3e-5 * (it + 1), (it, err)
+        eg = r.error_sinogram()
+    assert np.abs(eg.ravel() - e.ravel()).max() < 1e-4 * np.abs(case.y).max()
+
+
+@pytest.mark.parametrize("cluster", [1, 2])
+def test_bench_shape_converged_matches_oracle(m720, cluster):
+    """Asynchronous GPU-ICD in the bench's launch shape (persistent grid, random orders, 25 %
+    SV selection, zero-skipping off) reaches the oracle's MAP point: 1 HU / 1e-4."""
+    cfg, case, g, og, Aq = m720
+    pr = O.Prior(sigma=cfg.sigma, nbhd=26)
+    x = np.zeros(cfg.nz * cfg.n * cfg.n)
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+    O.icd_run(og, pr, Aq, case.w, x, e, 80, seed=3000, zero_skip=False)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
+                         M.Options(sv_side=cfg.sv_side, zero_skip=0, cluster=cluster)) as r:
+        r.set_sinogram(case.y, case.w)
+        r.reconstruct(200)
+        xg = r.image().ravel().astype(np.float64)
+    assert O.rmse_hu(xg, x) < 1.0
+    cg = O.cost(og, pr, Aq, case.y, case.w, xg)
+    co = O.cost(og, pr, Aq, case.y, case.w, x)
+    assert abs(cg - co) <= 1e-4 * abs(co), (cg, co)
+
+
+def test_cluster_option_validation():
+    """cluster = 2 needs uint8 A and an even number of 128-view warps (include/mbir.h)."""
+    cfg = CONFIGS["cfg1"]  # 90 views: one warp of 1 view per lane
+    g, _ = geoms(cfg)
+    with pytest.raises(M.MbirError) as ei:
+        M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side, cluster=2))
+    assert ei.value.code == -1
+    with M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side)) as r:
+        assert r.sizes()["cluster"] == 1

@@ -19,13 +19,14 @@ ap.add_argument("--iters", type=int, default=12)
 ap.add_argument("--zero-skip", type=int, default=1)
 ap.add_argument("--sv-side", type=int, default=0)
 ap.add_argument("--batch-svs", type=int, default=0)
+ap.add_argument("--cluster", type=int, default=0)
 a = ap.parse_args()
 cfg = CONFIGS[a.config]
 y, w = make_sinogram_torch(cfg, 0, "cuda")
 g = M.Geometry(cfg.n, cfg.n, cfg.nz, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dchannel)
 r = M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=cfg.nbhd),
                     M.Options(sv_side=a.sv_side or cfg.sv_side, zero_skip=a.zero_skip,
-                              batch_svs=a.batch_svs))
+                              batch_svs=a.batch_svs, cluster=a.cluster))
 r.set_sinogram(y, w)
 print(json.dumps(r.sizes()))
 for rep in range(2):
