@@ -568,9 +568,11 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     h->A.V = G.nviews;
     // ---- update-kernel shape: fat view warps (4 views per lane, <= 6 warps) keep the per-voxel
     // per-warp overhead (reduction, barrier, delta) small; tiny view counts use 1 per lane
+    // (2 views per lane in 12 view warps was measured too: 13 warps leave 128 registers per
+    // thread and the gather spills)
     h->vpt = G.nviews > 128 ? 4 : 1;
     h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
-    if (h->nvw > 6) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
+    if (h->nvw * h->vpt > 24) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
     h->Vs = h->nvw * 32 * h->vpt;
     h->A.vpt = h->vpt;
     h->A.VA = h->Vs;  // thread-major record positions (apos); a multiple of 32 -> TMA-sized

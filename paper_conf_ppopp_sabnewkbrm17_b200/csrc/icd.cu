@@ -103,46 +103,13 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z)
     return z ^ (z >> 31);
 }
 
-struct PriSlot {
-    float sb, sbx, v, pad;
+// Neighbour slots of a prior-warp lane: half-warp h = lane >> 4 works on voxel a (h = 0) or b
+// (h = 1) of a pair; its lane i owns neighbours i and i + 16 of the neighbourhood (reading R2):
+// offset (dx, dy, dz), tile-index offset dt and weight w (0: no neighbour)
+struct NbrLane {
+    int dx[2], dy[2], dz[2], dt[2];
+    float w[2];
 };
-
-// q-GGMRF surrogate sums of Alg1:7 for the voxel at packed tile coordinate tofv (ly << 8 | lx):
-// lane r < nnb owns neighbour r (offset ndx/ndy/ndz, weight nbw); returns the warp-reduced
-// sums sbv = sum b_r phi(v - x_r) and sbx = sum b_r phi(v - x_r) x_r, plus this lane's own
-// (bt, xr) and the voxel's value v.  Free boundary: off-image neighbours contribute nothing.
-// Neighbours at packed tile positions ov0 / ov1 (same slice) take the values xv0 / xv1 instead
-// of the tile's: the voxels just updated, whose new values the calling warp holds in registers
-// before they are stored to the tile.
-__device__ __forceinline__ void prior_terms(int tofv, const float* xt, int cslot, int TW, int gx0,
-                                            int gy0, int zg, const IcdParams& P, int ndx, int ndy,
-                                            int ndz, float nbw, int lane, int nnb, float& sbv,
-                                            float& sbx, float& bt, float& xr, float& v,
-                                            int ov0 = -1 << 20, float xv0 = 0.f, int ov1 = -1 << 20,
-                                            float xv1 = 0.f)
-{
-    const int lx = tofv & 255, ly = tofv >> 8;
-    v = xt[cslot + ly * TW + lx];
-    bt = 0.f;
-    xr = 0.f;
-    if (lane < nnb) {
-        const int gx = gx0 + lx + ndx, gy = gy0 + ly + ndy, gz = zg + ndz;
-        if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
-            xr = xt[cslot + (ndz * TW + ly + ndy) * TW + lx + ndx];
-            const int pos = ndz == 0 ? ((ly + ndy) << 8) + lx + ndx : -2 << 20;
-            if (pos == ov0) xr = xv0;
-            if (pos == ov1) xr = xv1;
-            bt = nbw * phi_f(v - xr);
-        }
-    }
-    sbv = bt;
-    sbx = bt * xr;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        sbv += __shfl_xor_sync(kFull, sbv, o);
-        sbx += __shfl_xor_sync(kFull, sbx, o);
-    }
-}
 
 // surrogate terms of a pair of consecutive voxels (a, b): a's sums, b's sums computed with a's
 // OLD value, and -- if a is b's neighbour -- that neighbour's term (btab) and weight (bab)
@@ -150,12 +117,19 @@ struct PriPair {
     float sa, sxa, va, sb, sxb, vb, btab, bab;
 };
 
-// sum of 8 consecutive floats (16-byte aligned) with paired-fp32 adds
-__device__ __forceinline__ float sum8(const float* r)
+// sum of NS (8 or 16) consecutive floats (16-byte aligned) with paired-fp32 adds, in a fixed
+// order (every warp of the task gets the same bits)
+template <int NS>
+__device__ __forceinline__ float sum_slots(const float* r)
 {
     const float4 a = ((const float4*)r)[0], b = ((const float4*)r)[1];
-    const float2 s = __fadd2_rn(__fadd2_rn(make_float2(a.x, a.y), make_float2(a.z, a.w)),
-                                __fadd2_rn(make_float2(b.x, b.y), make_float2(b.z, b.w)));
+    float2 s = __fadd2_rn(__fadd2_rn(make_float2(a.x, a.y), make_float2(a.z, a.w)),
+                          __fadd2_rn(make_float2(b.x, b.y), make_float2(b.z, b.w)));
+    if (NS == 16) {
+        const float4 c = ((const float4*)r)[2], d = ((const float4*)r)[3];
+        s = __fadd2_rn(s, __fadd2_rn(__fadd2_rn(make_float2(c.x, c.y), make_float2(c.z, c.w)),
+                                     __fadd2_rn(make_float2(d.x, d.y), make_float2(d.z, d.w))));
+    }
     return s.x + s.y;
 }
 
@@ -199,7 +173,7 @@ __device__ __forceinline__ void shifted(uint32_t cw, const float2 (&a)[2], int d
 }
 
 // this thread's VPT adjacent A records (apos) from a stage: code words + dequantised values as
-// channel pairs, and (VPT == 4) the 4 band offsets packed in one word
+// channel pairs, and (VPT 2, 4) the band offsets packed in one word
 template <int VPT, bool U8>
 __device__ __forceinline__ void load_records(const unsigned char* stg, int off_in_stage, int tp,
                                              uint32_t (&cw)[VPT], float2 (&f)[VPT][2], uint32_t& ob)
@@ -211,6 +185,10 @@ __device__ __forceinline__ void load_records(const unsigned char* stg, int off_i
             cw[VPT > 1 ? 1 : 0] = c4.y;
             cw[VPT > 2 ? 2 : 0] = c4.z;
             cw[VPT > 3 ? 3 : 0] = c4.w;
+        } else if (VPT == 2) {
+            const uint2 c2 = ((const uint2*)stg)[tp];
+            cw[0] = c2.x;
+            cw[VPT > 1 ? 1 : 0] = c2.y;
         } else {
 #pragma unroll
             for (int t = 0; t < VPT; ++t) cw[t] = ((const uint32_t*)stg)[tp * VPT + t];
@@ -230,34 +208,66 @@ __device__ __forceinline__ void load_records(const unsigned char* stg, int off_i
         }
     }
     if (VPT == 4) ob = ((const uint32_t*)(stg + off_in_stage))[tp];
+    if (VPT == 2) ob = ((const uint16_t*)(stg + off_in_stage))[tp];
 }
 
-// prior warp: PriPair for voxels (i0, i0+1) of the visiting order from the current x tile
+// prior warp: PriPair for voxels (i0, i0+1) of the visiting order from the current x tile.
+// Alg1:7's q-GGMRF surrogate sums sb = sum_r b_r phi(v - x_r), sx = sum_r b_r phi(v - x_r) x_r
+// over the neighbourhood (free boundary: off-image neighbours contribute nothing), voxel a on
+// lanes 0-15 and voxel b (with a's OLD value) on lanes 16-31, two neighbours per lane, so both
+// voxels' terms are one latency chain and a 4-level half-warp reduction.
 __device__ __forceinline__ void prior_pair(const int* tof, int i0, int nact, const float* xt, int cslot,
                                            int TW, int gx0, int gy0, int zg, const IcdParams& P,
-                                           int ndx, int ndy, int ndz, float nbw, int lane, int nnb,
-                                           PriPair* out)
+                                           const NbrLane& nb, int lane, PriPair* out)
 {
-    const int ta = tof[i0];
-    float s0, x0, bt0, xr0, v0;
-    prior_terms(ta, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, nnb, s0, x0, bt0, xr0, v0);
-    PriPair pp{s0, x0, v0, 0.f, 0.f, 0.f, 0.f, 0.f};
-    if (i0 + 1 < nact) {
-        const int tb = tof[i0 + 1];
-        float s1, x1, bt1, xr1, v1;
-        prior_terms(tb, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, nnb, s1, x1, bt1, xr1, v1);
-        pp.sb = s1;
-        pp.sxb = x1;
-        pp.vb = v1;
-        const int dx = (ta & 255) - (tb & 255), dy = (ta >> 8) - (tb >> 8);
-        if (dx >= -1 && dx <= 1 && dy >= -1 && dy <= 1) {
-            const bool mine = lane < nnb && ndx == dx && ndy == dy && ndz == 0;
-            const int src = __ffs(__ballot_sync(0xffffffffu, mine)) - 1;
-            pp.btab = __shfl_sync(0xffffffffu, bt1, src);
-            pp.bab = __shfl_sync(0xffffffffu, nbw, src);
+    const bool hasb = i0 + 1 < nact;
+    const int ta = tof[i0], tb = hasb ? tof[i0 + 1] : ta;
+    const int tv = lane < 16 ? ta : tb;
+    const int lx = tv & 255, ly = tv >> 8;
+    const int c0 = cslot + ly * TW + lx;
+    const float v = xt[c0];
+    float sb = 0.f, sx = 0.f, btn = 0.f, bwn = 0.f;  // btn, bwn: this lane's term / weight whose
+    bool mine = false;                               // neighbour is voxel a
+    const int dxa = (ta & 255) - lx, dya = (ta >> 8) - ly;  // a relative to this half's voxel
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const int gx = gx0 + lx + nb.dx[k], gy = gy0 + ly + nb.dy[k], gz = zg + nb.dz[k];
+        if (nb.w[k] != 0.f && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
+            const float xr = xt[c0 + nb.dt[k]];
+            const float bt = nb.w[k] * phi_f(v - xr);
+            sb += bt;
+            sx += bt * xr;
+            if (nb.dz[k] == 0 && nb.dx[k] == dxa && nb.dy[k] == dya) {
+                btn = bt;
+                bwn = nb.w[k];
+                mine = true;
+            }
         }
     }
-    if (lane == 0) *out = pp;
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) {
+        sb += __shfl_xor_sync(kFull, sb, o);
+        sx += __shfl_xor_sync(kFull, sx, o);
+    }
+    // a's neighbour term in b's sums (a and b are distinct voxels, so only lanes >= 16 can own it)
+    const unsigned who = __ballot_sync(kFull, mine && lane >= 16 && hasb);
+    const int src = who ? __ffs(who) - 1 : 0;
+    const float btab = __shfl_sync(kFull, btn, src);
+    const float bab = __shfl_sync(kFull, bwn, src);
+    const float sbb = __shfl_sync(kFull, sb, 16), sxb = __shfl_sync(kFull, sx, 16), vb = __shfl_sync(kFull, v, 16);
+    if (lane == 0) {
+        PriPair pp{sb, sx, v, 0.f, 0.f, 0.f, 0.f, 0.f};
+        if (hasb) {
+            pp.sb = sbb;
+            pp.sxb = sxb;
+            pp.vb = vb;
+            if (who) {
+                pp.btab = btab;
+                pp.bab = bab;
+            }
+        }
+        *out = pp;
+    }
 }
 
 // ---- TMA (cp.async.bulk) + mbarrier helpers for the A-record ring ----
@@ -292,6 +302,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
 __device__ __forceinline__ void cp_async16(void* dst, const void* src)
 {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* dst, const void* src)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async4(void* dst, const void* src)
 {
@@ -363,9 +377,13 @@ __device__ __forceinline__ void cluster_sync_all()
 
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
 
-// the update kernel's SVB column stride: the most views one CTA can hold (6 / CL view warps x
-// 32 lanes x VPT views), fixed at compile time whatever the actual view count
-__host__ __device__ constexpr int svb_stride(int vpt, int cl = 1) { return 6 / cl * 32 * vpt; }
+// the update kernel's SVB column stride: the most views one CTA can hold (VPT = 1: 6 view warps
+// of 32; VPT >= 2: 768 views = 24 / VPT view warps, / CL), fixed at compile time whatever the
+// actual view count
+__host__ __device__ constexpr int svb_stride(int vpt, int cl = 1) { return (vpt == 1 ? 192 : 768) / cl; }
+
+// partial-sum slots per quantity in the pair exchange (>= view warps of a task)
+__host__ __device__ constexpr int red_slots(int vpt) { return vpt == 2 ? 16 : 8; }
 
 // pair-exchange buffers of the update kernel (red partials / prior terms): the cluster variant
 // needs 3 (a CTA can run one pair ahead of its peer), 4 keeps the index a mask
@@ -387,7 +405,7 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.list = o;  o = align16(o + S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
     L.tof = o;   o = align16(o + S2 * 4);
-    L.red = o;   o = align16(o + kPairBufs * 24 * 4);  // [bufs][3 quantities][8 view warps]
+    L.red = o;   o = align16(o + kPairBufs * 3 * 16 * 4);  // [bufs][3 quantities][<= 16 view warps]
     L.pri = o;   o = align16(o + kPairBufs * (int)sizeof(PriPair));
     L.vscale = o; o = align16(o + S2 * 4);
     L.vth2 = o;  o = align16(o + S2 * 4);
@@ -422,10 +440,10 @@ __device__ __forceinline__ void band_info(const IcdParams& P, int tk, uint32_t* 
 // CTAs per SM; per voxel pair the CTAs exchange their partial sums through distributed shared
 // memory, so both derive the same deltas.  Two independent tasks per SM let one CTA's pack and
 // write-back overlap the other's voxel loop.
-// CL = 1: one CTA of <= 6 view warps + the prior warp per SM; CL = 2: two CTAs of 3 view warps +
-// the prior warp per SM (8 warps: the full register budget per thread)
+// CL = 1: one CTA per SM of <= 6 (VPT 1, 4) or 12 (VPT 2) view warps + the prior warp; CL = 2:
+// two CTAs of 3 view warps + the prior warp per SM (8 warps: the full register budget)
 template <int VPT, bool U8, int NNB, int R, int CL>
-__global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv(const IcdParams P)
+__global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 1 ? 1 : 2) k_icd_sv(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -444,6 +462,7 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
     const int VL = P.A.VA / CL;          // record positions / SVB columns of this CTA
     const int vbase = (int)crank * VL;   // first view (and record position) of this CTA
     constexpr int VS = svb_stride(VPT, CL);  // SVB view stride: compile-time, so row offsets are immediates
+    constexpr int NSL = red_slots(VPT);      // pair-exchange slots per quantity
     const SmemLayout& L = P.lay;
     float* sb_e = (float*)(smem + L.sb_e);
     float* sb_w = (float*)(smem + L.sb_w);
@@ -464,7 +483,7 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
     uint64_t* pairbar = mbar;              // [kPairBufs] (CL = 2): both CTAs' partials + prior terms
     uint64_t* taskbar = pairbar + kPairBufs;  // (CL = 2, rank 1): the next task id has arrived
 
-    if (threadIdx.x < kPairBufs * 24) red[threadIdx.x] = 0.f;  // slots >= nvw stay zero
+    for (int i = threadIdx.x; i < kPairBufs * 3 * NSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay zero
     // SVB rows outside a visit's band are never packed: start them finite (zero)
     for (int i = threadIdx.x; i < (L.sb_w - L.sb_e) / 16; i += blockDim.x) {
         ((float4*)(smem + L.sb_e))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -489,13 +508,16 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
     uint32_t ntask = 0; // tasks with a voxel loop so far (task-id handoff parity, CL = 2)
     // prior-warp lane r owns neighbour r: its offset and weight live in registers (a per-lane
     // __constant__ index would serialise in the constant cache on every voxel)
-    int ndx = 0, ndy = 0, ndz = 0;
-    float nbw = 0.f;
-    if (lane < c_prior.nnb) {
-        ndx = c_prior.dx[lane];
-        ndy = c_prior.dy[lane];
-        ndz = c_prior.dz[lane];
-        nbw = c_prior.b[lane];
+    NbrLane nb;
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const int r = (lane & 15) + 16 * k;
+        const bool ok = r < c_prior.nnb;
+        nb.dx[k] = ok ? c_prior.dx[r] : 0;
+        nb.dy[k] = ok ? c_prior.dy[r] : 0;
+        nb.dz[k] = ok ? c_prior.dz[r] : 0;
+        nb.w[k] = ok ? c_prior.b[r] : 0.f;
+        nb.dt[k] = (nb.dz[k] * (side + 2) + nb.dy[k]) * (side + 2) + nb.dx[k];
     }
 
     // this launch's batch: flat tasks [start, end) of the phase list (sched.cu k_flatten),
@@ -589,16 +611,17 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                 if (U8) {
                     if (VPT == 4)
                         cp_async16(st + tp * 16, P.A.codes + rec + tp * 4);
+                    else if (VPT == 2)
+                        cp_async8(st + tp * 8, P.A.codes + rec + tp * 2);
                     else
                         cp_async4(st + tp * 4, P.A.codes + rec + tp);
                 } else {
 #pragma unroll
                     for (int t = 0; t < VPT; ++t) cp_async16(st + (tp * VPT + t) * 16, P.A.vals + rec + tp * VPT + t);
                 }
-                if (VPT == 4)
-                    cp_async4(st + L.off_in_stage + tp * 4, P.A.off + rec + tp * 4);
-                else if ((tp & 3) == 0)
-                    cp_async4(st + L.off_in_stage + tp, P.A.off + rec + tp);
+                // offsets: VPT bytes per thread, copied as 4-byte words by every (4 / VPT)-th lane
+                if ((tp & (4 / VPT - 1)) == 0)
+                    cp_async4(st + L.off_in_stage + tp * VPT, P.A.off + rec + tp * VPT);
             }
             cp_async_commit();
         };
@@ -765,7 +788,9 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                         uint32_t ca[VPT], cb[VPT], oba = 0, obb = 0;
                         load_records<VPT, U8>(sta, L.off_in_stage, tp, ca, fa, oba);
                         if (HB) load_records<VPT, U8>(stb, L.off_in_stage, tp, cb, fb, obb);
-                        float2 acc = make_float2(0.f, 0.f), accb = acc, acch = acc;
+                        // two accumulator sets (even / odd views) halve the FFMA2 dependency chains
+                        float2 acc[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+                        float2 accb[2] = {acc[0], acc[0]}, acch[2] = {acc[0], acc[0]};
 #pragma unroll
                         for (int t = 0; t < VPT; ++t) {
                             // padded views (k >= V) have zero A: no per-view branch
@@ -775,8 +800,8 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                             ea[t][0] = make_float2(pe[0], pe[VS]);
                             ea[t][1] = make_float2(pe[2 * VS], pe[3 * VS]);
                             const float2 w0 = make_float2(pw[0], pw[VS]), w1 = make_float2(pw[2 * VS], pw[3 * VS]);
-                            acc = __ffma2_rn(__fmul2_rn(w0, ea[t][0]), fa[t][0], acc);
-                            acc = __ffma2_rn(__fmul2_rn(w1, ea[t][1]), fa[t][1], acc);
+                            acc[t & 1] = __ffma2_rn(__fmul2_rn(w0, ea[t][0]), fa[t][0], acc[t & 1]);
+                            acc[t & 1] = __ffma2_rn(__fmul2_rn(w1, ea[t][1]), fa[t][1], acc[t & 1]);
                             if (HB) {
                                 ob[t] = VPT == 4 ? (int)((obb >> (8 * t)) & 255u) : (int)stb[L.off_in_stage + tp * VPT + t];
                                 shifted<U8>(ca[t], fa[t], ob[t] - oa[t], fab[t]);  // A_a on b's channels
@@ -786,14 +811,16 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                                 eb[t][1] = make_float2(qe[2 * VS], qe[3 * VS]);
                                 const float2 wb0 = __fmul2_rn(make_float2(qw[0], qw[VS]), fb[t][0]);
                                 const float2 wb1 = __fmul2_rn(make_float2(qw[2 * VS], qw[3 * VS]), fb[t][1]);
-                                accb = __ffma2_rn(wb0, eb[t][0], accb);
-                                accb = __ffma2_rn(wb1, eb[t][1], accb);
-                                acch = __ffma2_rn(wb0, fab[t][0], acch);
-                                acch = __ffma2_rn(wb1, fab[t][1], acch);
+                                accb[t & 1] = __ffma2_rn(wb0, eb[t][0], accb[t & 1]);
+                                accb[t & 1] = __ffma2_rn(wb1, eb[t][1], accb[t & 1]);
+                                acch[t & 1] = __ffma2_rn(wb0, fab[t][0], acch[t & 1]);
+                                acch[t & 1] = __ffma2_rn(wb1, fab[t][1], acch[t & 1]);
                             }
                         }
-                        float2 gab = make_float2(acc.x + acc.y, accb.x + accb.y);
-                        float hh = acch.x + acch.y;
+                        const float2 ac = __fadd2_rn(acc[0], acc[1]), acb = __fadd2_rn(accb[0], accb[1]);
+                        const float2 ach = __fadd2_rn(acch[0], acch[1]);
+                        float2 gab = make_float2(ac.x + ac.y, acb.x + acb.y);
+                        float hh = ach.x + ach.y;
 #pragma unroll
                         for (int o = 16; o > 0; o >>= 1) {
                             const float2 r = make_float2(__shfl_xor_sync(kFull, gab.x, o), __shfl_xor_sync(kFull, gab.y, o));
@@ -805,17 +832,17 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                         copy_record(idx + R, tp);
                         copy_record(idx + 1 + R, tp);
                         if (lane == 0) {
-                            float* rs = red + buf * 24 + gvw;
+                            float* rs = red + buf * 3 * NSL + gvw;
                             rs[0] = gab.x;
-                            rs[8] = gab.y;
-                            rs[16] = hh;
+                            rs[NSL] = gab.y;
+                            rs[2 * NSL] = hh;
                             if (CL == 2) {
                                 // the same slots of the peer CTA, then arrive on both CTAs'
                                 // pair barriers (the release orders the stores)
                                 const uint32_t pa = peer_addr(rs, crank ^ 1u);
                                 st_peer_f32(pa, gab.x);
-                                st_peer_f32(pa + 32, gab.y);
-                                st_peer_f32(pa + 64, hh);
+                                st_peer_f32(pa + 4 * NSL, gab.y);
+                                st_peer_f32(pa + 8 * NSL, hh);
                                 mbar_arrive_peer(peer_addr(pairbar + buf, crank ^ 1u));
                                 mbar_arrive(pairbar + buf);
                             }
@@ -828,7 +855,7 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                 } else if (idx == 0) {
                     // prior warp: the surrogate terms of a pair are published after the previous
                     // pair's barrier; only the first pair's are computed here
-                    prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB, pri + buf);
+                    prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + buf);
                 }
                 {
                     // the view warps and the prior warp meet (CL = 1: named barrier 1; CL = 2: the
@@ -847,8 +874,8 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                         atomicAdd(P.tprof + 10 + warp, (unsigned long long)(clock64() - tw0));
                 }
                 // every warp derives the same two deltas (identical inputs, identical order)
-                const float* rb = red + buf * 24;  // nvw <= 8 partials per quantity, rest 0
-                const float sa = sum8(rb), sbs = sum8(rb + 8), sh = sum8(rb + 16);
+                const float* rb = red + buf * 3 * NSL;  // nvw <= NSL partials per quantity, rest 0
+                const float sa = sum_slots<NSL>(rb), sbs = sum_slots<NSL>(rb + NSL), sh = sum_slots<NSL>(rb + 2 * NSL);
                 const PriPair pp = pri[buf];
                 const float scale_a = vscale[idx];
                 float ua = pp.va;
@@ -886,7 +913,7 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                     // a's channels
                     const float sda = scale_a * da, sdb = scale_b * db;
                     if (sda != 0.f || sdb != 0.f) {
-                        const float2 na = make_float2(-sda, -sda), nb = make_float2(-sdb, -sdb);
+                        const float2 na = make_float2(-sda, -sda), ndb = make_float2(-sdb, -sdb);
                         auto put2 = [&](float* p, float2 v0, float2 v1) {
                             p[0] = v0.x;
                             p[VS] = v0.y;
@@ -899,8 +926,8 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                                  __ffma2_rn(fa[t][1], na, ea[t][1]));
                             if (hasb)
                                 put2(sb_e + ob[t] * VS + kv[t],
-                                     __ffma2_rn(fb[t][0], nb, __ffma2_rn(fab[t][0], na, eb[t][0])),
-                                     __ffma2_rn(fb[t][1], nb, __ffma2_rn(fab[t][1], na, eb[t][1])));
+                                     __ffma2_rn(fb[t][0], ndb, __ffma2_rn(fab[t][0], na, eb[t][0])),
+                                     __ffma2_rn(fb[t][1], ndb, __ffma2_rn(fab[t][1], na, eb[t][1])));
                         }
                     }
                 } else {
@@ -920,7 +947,7 @@ __global__ void __launch_bounds__(CL == 1 ? 224 : 128, CL == 1 ? 1 : 2) k_icd_sv
                     __syncwarp();
                     const long long tr0 = P.tprof ? clock64() : 0;
                     if (idx + 2 < nact)
-                        prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, ndx, ndy, ndz, nbw, lane, NNB,
+                        prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
                                    pri + (pn + 1) % kPairBufs);
                     if (P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
                 }
