@@ -604,24 +604,32 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
         // into stage (gseq + j) % R, one commit group per voxel (empty past the visit's end).  A
         // thread reads back only what it copied (VPT = 1: its lane quad's offset word), so the
         // A stream needs no cross-warp synchronisation: per-thread LDGSTS + wait_group.
+        // (per-task bases: this thread's slice of the SV's records in global memory and of a stage)
+        constexpr int CB = U8 ? 4 : 16;  // record bytes per view position
+        const int tpm = vw * 32 + lane;
+        const unsigned char* g_code = (const unsigned char*)(U8 ? (const void*)P.A.codes : (const void*)P.A.vals) +
+                                      ((size_t)arec * P.A.VA + vbase + tpm * VPT) * CB;
+        const unsigned char* g_off = P.A.off + (size_t)arec * P.A.VA + vbase + tpm * VPT;
         auto copy_record = [&](int j, int tp) {
+            (void)tp;
             if (j < nact) {
                 unsigned char* st = astage + ((gseq + (uint32_t)j) % R) * L.stage_bytes;
-                const size_t rec = (arec + list[j]) * (size_t)P.A.VA + vbase;
+                const int v = list[j];
+                const unsigned char* gc = g_code + (size_t)v * (P.A.VA * CB);
                 if (U8) {
                     if (VPT == 4)
-                        cp_async16(st + tp * 16, P.A.codes + rec + tp * 4);
+                        cp_async16(st + tpm * 16, gc);
                     else if (VPT == 2)
-                        cp_async8(st + tp * 8, P.A.codes + rec + tp * 2);
+                        cp_async8(st + tpm * 8, gc);
                     else
-                        cp_async4(st + tp * 4, P.A.codes + rec + tp);
+                        cp_async4(st + tpm * 4, gc);
                 } else {
 #pragma unroll
-                    for (int t = 0; t < VPT; ++t) cp_async16(st + (tp * VPT + t) * 16, P.A.vals + rec + tp * VPT + t);
+                    for (int t = 0; t < VPT; ++t) cp_async16(st + (tpm * VPT + t) * 16, gc + t * 16);
                 }
                 // offsets: VPT bytes per thread, copied as 4-byte words by every (4 / VPT)-th lane
-                if ((tp & (4 / VPT - 1)) == 0)
-                    cp_async4(st + L.off_in_stage + tp * VPT, P.A.off + rec + tp * VPT);
+                if ((tpm & (4 / VPT - 1)) == 0)
+                    cp_async4(st + L.off_in_stage + tpm * VPT, g_off + (size_t)v * P.A.VA);
             }
             cp_async_commit();
         };
@@ -720,13 +728,14 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
                 const uint32_t bi = vbase + kk < V ? binfo[tb * VL + kk] : 0u;
                 const int bwt = (int)(bi & 31u), sk = (int)(bi >> 5) & 3;
                 const uint32_t bmask = ((1u << bwt) - 1u) << sk;  // band's window positions
-                if (!isw) {
+                if (!isw && !(P.dbg & 128)) {  // (dbg 128: timing ablation)
 #pragma unroll
                     for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), v4[m]);
                 }
                 float* d = (isw ? sb_w : sb_e) + kk - sk * VS;  // + p * VS = band column p - sk of view kk
                 const float* sr = stg_w + lane * 33;
                 put(v4);
+                if (P.tprof && threadIdx.x == 0 && t == 0 && isw) tpb = clock64();
 #pragma unroll
                 for (int p = 0; p < 32; ++p)
                     if (bmask & (1u << p)) d[p * VS] = sr[p];
@@ -862,7 +871,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
                     // pair mbarrier, which also collects the peer CTA's view warps)
                     const long long tw0 = P.tprof ? clock64() : 0;
                     if (CL == 1) {
-                        asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
+                        if (!(P.dbg & 64)) asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
                     } else {
                         if (is_prior) {
                             __syncwarp();
@@ -912,7 +921,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
                     // entries the two voxels share with the full value, so A_b is never needed on
                     // a's channels
                     const float sda = scale_a * da, sdb = scale_b * db;
-                    if (sda != 0.f || sdb != 0.f) {
+                    if ((sda != 0.f || sdb != 0.f) && !(P.dbg & 16)) {  // (dbg 16: timing ablation)
                         const float2 na = make_float2(-sda, -sda), ndb = make_float2(-sdb, -sdb);
                         auto put2 = [&](float* p, float2 v0, float2 v1) {
                             p[0] = v0.x;
@@ -946,7 +955,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
                     }
                     __syncwarp();
                     const long long tr0 = P.tprof ? clock64() : 0;
-                    if (idx + 2 < nact)
+                    if (idx + 2 < nact && !(P.dbg & 32))  // (dbg 32: timing ablation)
                         prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
                                    pri + (pn + 1) % kPairBufs);
                     if (P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
