@@ -211,6 +211,41 @@ __device__ __forceinline__ void load_records(const unsigned char* stg, int off_i
     if (VPT == 2) ob = ((const uint16_t*)(stg + off_in_stage))[tp];
 }
 
+// this thread's VPT adjacent records (apos) from a stage as raw words (CW = 1: a uint8 code word
+// per view; CW = 4: fp32 values), and the band offsets packed in one word (VPT bytes)
+template <int VPT, int CW>
+__device__ __forceinline__ void load_words(const unsigned char* stg, int off_in_stage, int tp,
+                                           uint32_t (&c)[VPT][CW], uint32_t& ob)
+{
+    if (CW == 1 && VPT == 4) {
+        const uint4 c4 = ((const uint4*)stg)[tp];
+        c[0][0] = c4.x;
+        c[VPT > 1 ? 1 : 0][0] = c4.y;
+        c[VPT > 2 ? 2 : 0][0] = c4.z;
+        c[VPT > 3 ? 3 : 0][0] = c4.w;
+    } else if (CW == 1 && VPT == 2) {
+        const uint2 c2 = ((const uint2*)stg)[tp];
+        c[0][0] = c2.x;
+        c[VPT > 1 ? 1 : 0][0] = c2.y;
+    } else {
+#pragma unroll
+        for (int t = 0; t < VPT; ++t) {
+            if (CW == 4) {
+                const uint4 v = ((const uint4*)stg)[tp * VPT + t];
+                c[t][0] = v.x;
+                c[t][CW > 1 ? 1 : 0] = v.y;
+                c[t][CW > 2 ? 2 : 0] = v.z;
+                c[t][CW > 3 ? 3 : 0] = v.w;
+            } else {
+                c[t][0] = ((const uint32_t*)stg)[tp * VPT + t];
+            }
+        }
+    }
+    if (VPT == 4) ob = ((const uint32_t*)(stg + off_in_stage))[tp];
+    if (VPT == 2) ob = ((const uint16_t*)(stg + off_in_stage))[tp];
+    if (VPT == 1) ob = stg[off_in_stage + tp];
+}
+
 // prior warp: PriPair for voxels (i0, i0+1) of the visiting order from the current x tile.
 // Alg1:7's q-GGMRF surrogate sums sb = sum_r b_r phi(v - x_r), sx = sum_r b_r phi(v - x_r) x_r
 // over the neighbourhood (free boundary: off-image neighbours contribute nothing), voxel a on
@@ -442,8 +477,8 @@ __device__ __forceinline__ void band_info(const IcdParams& P, int tk, uint32_t* 
 // write-back overlap the other's voxel loop.
 // CL = 1: one CTA per SM of <= 6 (VPT 1, 4) or 12 (VPT 2) view warps + the prior warp; CL = 2:
 // two CTAs of 3 view warps + the prior warp per SM (8 warps: the full register budget)
-template <int VPT, bool U8, int NNB, int R, int CL>
-__global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 1 ? 1 : 2) k_icd_sv(const IcdParams P)
+template <int VPT, bool U8, int NNB, int R, int CL, bool PROF>
+__global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ? 416 : 224), CL == 1 ? 1 : 2) k_icd_sv(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -490,7 +525,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
         ((float4*)(smem + L.sb_w))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
     }
     if (threadIdx.x == 0) {
-        for (int b = 0; b < kPairBufs; ++b) mbar_init(pairbar + b, nvw + 1);  // all view warps + prior
+        for (int b = 0; b < kPairBufs; ++b) mbar_init(pairbar + b, nvw);  // all view warps of the task
         mbar_init(taskbar, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -550,7 +585,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
         const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
 
         long long tp0 = 0, tp1 = 0, tp1b = 0, tp2 = 0, tp3 = 0, tpa = 0, tpb = 0, tpc = 0;
-        if (P.tprof && threadIdx.x == 0) tp0 = clock64();
+        if (PROF && P.tprof && threadIdx.x == 0) tp0 = clock64();
         // ---- 1. x tile (+1 halo ring, +-1 slice in 3-D) into shared memory
         for (int i = threadIdx.x; i < (NNB == 26 ? 3 : 1) * TW * TW; i += blockDim.x) {
             const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
@@ -676,7 +711,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
             }
         }
 
-        if (P.tprof && threadIdx.x == 0) tp1 = clock64();
+        if (PROF && P.tprof && threadIdx.x == 0) tp1 = clock64();
         // ---- 4. view threads: SVB pack (coalesced 128-byte band rows, transposed by shuffles);
         //         e_init rows go to this CTA's L2-resident scratch tile for the write-back
         float* scr = P.scratch + (size_t)blockIdx.x * (size_t)P.Vs * 32;
@@ -735,7 +770,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
                 float* d = (isw ? sb_w : sb_e) + kk - sk * VS;  // + p * VS = band column p - sk of view kk
                 const float* sr = stg_w + lane * 33;
                 put(v4);
-                if (P.tprof && threadIdx.x == 0 && t == 0 && isw) tpb = clock64();
+                if (PROF && P.tprof && threadIdx.x == 0 && t == 0 && isw) tpb = clock64();
 #pragma unroll
                 for (int p = 0; p < 32; ++p)
                     if (bmask & (1u << p)) d[p * VS] = sr[p];
@@ -746,16 +781,16 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
                 float4 wa[8], ea[8];
                 issue(t, true, wa);
                 issue(t, false, ea);
-                if (P.tprof && threadIdx.x == 0 && t == 0) tpa = clock64();
+                if (PROF && P.tprof && threadIdx.x == 0 && t == 0) tpa = clock64();
                 finish(t, true, wa);
                 finish(t, false, ea);
-                if (P.tprof && threadIdx.x == 0 && t == 0) tpc = clock64();
+                if (PROF && P.tprof && threadIdx.x == 0 && t == 0) tpc = clock64();
             }
-            if (P.tprof && threadIdx.x == 0) tp1b = clock64();
+            if (PROF && P.tprof && threadIdx.x == 0) tp1b = clock64();
         }
         __syncthreads();
 
-        if (P.tprof && threadIdx.x == 0) tp2 = clock64();
+        if (PROF && P.tprof && threadIdx.x == 0) tp2 = clock64();
         // ---- 5. sequential-exact voxel loop, TWO voxels (a, b) per barrier.  Both are gathered
         //         from the same state of e, together with the overlap H = sum w A_b A_a over their
         //         shared sinogram entries; after the barrier every warp computes delta_a, then
@@ -764,125 +799,201 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
         //         neighbour, then delta_b -- exactly sequential ICD in the visiting order.
         float amount = 0.f;
         const int cslot = (zc * TW + 1) * TW + 1;  // tile index of local (0,0)
-        const int npair_threads = (nvl + 1) * 32;  // view warps + prior warp meet per pair
-        {
-            // the A records of the first R voxels (every stage is free: the previous visit ended
-            // with a CTA-wide barrier)
-            if (is_view)
-                for (int i = 0; i < R; ++i) copy_record(i, vw * 32 + lane);
-            for (int idx = 0; idx < nact; idx += 2) {
+        // Two named barriers per pair: A (1) -- the view warps' partial sums of the pair are in
+        // `red` (view warps arrive, the prior warp waits); B (2) -- the prior warp has published the
+        // pair's two deltas (prior warp arrives, view warps wait).  Only the prior warp evaluates
+        // the delta chain; the view warps prepare the next pair's e-independent state (records, w,
+        // w*A, the overlap H) while it runs, then scatter, then gather the next pair's e.
+        const int npair_threads = (nvl + 1) * 32;  // view warps + prior warp
+        float* dslot = (float*)(smem + L.misc) + 4;  // [2 pairs][2]: scale_a*delta_a, scale_b*delta_b
+        if (is_view) {
+            const int tp = vw * 32 + lane;  // this thread's record position in a stage
+            // Per-pair state of a view thread, for its VPT views: band offsets of a and b (packed
+            // bytes), their A records (uint8 code words, or fp32 values as bits), w*A_a, w*A_b on
+            // their own channels (channel pairs (0,1), (2,3) for the paired-fp32 FFMA2/FMUL2 of
+            // sm_100), and the warp-reduced overlap H = sum w A_b A_a.  None of it depends on e.
+            constexpr int CW = U8 ? 1 : 4;  // record words per view
+            struct PairState {
+                uint32_t oa, ob;
+                uint32_t ca[VPT][CW], cb[VPT][CW];
+                float2 wa[VPT][2], wb[VPT][2];
+                float hh;
+            };
+            // A values of a record as channel pairs
+            auto avals = [&](const uint32_t (&c)[CW], float2 (&f)[2]) {
+                if (U8) {
+                    f[0] = dq2(c[0], 0);
+                    f[1] = dq2(c[0], 2);
+                } else {
+                    f[0] = make_float2(__uint_as_float(c[0]), __uint_as_float(c[CW > 1 ? 1 : 0]));
+                    f[1] = make_float2(__uint_as_float(c[CW > 2 ? 2 : 0]), __uint_as_float(c[CW > 3 ? 3 : 0]));
+                }
+            };
+            auto off_of = [&](uint32_t packed, int t) { return (int)((packed >> (8 * t)) & 255u); };
+            // voxels j, j + 1 of the visiting order -> ps.  A pair without a second voxel (the
+            // last step of an odd visit, hb = false) gets a dummy b with zero A on a's channels:
+            // its theta1 and H vanish, its delta is 0, and its scatter rewrites a's entries with
+            // the same values -- no branches on the pair's shape.
+            auto prep = [&](int j, bool hb, PairState& ps) {
+                const long long tf0 = (PROF && P.tprof) ? clock64() : 0;
+                // this thread's copies of voxels j, j + 1 have landed (R voxels' groups are in
+                // flight: j .. j + R - 1)
+                cp_async_wait<R - 2>();
+                if (VPT != 4) __syncwarp();  // offset words copied by another lane of the warp
+                if (PROF && P.tprof && lane == 0)   // development aid: A-stream wait
+                    atomicAdd(P.tprof + 22 + (j >= R), (unsigned long long)(clock64() - tf0));
+                const unsigned char* sta = astage + ((gseq + (uint32_t)j) % R) * L.stage_bytes;
+                const unsigned char* stb = astage + ((gseq + (uint32_t)j + 1) % R) * L.stage_bytes;
+                load_words<VPT, CW>(sta, L.off_in_stage, tp, ps.ca, ps.oa);
+                load_words<VPT, CW>(stb, L.off_in_stage, tp, ps.cb, ps.ob);
+                ps.ob = hb ? ps.ob : ps.oa;
+#pragma unroll
+                for (int t = 0; t < VPT; ++t)
+#pragma unroll
+                    for (int c = 0; c < CW; ++c) ps.cb[t][c] = hb ? ps.cb[t][c] : 0u;
+                float2 h2[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+#pragma unroll
+                for (int t = 0; t < VPT; ++t) {
+                    // padded views (k >= V) have zero A: no per-view branch
+                    float2 fa[2], fb[2], fab[2];
+                    avals(ps.ca[t], fa);
+                    avals(ps.cb[t], fb);
+                    const int oa = off_of(ps.oa, t), ob = off_of(ps.ob, t);
+                    shifted<U8>(ps.ca[t][0], fa, ob - oa, fab);  // A_a on b's channels
+                    const float* pw = sb_w + oa * VS + kv[t];
+                    const float* qw = sb_w + ob * VS + kv[t];
+                    ps.wa[t][0] = __fmul2_rn(make_float2(pw[0], pw[VS]), fa[0]);
+                    ps.wa[t][1] = __fmul2_rn(make_float2(pw[2 * VS], pw[3 * VS]), fa[1]);
+                    ps.wb[t][0] = __fmul2_rn(make_float2(qw[0], qw[VS]), fb[0]);
+                    ps.wb[t][1] = __fmul2_rn(make_float2(qw[2 * VS], qw[3 * VS]), fb[1]);
+                    h2[t & 1] = __ffma2_rn(ps.wb[t][0], fab[0], h2[t & 1]);
+                    h2[t & 1] = __ffma2_rn(ps.wb[t][1], fab[1], h2[t & 1]);
+                }
+                const float2 hs = __fadd2_rn(h2[0], h2[1]);
+                float hh = hs.x + hs.y;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) hh += __shfl_xor_sync(kFull, hh, o);
+                ps.hh = hh;
+            };
+            // one voxel pair: theta1 partials from e -> barrier A -> the next pair's state ->
+            // barrier B (deltas) -> scatter -> refill the next pair's stages
+            auto pair_step = [&](int idx, PairState& cur, PairState& nxt) {
                 const uint32_t pn = pseq + (uint32_t)(idx >> 1);  // running pair number
                 const int buf = (int)(pn % kPairBufs);
-                const bool hasb = idx + 1 < nact;
-                const uint32_t g = gseq + idx;
-                const unsigned char* sta = astage + (g % R) * L.stage_bytes;
-                const unsigned char* stb = astage + ((g + 1) % R) * L.stage_bytes;
-                // per view t of this thread: e on a's / b's 4 channels, A_a, A_b on their own
-                // channels and A_a on b's channels, as channel pairs (0,1), (2,3) for the
-                // paired-fp32 FFMA2/FMUL2 of sm_100 (one instruction per two channels)
-                float2 ea[VPT][2], eb[VPT][2], fa[VPT][2], fb[VPT][2], fab[VPT][2];
-                int oa[VPT], ob[VPT];
-                if (is_view) {
-                    const int tp = vw * 32 + lane;
-                    // HB: the pair has a second voxel (all but the last step of an odd visit)
-                    auto gather = [&](auto hb) {
-                        constexpr bool HB = decltype(hb)::value;
-                        const long long tf0 = P.tprof ? clock64() : 0;
-                        // this thread's copies of voxels idx, idx + 1 have landed (R voxels'
-                        // groups are in flight: idx .. idx + R - 1)
-                        cp_async_wait<R - 2>();
-                        if (VPT != 4) __syncwarp();  // offset words copied by the lane quad's first lane
-                        if (P.tprof && lane == 0)  // development aid: A-stream wait
-                            atomicAdd(P.tprof + 22 + (idx >= R), (unsigned long long)(clock64() - tf0));
-                        uint32_t ca[VPT], cb[VPT], oba = 0, obb = 0;
-                        load_records<VPT, U8>(sta, L.off_in_stage, tp, ca, fa, oba);
-                        if (HB) load_records<VPT, U8>(stb, L.off_in_stage, tp, cb, fb, obb);
-                        // two accumulator sets (even / odd views) halve the FFMA2 dependency chains
-                        float2 acc[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-                        float2 accb[2] = {acc[0], acc[0]}, acch[2] = {acc[0], acc[0]};
-#pragma unroll
-                        for (int t = 0; t < VPT; ++t) {
-                            // padded views (k >= V) have zero A: no per-view branch
-                            oa[t] = VPT == 4 ? (int)((oba >> (8 * t)) & 255u) : (int)sta[L.off_in_stage + tp * VPT + t];
-                            const float* pe = sb_e + oa[t] * VS + kv[t];
-                            const float* pw = sb_w + oa[t] * VS + kv[t];
-                            ea[t][0] = make_float2(pe[0], pe[VS]);
-                            ea[t][1] = make_float2(pe[2 * VS], pe[3 * VS]);
-                            const float2 w0 = make_float2(pw[0], pw[VS]), w1 = make_float2(pw[2 * VS], pw[3 * VS]);
-                            acc[t & 1] = __ffma2_rn(__fmul2_rn(w0, ea[t][0]), fa[t][0], acc[t & 1]);
-                            acc[t & 1] = __ffma2_rn(__fmul2_rn(w1, ea[t][1]), fa[t][1], acc[t & 1]);
-                            if (HB) {
-                                ob[t] = VPT == 4 ? (int)((obb >> (8 * t)) & 255u) : (int)stb[L.off_in_stage + tp * VPT + t];
-                                shifted<U8>(ca[t], fa[t], ob[t] - oa[t], fab[t]);  // A_a on b's channels
-                                const float* qe = sb_e + ob[t] * VS + kv[t];
-                                const float* qw = sb_w + ob[t] * VS + kv[t];
-                                eb[t][0] = make_float2(qe[0], qe[VS]);
-                                eb[t][1] = make_float2(qe[2 * VS], qe[3 * VS]);
-                                const float2 wb0 = __fmul2_rn(make_float2(qw[0], qw[VS]), fb[t][0]);
-                                const float2 wb1 = __fmul2_rn(make_float2(qw[2 * VS], qw[3 * VS]), fb[t][1]);
-                                accb[t & 1] = __ffma2_rn(wb0, eb[t][0], accb[t & 1]);
-                                accb[t & 1] = __ffma2_rn(wb1, eb[t][1], accb[t & 1]);
-                                acch[t & 1] = __ffma2_rn(wb0, fab[t][0], acch[t & 1]);
-                                acch[t & 1] = __ffma2_rn(wb1, fab[t][1], acch[t & 1]);
-                            }
-                        }
-                        const float2 ac = __fadd2_rn(acc[0], acc[1]), acb = __fadd2_rn(accb[0], accb[1]);
-                        const float2 ach = __fadd2_rn(acch[0], acch[1]);
-                        float2 gab = make_float2(ac.x + ac.y, acb.x + acb.y);
-                        float hh = ach.x + ach.y;
-#pragma unroll
-                        for (int o = 16; o > 0; o >>= 1) {
-                            const float2 r = make_float2(__shfl_xor_sync(kFull, gab.x, o), __shfl_xor_sync(kFull, gab.y, o));
-                            gab = __fadd2_rn(gab, r);
-                            if (HB) hh += __shfl_xor_sync(kFull, hh, o);
-                        }
-                        // the pair's stages are consumed (every lane's values are in registers and
-                        // reduced): refill them with the records R voxels ahead
-                        copy_record(idx + R, tp);
-                        copy_record(idx + 1 + R, tp);
-                        if (lane == 0) {
-                            float* rs = red + buf * 3 * NSL + gvw;
-                            rs[0] = gab.x;
-                            rs[NSL] = gab.y;
-                            rs[2 * NSL] = hh;
-                            if (CL == 2) {
-                                // the same slots of the peer CTA, then arrive on both CTAs'
-                                // pair barriers (the release orders the stores)
-                                const uint32_t pa = peer_addr(rs, crank ^ 1u);
-                                st_peer_f32(pa, gab.x);
-                                st_peer_f32(pa + 4 * NSL, gab.y);
-                                st_peer_f32(pa + 8 * NSL, hh);
-                                mbar_arrive_peer(peer_addr(pairbar + buf, crank ^ 1u));
-                                mbar_arrive(pairbar + buf);
-                            }
-                        }
-                    };
-                    if (hasb)
-                        gather(BoolTag<true>{});
-                    else
-                        gather(BoolTag<false>{});
-                } else if (idx == 0) {
-                    // prior warp: the surrogate terms of a pair are published after the previous
-                    // pair's barrier; only the first pair's are computed here
-                    prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + buf);
-                }
+                // ---- the pair's theta1 partials: sum (w A_a) e and sum (w A_b) e over this
+                //      thread's views, from the state of e after the previous pair's scatter
+                float2 ea[VPT][2], eb[VPT][2];
                 {
-                    // the view warps and the prior warp meet (CL = 1: named barrier 1; CL = 2: the
-                    // pair mbarrier, which also collects the peer CTA's view warps)
-                    const long long tw0 = P.tprof ? clock64() : 0;
-                    if (CL == 1) {
-                        if (!(P.dbg & 64)) asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
-                    } else {
-                        if (is_prior) {
-                            __syncwarp();
-                            if (lane == 0) mbar_arrive(pairbar + buf);  // pri[buf] is published
-                        }
-                        mbar_wait_cluster(pairbar + buf, (pn / kPairBufs) & 1u);
+                    float2 acc[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+                    float2 accb[2] = {acc[0], acc[0]};
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t) {
+                        const float* pe = sb_e + off_of(cur.oa, t) * VS + kv[t];
+                        const float* qe = sb_e + off_of(cur.ob, t) * VS + kv[t];
+                        ea[t][0] = make_float2(pe[0], pe[VS]);
+                        ea[t][1] = make_float2(pe[2 * VS], pe[3 * VS]);
+                        eb[t][0] = make_float2(qe[0], qe[VS]);
+                        eb[t][1] = make_float2(qe[2 * VS], qe[3 * VS]);
+                        acc[t & 1] = __ffma2_rn(cur.wa[t][0], ea[t][0], acc[t & 1]);
+                        acc[t & 1] = __ffma2_rn(cur.wa[t][1], ea[t][1], acc[t & 1]);
+                        accb[t & 1] = __ffma2_rn(cur.wb[t][0], eb[t][0], accb[t & 1]);
+                        accb[t & 1] = __ffma2_rn(cur.wb[t][1], eb[t][1], accb[t & 1]);
                     }
-                    if (P.tprof && lane == 0)  // development aid: per-warp wait at the pair barrier
+                    const float2 ac = __fadd2_rn(acc[0], acc[1]), acb = __fadd2_rn(accb[0], accb[1]);
+                    float2 gab = make_float2(ac.x + ac.y, acb.x + acb.y);
+#pragma unroll
+                    for (int o = 16; o > 0; o >>= 1) {
+                        const float2 r = make_float2(__shfl_xor_sync(kFull, gab.x, o), __shfl_xor_sync(kFull, gab.y, o));
+                        gab = __fadd2_rn(gab, r);
+                    }
+                    if (lane == 0) {
+                        float* rs = red + buf * 3 * NSL + gvw;
+                        rs[0] = gab.x;
+                        rs[NSL] = gab.y;
+                        rs[2 * NSL] = cur.hh;
+                        if (CL == 2) {
+                            // the same slots of the peer CTA, then arrive on both CTAs' pair
+                            // barriers (the release orders the stores)
+                            const uint32_t pa = peer_addr(rs, crank ^ 1u);
+                            st_peer_f32(pa, gab.x);
+                            st_peer_f32(pa + 4 * NSL, gab.y);
+                            st_peer_f32(pa + 8 * NSL, cur.hh);
+                            mbar_arrive_peer(peer_addr(pairbar + buf, crank ^ 1u));
+                            mbar_arrive(pairbar + buf);
+                        }
+                    }
+                }
+                // barrier A: arrive (the prior warp derives the deltas)
+                if (CL == 1) asm volatile("bar.arrive 1, %0;" ::"r"(npair_threads) : "memory");
+                // ---- meanwhile: the next pair's e-independent state
+                if (idx + 2 < nact) prep(idx + 2, idx + 3 < nact, nxt);
+                // ---- barrier B: the deltas are published
+                {
+                    const long long tw0 = (PROF && P.tprof) ? clock64() : 0;
+                    asm volatile("bar.sync 2, %0;" ::"r"(npair_threads) : "memory");
+                    if (PROF && P.tprof && lane == 0)  // development aid: per-warp wait for the deltas
                         atomicAdd(P.tprof + 10 + warp, (unsigned long long)(clock64() - tw0));
                 }
-                // every warp derives the same two deltas (identical inputs, identical order)
+                // ---- Alg1:9-11 for both voxels on this thread's views: a's channels first with
+                //      a's update, then b's channels with both updates -- b's path rewrites the
+                //      entries the two voxels share with the full value, so A_b is never needed on
+                //      a's channels
+                const float sda = dslot[(pn & 1) * 2], sdb = dslot[(pn & 1) * 2 + 1];
+                if ((sda != 0.f || sdb != 0.f) && !(P.dbg & 16)) {  // (dbg 16: timing ablation)
+                    const float2 nda = make_float2(-sda, -sda), ndb = make_float2(-sdb, -sdb);
+                    auto put2 = [&](float* p, float2 v0, float2 v1) {
+                        p[0] = v0.x;
+                        p[VS] = v0.y;
+                        p[2 * VS] = v1.x;
+                        p[3 * VS] = v1.y;
+                    };
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t) {
+                        float2 fa[2], fb[2], fab[2];
+                        avals(cur.ca[t], fa);
+                        avals(cur.cb[t], fb);
+                        const int oa = off_of(cur.oa, t), ob = off_of(cur.ob, t);
+                        shifted<U8>(cur.ca[t][0], fa, ob - oa, fab);
+                        put2(sb_e + oa * VS + kv[t], __ffma2_rn(fa[0], nda, ea[t][0]), __ffma2_rn(fa[1], nda, ea[t][1]));
+                        put2(sb_e + ob * VS + kv[t], __ffma2_rn(fb[0], ndb, __ffma2_rn(fab[0], nda, eb[t][0])),
+                             __ffma2_rn(fb[1], ndb, __ffma2_rn(fab[1], nda, eb[t][1])));
+                    }
+                }
+                // the next pair's stages are consumed (its state is in registers): refill them
+                // with the records R voxels ahead
+                copy_record(idx + 2 + R, tp);
+                copy_record(idx + 3 + R, tp);
+            };
+            // the A records of the first R voxels (every stage is free: the previous visit ended
+            // with a CTA-wide barrier), then the first pair's state; its stages are refilled.
+            // The pair loop is unrolled by two so the two states swap roles without copies.
+            PairState st0, st1;
+            for (int i = 0; i < R; ++i) copy_record(i, tp);
+            prep(0, 1 < nact, st0);
+            copy_record(R, tp);
+            copy_record(R + 1, tp);
+            for (int idx = 0; idx < nact; idx += 4) {
+                pair_step(idx, st0, st1);
+                if (idx + 2 < nact) pair_step(idx + 2, st1, st0);
+            }
+        } else {
+            // ---- prior warp: the surrogate terms of the first pair, then per pair: wait for the
+            //      view warps' partial sums (A), derive both deltas (every lane, identical
+            //      inputs), publish them (B), store the new values, next pair's surrogate terms
+            prior_pair(tof, 0, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + (pseq % kPairBufs));
+            for (int idx = 0; idx < nact; idx += 2) {
+                const uint32_t pn = pseq + (uint32_t)(idx >> 1);
+                const int buf = (int)(pn % kPairBufs);
+                const bool hasb = idx + 1 < nact;
+                {
+                    const long long tw0 = (PROF && P.tprof) ? clock64() : 0;
+                    if (CL == 1)
+                        asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
+                    else
+                        mbar_wait_cluster(pairbar + buf, (pn / kPairBufs) & 1u);
+                    if (PROF && P.tprof && lane == 0)  // development aid: wait for the partial sums
+                        atomicAdd(P.tprof + 10 + warp, (unsigned long long)(clock64() - tw0));
+                }
                 const float* rb = red + buf * 3 * NSL;  // nvw <= NSL partials per quantity, rest 0
                 const float sa = sum_slots<NSL>(rb), sbs = sum_slots<NSL>(rb + NSL), sh = sum_slots<NSL>(rb + 2 * NSL);
                 const PriPair pp = pri[buf];
@@ -915,57 +1026,35 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
                     if (c_prior.positivity) ub = fmaxf(ub, 0.f);
                     db = ub - pp.vb;
                 }
-                if (is_view) {
-                    // Alg1:9-11 for both voxels on this thread's views: a's channels first with
-                    // a's update, then b's channels with both updates -- b's path rewrites the
-                    // entries the two voxels share with the full value, so A_b is never needed on
-                    // a's channels
-                    const float sda = scale_a * da, sdb = scale_b * db;
-                    if ((sda != 0.f || sdb != 0.f) && !(P.dbg & 16)) {  // (dbg 16: timing ablation)
-                        const float2 na = make_float2(-sda, -sda), ndb = make_float2(-sdb, -sdb);
-                        auto put2 = [&](float* p, float2 v0, float2 v1) {
-                            p[0] = v0.x;
-                            p[VS] = v0.y;
-                            p[2 * VS] = v1.x;
-                            p[3 * VS] = v1.y;
-                        };
-#pragma unroll
-                        for (int t = 0; t < VPT; ++t) {
-                            put2(sb_e + oa[t] * VS + kv[t], __ffma2_rn(fa[t][0], na, ea[t][0]),
-                                 __ffma2_rn(fa[t][1], na, ea[t][1]));
-                            if (hasb)
-                                put2(sb_e + ob[t] * VS + kv[t],
-                                     __ffma2_rn(fb[t][0], ndb, __ffma2_rn(fab[t][0], na, eb[t][0])),
-                                     __ffma2_rn(fb[t][1], ndb, __ffma2_rn(fab[t][1], na, eb[t][1])));
-                        }
-                    }
-                } else {
-                    // prior warp: store the pair's new values, then the next pair's surrogate
-                    // terms (published for the view warps before the next barrier)
-                    if (lane == 0) {
-                        if (idx + 2 * R < nact) prefetch_record(idx + 2 * R);
-                        if (idx + 1 + 2 * R < nact) prefetch_record(idx + 1 + 2 * R);
-                        const int ta = tof[idx];
-                        xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
-                        if (hasb) {
-                            const int tbv = tof[idx + 1];
-                            xt[cslot + (tbv >> 8) * TW + (tbv & 255)] = ub;
-                        }
-                        amount += fabsf(da) + fabsf(db);
-                    }
-                    __syncwarp();
-                    const long long tr0 = P.tprof ? clock64() : 0;
-                    if (idx + 2 < nact && !(P.dbg & 32))  // (dbg 32: timing ablation)
-                        prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
-                                   pri + (pn + 1) % kPairBufs);
-                    if (P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
+                if (lane == 0) {
+                    dslot[(pn & 1) * 2] = scale_a * da;
+                    dslot[(pn & 1) * 2 + 1] = scale_b * db;
                 }
+                asm volatile("bar.arrive 2, %0;" ::"r"(npair_threads) : "memory");  // barrier B
+                // the pair's new values, then the next pair's surrogate terms
+                if (lane == 0) {
+                    if (idx + 2 * R < nact) prefetch_record(idx + 2 * R);
+                    if (idx + 1 + 2 * R < nact) prefetch_record(idx + 1 + 2 * R);
+                    const int ta = tof[idx];
+                    xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
+                    if (hasb) {
+                        const int tbv = tof[idx + 1];
+                        xt[cslot + (tbv >> 8) * TW + (tbv & 255)] = ub;
+                    }
+                    amount += fabsf(da) + fabsf(db);
+                }
+                __syncwarp();
+                const long long tr0 = (PROF && P.tprof) ? clock64() : 0;
+                if (idx + 2 < nact && !(P.dbg & 32))  // (dbg 32: timing ablation)
+                    prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
+                               pri + (pn + 1) % kPairBufs);
+                if (PROF && P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
             }
         }
         gseq += nact;
         pseq += (uint32_t)(nact + 1) >> 1;
         ++ntask;
-        if (P.tprof && threadIdx.x == 0) tp3 = clock64();
+        if (PROF && P.tprof && threadIdx.x == 0) tp3 = clock64();
         __syncthreads();
 
         // ---- 6. write-back: delta e of the band, atomically, and the SV's voxels
@@ -1063,7 +1152,7 @@ __global__ void __launch_bounds__(CL == 2 ? 128 : (VPT == 2 ? 416 : 224), CL == 
             }
         }
         if (CL == 2) cluster_sync_all(); else __syncthreads();
-        if (P.tprof && threadIdx.x == 0 && crank == 0) {
+        if (PROF && P.tprof && threadIdx.x == 0 && crank == 0) {
             const long long tp4 = clock64();
             atomicAdd(P.tprof + 0, (unsigned long long)(tp1 - tp0));  // x tile, zero-skip, order
             atomicAdd(P.tprof + 1, (unsigned long long)(tp2 - tp1));  // SVB pack (+ first A stage)
@@ -1256,7 +1345,10 @@ template <int VPT, bool U8, int NNB, int CL>
 static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t st)
 {
     constexpr int R = ring_depth(U8, CL);
-    auto kern = k_icd_sv<VPT, U8, NNB, R, CL>;
+    // the phase-profiling instrumentation (env MBIR_PHASE_PROFILE) is compiled only into the
+    // bench's configuration; every other launch runs the instrumentation-free kernel
+    constexpr bool kProfiled = VPT == 4 && U8 && CL == 1;
+    auto kern = (kProfiled && p.tprof) ? k_icd_sv<VPT, U8, NNB, R, CL, kProfiled> : k_icd_sv<VPT, U8, NNB, R, CL, false>;
     IcdParams q = p;
     q.lay = smem_layout(p.rows, svb_stride(VPT, CL), p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, CL);
     const int smem = q.lay.total;
@@ -1289,7 +1381,7 @@ template <int VPT, bool U8, int NNB, int CL>
 static int resident_ctas_t(const IcdParams& p)
 {
     constexpr int R = ring_depth(U8, CL);
-    auto kern = k_icd_sv<VPT, U8, NNB, R, CL>;
+    auto kern = k_icd_sv<VPT, U8, NNB, R, CL, false>;
     const int smem = smem_layout(p.rows, svb_stride(VPT, CL), p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, CL).total;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
     cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
@@ -1332,6 +1424,7 @@ int icd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int c
         if (quantize) return nnb == 26 ? resident_ctas_t<1, true, 26, 1>(p) : resident_ctas_t<1, true, 8, 1>(p);
         return nnb == 26 ? resident_ctas_t<1, false, 26, 1>(p) : resident_ctas_t<1, false, 8, 1>(p);
     }
+    if (quantize && cl == 2 && vpt == 2) return nnb == 26 ? resident_ctas_t<2, true, 26, 2>(p) : resident_ctas_t<2, true, 8, 2>(p);
     if (quantize && cl == 2) return nnb == 26 ? resident_ctas_t<4, true, 26, 2>(p) : resident_ctas_t<4, true, 8, 2>(p);
     if (quantize) return nnb == 26 ? resident_ctas_t<4, true, 26, 1>(p) : resident_ctas_t<4, true, 8, 1>(p);
     return nnb == 26 ? resident_ctas_t<4, false, 26, 1>(p) : resident_ctas_t<4, false, 8, 1>(p);
@@ -1344,6 +1437,8 @@ cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int 
         if (quantize) return nnb == 26 ? launch_icd_t<1, true, 26, 1>(p, gx, gy, st) : launch_icd_t<1, true, 8, 1>(p, gx, gy, st);
         return nnb == 26 ? launch_icd_t<1, false, 26, 1>(p, gx, gy, st) : launch_icd_t<1, false, 8, 1>(p, gx, gy, st);
     }
+    if (quantize && cl == 2 && vpt == 2)
+        return nnb == 26 ? launch_icd_t<2, true, 26, 2>(p, gx, gy, st) : launch_icd_t<2, true, 8, 2>(p, gx, gy, st);
     if (quantize && cl == 2)
         return nnb == 26 ? launch_icd_t<4, true, 26, 2>(p, gx, gy, st) : launch_icd_t<4, true, 8, 2>(p, gx, gy, st);
     if (quantize) return nnb == 26 ? launch_icd_t<4, true, 26, 1>(p, gx, gy, st) : launch_icd_t<4, true, 8, 1>(p, gx, gy, st);
