@@ -646,9 +646,10 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
 
     // ---- state buffers
     const size_t ns = sino_elems(h), pl = plane_elems(h);
-    if ((r = dalloc(h, &h->d_y, ns))) return bail(r);
-    if ((r = dalloc(h, &h->d_w, ns))) return bail(r);
-    if ((r = dalloc(h, &h->d_e, ns))) return bail(r);
+    // (+32 floats: the update kernel reads whole 32-float windows around band rows)
+    if ((r = dalloc(h, &h->d_y, ns + 32))) return bail(r);
+    if ((r = dalloc(h, &h->d_w, ns + 32))) return bail(r);
+    if ((r = dalloc(h, &h->d_e, ns + 32))) return bail(r);
     if ((r = dalloc(h, &h->d_x, pl * (G.nz_local + 2)))) return bail(r);
     if ((r = dalloc(h, &h->d_theta2, (size_t)G.nz_local * h->nsv * h->S2))) return bail(r);
     if ((r = dalloc(h, &h->d_amount, (size_t)G.nz_local * h->nsv))) return bail(r);

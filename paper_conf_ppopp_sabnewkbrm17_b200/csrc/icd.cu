@@ -447,10 +447,13 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     L.misc = o;  o = align16(o + 16 * 4);
     L.off_in_stage = VL * (u8 ? 4 : 16);
     L.stage_bytes = align16(L.off_in_stage + VL);
-    L.astage = o; o = align16(o + nstage * L.stage_bytes);
+    // the A-record ring (voxel loop) and the transpose staging tiles (pack, write-back) are never
+    // live at the same time: they share one region
+    L.astage = o;
+    L.staging = o;
+    o = align16(o + max(nstage * L.stage_bytes, nvl * 32 * 33 * 4));  // staging: a 32x33 tile per view warp
     // pair[kPairBufs], task[1]
     L.mbar = o;  o = align16(o + (kPairBufs + 1) * 8);
-    L.staging = o; o = align16(o + nvl * 32 * 33 * 4);  // one 32x33 transpose tile per view warp
     L.binfo = o; o = align16(o + 2 * VL * 4);           // band (row offset << 5 | width), 2 tasks
     L.total = o;
     return L;
@@ -587,13 +590,30 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
         long long tp0 = 0, tp1 = 0, tp1b = 0, tp2 = 0, tp3 = 0, tpa = 0, tpb = 0, tpc = 0;
         if (PROF && P.tprof && threadIdx.x == 0) tp0 = clock64();
         // ---- 1. x tile (+1 halo ring, +-1 slice in 3-D) into shared memory
-        for (int i = threadIdx.x; i < (NNB == 26 ? 3 : 1) * TW * TW; i += blockDim.x) {
-            const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
-            const int gx = gx0 - 1 + tx, gy = gy0 - 1 + ty;
-            const int zs = (NNB == 26) ? z + tz : z + 1;  // storage slice (halo at 0, nz+1)
-            float v = 0.f;
-            if (gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny) v = P.x[zs * plane + (size_t)gy * P.nx + gx];
-            xt[i] = v;
+        {
+            // all of a thread's loads first (clamped, always in bounds), then the zeroing of
+            // off-image entries and the stores: the loads are in flight together
+            constexpr int XMAX = 4;  // tile entries per thread and round
+            const int ntile = (NNB == 26 ? 3 : 1) * TW * TW;
+            for (int i0 = 0; i0 < ntile; i0 += XMAX * blockDim.x) {
+            float xv[XMAX];
+            bool inb[XMAX];
+#pragma unroll
+            for (int u = 0; u < XMAX; ++u) {
+                const int i = i0 + threadIdx.x + u * blockDim.x;
+                const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
+                const int gx = gx0 - 1 + tx, gy = gy0 - 1 + ty;
+                const int zs = (NNB == 26) ? z + tz : z + 1;  // storage slice (halo at 0, nz+1)
+                inb[u] = i < ntile && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny;
+                const int cx = min(max(gx, 0), P.nx - 1), cy = min(max(gy, 0), P.ny - 1);
+                xv[u] = i < ntile ? P.x[(size_t)min(zs, P.nz_local + 1) * plane + (size_t)cy * P.nx + cx] : 0.f;
+            }
+#pragma unroll
+            for (int u = 0; u < XMAX; ++u) {
+                const int i = i0 + threadIdx.x + u * blockDim.x;
+                if (i < ntile) xt[i] = inb[u] ? xv[u] : 0.f;
+            }
+            }
         }
         __syncthreads();
 
@@ -737,14 +757,17 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
 #pragma unroll
                 for (int m = 0; m < 8; ++m) {
                     const int i = 4 * m + sub;
-                    const int oi = __shfl_sync(kFull, rot, i), wi = __shfl_sync(kFull, bwt, i);
+                    const int oi = __shfl_sync(kFull, rot, i);
+                    // unconditional loads (no consumer until the staging, so all 8 are in flight):
+                    // the whole aligned window is read even past the band (padded views read the
+                    // slice start); only band positions are ever stored, and the sinogram
+                    // allocations carry 32 floats of tail padding for the last row's window
                     const int s = oi & 3;
-                    const bool ok = vbase + k0 + i < V && 4 * ch < s + wi;
                     const size_t a4 = (size_t)(oi - s) + 4 * ch;
                     if (isw)
-                        v4[m] = ok ? __ldg((const float4*)(wz + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                        v4[m] = __ldg((const float4*)(wz + a4));
                     else
-                        v4[m] = ok ? __ldcg((const float4*)(ez + a4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                        v4[m] = __ldcg((const float4*)(ez + a4));
                 }
             };
             auto put = [&](const float4 (&v)[8]) {
@@ -1330,10 +1353,10 @@ __global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
 
 }  // namespace
 
-// A-record ring depth (voxels of TMA lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
+// A-record ring depth (voxels of cp.async lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
 // (the pair loop needs >= 4: the current pair's two stages plus the next pair's two).  The
-// cluster variant holds half a record per stage but must fit two CTAs per SM: 6 stages.
-constexpr int ring_depth(bool u8, int cl) { return u8 ? (cl == 2 ? 6 : 8) : 4; }
+// cluster variant holds half a record per stage but must fit two CTAs per SM.
+constexpr int ring_depth(bool u8, int cl) { return u8 ? (cl == 2 ? 8 : 12) : 4; }
 
 int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl)
 {
