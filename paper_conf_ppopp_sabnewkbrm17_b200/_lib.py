@@ -88,10 +88,12 @@ _lib = None
 
 
 def load(path: str = LIB_PATH):
-    """Load libmbir.so (raises if it is missing -- no fallback)."""
+    """Load libmbir.so (raises if it is missing -- no fallback).  MBIR_LIB may name another
+    in-tree build of the same library (A/B kernel experiments)."""
     global _lib
     if _lib is not None:
         return _lib
+    path = os.environ.get("MBIR_LIB", path)
     if not os.path.exists(path):
         raise ImportError(f"{path} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
     L = C.CDLL(path)
