@@ -892,11 +892,9 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     h2[t & 1] = __ffma2_rn(ps.wb[t][0], fab[0], h2[t & 1]);
                     h2[t & 1] = __ffma2_rn(ps.wb[t][1], fab[1], h2[t & 1]);
                 }
+                // this lane's part of H; the warp reduction is done with the pair's theta1 sums
                 const float2 hs = __fadd2_rn(h2[0], h2[1]);
-                float hh = hs.x + hs.y;
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) hh += __shfl_xor_sync(kFull, hh, o);
-                ps.hh = hh;
+                ps.hh = hs.x + hs.y;
             };
             // one voxel pair: theta1 partials from e -> barrier A -> the next pair's state ->
             // barrier B (deltas) -> scatter -> refill the next pair's stages
@@ -924,23 +922,25 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     }
                     const float2 ac = __fadd2_rn(acc[0], acc[1]), acb = __fadd2_rn(accb[0], accb[1]);
                     float2 gab = make_float2(ac.x + ac.y, acb.x + acb.y);
+                    float hh = cur.hh;
 #pragma unroll
                     for (int o = 16; o > 0; o >>= 1) {
                         const float2 r = make_float2(__shfl_xor_sync(kFull, gab.x, o), __shfl_xor_sync(kFull, gab.y, o));
+                        hh += __shfl_xor_sync(kFull, hh, o);
                         gab = __fadd2_rn(gab, r);
                     }
                     if (lane == 0) {
                         float* rs = red + buf * 3 * NSL + gvw;
                         rs[0] = gab.x;
                         rs[NSL] = gab.y;
-                        rs[2 * NSL] = cur.hh;
+                        rs[2 * NSL] = hh;
                         if (CL == 2) {
                             // the same slots of the peer CTA, then arrive on both CTAs' pair
                             // barriers (the release orders the stores)
                             const uint32_t pa = peer_addr(rs, crank ^ 1u);
                             st_peer_f32(pa, gab.x);
                             st_peer_f32(pa + 4 * NSL, gab.y);
-                            st_peer_f32(pa + 8 * NSL, cur.hh);
+                            st_peer_f32(pa + 8 * NSL, hh);
                             mbar_arrive_peer(peer_addr(pairbar + buf, crank ^ 1u));
                             mbar_arrive(pairbar + buf);
                         }
