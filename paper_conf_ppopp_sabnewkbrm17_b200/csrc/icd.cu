@@ -412,6 +412,12 @@ __device__ __forceinline__ void cluster_sync_all()
 
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
 
+// row stride (floats) of a view warp's 32-row transpose staging tile: 16-byte rows, so a lane moves
+// 4 window positions with one STS.128 / LDS.128; every quarter-warp (one shared-memory wavefront
+// of a 128-bit access) then touches 8 distinct 4-bank groups, on the put (lanes span rows and
+// float4 chunks) and on the read (lane k reads its own row)
+constexpr int kStg = 36;
+
 // the update kernel's SVB column stride: the most views one CTA can hold (VPT = 1: 6 view warps
 // of 32; VPT >= 2: 768 views = 24 / VPT view warps, / CL), fixed at compile time whatever the
 // actual view count
@@ -451,7 +457,7 @@ __host__ __device__ inline SmemLayout smem_layout(int rows, int Vs, int side, in
     // live at the same time: they share one region
     L.astage = o;
     L.staging = o;
-    o = align16(o + max(nstage * L.stage_bytes, nvl * 32 * 33 * 4));  // staging: a 32x33 tile per view warp
+    o = align16(o + max(nstage * L.stage_bytes, nvl * 32 * kStg * 4));  // staging: a 32 x kStg tile per view warp
     // pair[kPairBufs], task[1]
     L.mbar = o;  o = align16(o + (kPairBufs + 1) * 8);
     L.binfo = o; o = align16(o + 2 * VL * 4);           // band (row offset << 5 | width), 2 tasks
@@ -514,7 +520,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
     float* vth2 = (float*)(smem + L.vth2);
     uint64_t* mbar = (uint64_t*)(smem + L.mbar);
     unsigned char* astage = smem + L.astage;
-    float* stg_w = (float*)(smem + L.staging) + vw * 32 * 33;
+    float* stg_w = (float*)(smem + L.staging) + vw * 32 * kStg;
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
     const size_t plane = (size_t)P.nx * P.ny;
@@ -587,7 +593,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
         const int gx0 = bx * side, gy0 = by * side;
         const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
 
-        long long tp0 = 0, tp1 = 0, tp1b = 0, tp2 = 0, tp3 = 0, tpa = 0, tpb = 0, tpc = 0;
+        long long tp0 = 0, tp1 = 0, tp1b = 0, tp2 = 0, tp3 = 0;
         if (PROF && P.tprof && threadIdx.x == 0) tp0 = clock64();
         // ---- 1. x tile (+1 halo ring, +-1 slice in 3-D) into shared memory
         {
@@ -770,16 +776,6 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                         v4[m] = __ldcg((const float4*)(ez + a4));
                 }
             };
-            auto put = [&](const float4 (&v)[8]) {
-#pragma unroll
-                for (int m = 0; m < 8; ++m) {
-                    const int i = 4 * m + sub;
-                    const float vv[4] = {v[m].x, v[m].y, v[m].z, v[m].w};
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) stg_w[i * 33 + 4 * ch + j] = vv[j];
-                }
-                __syncwarp();
-            };
             auto finish = [&](int t, bool isw, const float4 (&v4)[8]) {
                 const int k0 = (vw * VPT + t) * 32;
                 const int kk = k0 + lane;
@@ -791,23 +787,32 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), v4[m]);
                 }
                 float* d = (isw ? sb_w : sb_e) + kk - sk * VS;  // + p * VS = band column p - sk of view kk
-                const float* sr = stg_w + lane * 33;
-                put(v4);
-                if (PROF && P.tprof && threadIdx.x == 0 && t == 0 && isw) tpb = clock64();
 #pragma unroll
-                for (int p = 0; p < 32; ++p)
-                    if (bmask & (1u << p)) d[p * VS] = sr[p];
+                for (int m = 0; m < 8; ++m) *(float4*)(stg_w + (4 * m + sub) * kStg + 4 * ch) = v4[m];
+                __syncwarp();
+#pragma unroll
+                for (int q4 = 0; q4 < 8; ++q4) {
+                    const float4 r = *(const float4*)(stg_w + lane * kStg + 4 * q4);
+                    const float rv[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        if (bmask & (1u << (4 * q4 + j))) d[(4 * q4 + j) * VS] = rv[j];
+                }
                 __syncwarp();
             };
-#pragma unroll 1
+            // software pipeline over the VPT tiles: tile t + 1's 16 window loads are in flight
+            // while tile t is staged
+            float4 wa[2][8], ea[2][8];
+            issue(0, true, wa[0]);
+            issue(0, false, ea[0]);
+#pragma unroll
             for (int t = 0; t < VPT; ++t) {
-                float4 wa[8], ea[8];
-                issue(t, true, wa);
-                issue(t, false, ea);
-                if (PROF && P.tprof && threadIdx.x == 0 && t == 0) tpa = clock64();
-                finish(t, true, wa);
-                finish(t, false, ea);
-                if (PROF && P.tprof && threadIdx.x == 0 && t == 0) tpc = clock64();
+                if (t + 1 < VPT) {
+                    issue(t + 1, true, wa[(t + 1) & 1]);
+                    issue(t + 1, false, ea[(t + 1) & 1]);
+                }
+                finish(t, true, wa[t & 1]);
+                finish(t, false, ea[t & 1]);
             }
             if (PROF && P.tprof && threadIdx.x == 0) tp1b = clock64();
         }
@@ -1087,21 +1092,35 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
             // each aligned 32-float row window gets delta = final - e_init (band positions only)
             // with red.global.add.v4.f32
             const int sub = lane >> 3, ch = lane & 7;
-#pragma unroll 1
+            // e_init windows of tile t (L2-resident scratch), one tile ahead of the staging
+            auto ld_init = [&](int t, float4 (&s4)[8]) {
+                const int k0 = (vw * VPT + t) * 32;
+#pragma unroll
+                for (int m = 0; m < 8; ++m) s4[m] = __ldcg((const float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch));
+            };
+            float4 s4b[2][8];
+            ld_init(0, s4b[0]);
+#pragma unroll
             for (int t = 0; t < VPT; ++t) {
+                if (t + 1 < VPT) ld_init(t + 1, s4b[(t + 1) & 1]);
+                const float4 (&s4)[8] = s4b[t & 1];
                 const int k0 = (vw * VPT + t) * 32;
                 const int kk = k0 + lane;
                 const uint32_t bi = vbase + kk < V ? binfo[tb * VL + kk] : 0u;
                 const int bw = (int)(bi & 31u), roff = (int)(bi >> 5);
                 const uint32_t bmask = ((1u << bw) - 1u) << (roff & 3);
-                float4 s4[8];  // e_init windows, in flight during the staging below
-#pragma unroll
-                for (int m = 0; m < 8; ++m) s4[m] = __ldcg((const float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch));
+                // this view's final band -> its staging row (positions outside the band: 0)
                 const float* se = sb_e + kk - (roff & 3) * VS;
-                float* sr = stg_w + lane * 33;
 #pragma unroll
-                for (int p = 0; p < 32; ++p)
-                    if (bmask & (1u << p)) sr[p] = se[p * VS];
+                for (int q4 = 0; q4 < 8; ++q4) {
+                    float rv[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int p = 4 * q4 + j;
+                        rv[j] = (bmask & (1u << p)) ? se[p * VS] : 0.f;
+                    }
+                    *(float4*)(stg_w + lane * kStg + 4 * q4) = make_float4(rv[0], rv[1], rv[2], rv[3]);
+                }
                 __syncwarp();
 #pragma unroll
                 for (int m = 0; m < 8; ++m) {
@@ -1109,10 +1128,12 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     const int oi = __shfl_sync(kFull, roff, i);
                     const uint32_t nib = __shfl_sync(kFull, bmask, i) >> (4 * ch);
                     const int s = oi & 3;
+                    const float4 f4 = *(const float4*)(stg_w + i * kStg + 4 * ch);
+                    const float fv[4] = {f4.x, f4.y, f4.z, f4.w};
                     float d[4];
                     const float e0[4] = {s4[m].x, s4[m].y, s4[m].z, s4[m].w};
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) d[j] = (nib & (1u << j)) ? stg_w[i * 33 + 4 * ch + j] - e0[j] : 0.f;
+                    for (int j = 0; j < 4; ++j) d[j] = (nib & (1u << j)) ? fv[j] - e0[j] : 0.f;
                     if (vbase + k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
                         red_add_v4(ez + (oi - s) + 4 * ch, d[0], d[1], d[2], d[3]);
                 }
@@ -1184,9 +1205,6 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
             atomicAdd(P.tprof + 4, (unsigned long long)nact);
             atomicAdd(P.tprof + 5, 1ull);
             atomicAdd(P.tprof + 6, (unsigned long long)(tp1b - tp1));  // view-warp 0's own pack
-            atomicAdd(P.tprof + 7, (unsigned long long)(tpa - tp1));   // tile 0: issue of loads
-            atomicAdd(P.tprof + 8, (unsigned long long)(tpb - tpa));   // tile 0: loads landed
-            atomicAdd(P.tprof + 9, (unsigned long long)(tpc - tpb));   // tile 0: staging/transposes
         }
     }
 }
