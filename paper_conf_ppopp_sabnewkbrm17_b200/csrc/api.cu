@@ -103,6 +103,7 @@ struct mbir_handle {
     std::vector<cudaEvent_t> kev;  // per-launch event pairs of the update kernel (one iteration)
     int kev_used = 0;
     unsigned long long* d_tprof = nullptr;  // phase cycle counters (env MBIR_PHASE_PROFILE)
+    unsigned long long* d_trace = nullptr;  // per-pair clock trace of one visit (env MBIR_TRACE)
     std::string err;
 };
 
@@ -162,6 +163,7 @@ IcdParams make_params(mbir_handle* h)
     p.iter = h->iter;
     p.deterministic = h->o.deterministic;
     p.tprof = h->d_tprof;
+    p.trace = h->d_trace;
     p.dbg = getenv("MBIR_DBG") ? atoi(getenv("MBIR_DBG")) : 0;
     return p;
 }
@@ -469,7 +471,15 @@ void mbir_destroy(mbir_handle* h)
                     h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
                     h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count,
                     h->d_flat, h->d_brange, h->d_fetch, h->d_perm, h->d_counters, h->d_sum_delta,
-                    h->d_flag, h->d_acc, h->d_tprof};
+                    h->d_flag, h->d_acc, h->d_tprof, h->d_trace};
+    if (h->d_trace && getenv("MBIR_TRACE")) {  // development aid: raw clock stamps (tools/trace_visit.py)
+        std::vector<unsigned long long> t(1024);
+        cudaMemcpy(t.data(), h->d_trace, 1024 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+        if (FILE* f = fopen(getenv("MBIR_TRACE"), "wb")) {
+            fwrite(t.data(), sizeof(unsigned long long), t.size(), f);
+            fclose(f);
+        }
+    }
     for (void* p : ptrs)
         if (p) cudaFree(p);
     if (h->h_counters) cudaFreeHost(h->h_counters);
@@ -683,6 +693,10 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_sum_delta, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_flag, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_acc, 1))) return bail(r);
+    if (getenv("MBIR_TRACE")) {  // development aid: dumped to the file MBIR_TRACE names by mbir_destroy
+        if ((r = dalloc(h, &h->d_trace, 1024))) return bail(r);
+        cudaMemset(h->d_trace, 0, 1024 * sizeof(unsigned long long));
+    }
     if (getenv("MBIR_PHASE_PROFILE")) {
         if ((r = dalloc(h, &h->d_tprof, 32))) return bail(r);
         cudaMemset(h->d_tprof, 0, 32 * sizeof(unsigned long long));

@@ -588,6 +588,13 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
         if (q >= tend) break;
         const int tk = P.flat[q];
         const int z = tk >> 14, sv = tk & 16383;  // local slice, SV
+        // development aid (env MBIR_TRACE, profiled build only): clock64 stamps of every voxel pair
+        // of one SV visit (CTA 0's sixth task of the first launch), slot 1 + 16 * pair + k
+        const bool TR = PROF && P.trace && blockIdx.x == 0 && ntask == 5 && *(volatile unsigned long long*)P.trace == 0ull;
+        auto stamp = [&](int pair, int k) {
+            if (TR) P.trace[1 + 16 * pair + k] = (unsigned long long)clock64();
+        };
+        if (threadIdx.x == 0) stamp(60, 0);
         const int zg = P.z_offset + z;            // global slice
         const int bx = sv % P.nsvx, by = sv / P.nsvx;
         const int gx0 = bx * side, gy0 = by * side;
@@ -738,6 +745,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
         }
 
         if (PROF && P.tprof && threadIdx.x == 0) tp1 = clock64();
+        if (threadIdx.x == 0) stamp(60, 1);
         // ---- 4. view threads: SVB pack (coalesced 128-byte band rows, transposed by shuffles);
         //         e_init rows go to this CTA's L2-resident scratch tile for the write-back
         float* scr = P.scratch + (size_t)blockIdx.x * (size_t)P.Vs * 32;
@@ -819,6 +827,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
         __syncthreads();
 
         if (PROF && P.tprof && threadIdx.x == 0) tp2 = clock64();
+        if (threadIdx.x == 0) stamp(60, 2);
         // ---- 5. sequential-exact voxel loop, TWO voxels (a, b) per barrier.  Both are gathered
         //         from the same state of e, together with the overlap H = sum w A_b A_a over their
         //         shared sinogram entries; after the barrier every warp computes delta_a, then
@@ -905,6 +914,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
             // barrier B (deltas) -> scatter -> refill the next pair's stages
             auto pair_step = [&](int idx, PairState& cur, PairState& nxt) {
                 const uint32_t pn = pseq + (uint32_t)(idx >> 1);  // running pair number
+                if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 0 : 8);
                 const int buf = (int)(pn % kPairBufs);
                 // ---- the pair's theta1 partials: sum (w A_a) e and sum (w A_b) e over this
                 //      thread's views, from the state of e after the previous pair's scatter
@@ -952,13 +962,16 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     }
                 }
                 // barrier A: arrive (the prior warp derives the deltas)
+                if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 1 : 9);
                 if (CL == 1) asm volatile("bar.arrive 1, %0;" ::"r"(npair_threads) : "memory");
                 // ---- meanwhile: the next pair's e-independent state
                 if (idx + 2 < nact) prep(idx + 2, idx + 3 < nact, nxt);
+                if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 2 : 10);
                 // ---- barrier B: the deltas are published
                 {
                     const long long tw0 = (PROF && P.tprof) ? clock64() : 0;
                     asm volatile("bar.sync 2, %0;" ::"r"(npair_threads) : "memory");
+                    if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 3 : 11);
                     if (PROF && P.tprof && lane == 0)  // development aid: per-warp wait for the deltas
                         atomicAdd(P.tprof + 10 + warp, (unsigned long long)(clock64() - tw0));
                 }
@@ -987,6 +1000,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                              __ffma2_rn(fb[1], ndb, __ffma2_rn(fab[1], nda, eb[t][1])));
                     }
                 }
+                if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 4 : 12);
                 // the next pair's stages are consumed (its state is in registers): refill them
                 // with the records R voxels ahead
                 copy_record(idx + 2 + R, tp);
@@ -1015,10 +1029,12 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 const bool hasb = idx + 1 < nact;
                 {
                     const long long tw0 = (PROF && P.tprof) ? clock64() : 0;
+                    if (lane == 0) stamp(idx >> 1, 5);
                     if (CL == 1)
                         asm volatile("bar.sync 1, %0;" ::"r"(npair_threads) : "memory");
                     else
                         mbar_wait_cluster(pairbar + buf, (pn / kPairBufs) & 1u);
+                    if (lane == 0) stamp(idx >> 1, 6);
                     if (PROF && P.tprof && lane == 0)  // development aid: wait for the partial sums
                         atomicAdd(P.tprof + 10 + warp, (unsigned long long)(clock64() - tw0));
                 }
@@ -1058,6 +1074,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     dslot[(pn & 1) * 2] = scale_a * da;
                     dslot[(pn & 1) * 2 + 1] = scale_b * db;
                 }
+                if (lane == 0) stamp(idx >> 1, 7);
                 asm volatile("bar.arrive 2, %0;" ::"r"(npair_threads) : "memory");  // barrier B
                 // the pair's new values, then the next pair's surrogate terms
                 if (lane == 0) {
@@ -1077,12 +1094,14 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
                                pri + (pn + 1) % kPairBufs);
                 if (PROF && P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
+                if (lane == 0) stamp(idx >> 1, 13);
             }
         }
         gseq += nact;
         pseq += (uint32_t)(nact + 1) >> 1;
         ++ntask;
         if (PROF && P.tprof && threadIdx.x == 0) tp3 = clock64();
+        if (threadIdx.x == 0) stamp(60, 3);
         __syncthreads();
 
         // ---- 6. write-back: delta e of the band, atomically, and the SV's voxels
@@ -1196,6 +1215,10 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
             }
         }
         if (CL == 2) cluster_sync_all(); else __syncthreads();
+        if (threadIdx.x == 0) {
+            stamp(60, 4);
+            if (TR) P.trace[0] = 1ull + (unsigned long long)nact;
+        }
         if (PROF && P.tprof && threadIdx.x == 0 && crank == 0) {
             const long long tp4 = clock64();
             atomicAdd(P.tprof + 0, (unsigned long long)(tp1 - tp0));  // x tile, zero-skip, order
@@ -1389,7 +1412,7 @@ static cudaError_t launch_icd_t(const IcdParams& p, int gx, int gy, cudaStream_t
     // the phase-profiling instrumentation (env MBIR_PHASE_PROFILE) is compiled only into the
     // bench's configuration; every other launch runs the instrumentation-free kernel
     constexpr bool kProfiled = VPT == 4 && U8 && CL == 1;
-    auto kern = (kProfiled && p.tprof) ? k_icd_sv<VPT, U8, NNB, R, CL, kProfiled> : k_icd_sv<VPT, U8, NNB, R, CL, false>;
+    auto kern = (kProfiled && (p.tprof || p.trace)) ? k_icd_sv<VPT, U8, NNB, R, CL, kProfiled> : k_icd_sv<VPT, U8, NNB, R, CL, false>;
     IcdParams q = p;
     q.lay = smem_layout(p.rows, svb_stride(VPT, CL), p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, CL);
     const int smem = q.lay.total;

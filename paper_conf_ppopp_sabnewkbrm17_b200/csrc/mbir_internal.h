@@ -88,6 +88,7 @@ struct IcdParams {
     int zero_skip_active;
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
+    unsigned long long* trace;  // optional per-pair clock trace of one SV visit (env MBIR_TRACE)
     int dbg;                 // development switches (env MBIR_DBG): bit 0 no A-record L2 warm-up,
                              // bit 1 no band-row L2 warm-up
     SmemLayout lay;          // update-kernel smem layout (filled by launch_icd)

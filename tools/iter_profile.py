@@ -20,13 +20,14 @@ ap.add_argument("--zero-skip", type=int, default=1)
 ap.add_argument("--sv-side", type=int, default=0)
 ap.add_argument("--batch-svs", type=int, default=0)
 ap.add_argument("--cluster", type=int, default=0)
+ap.add_argument("--quantize", type=int, default=1)
 a = ap.parse_args()
 cfg = CONFIGS[a.config]
 y, w = make_sinogram_torch(cfg, 0, "cuda")
 g = M.Geometry(cfg.n, cfg.n, cfg.nz, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dchannel)
 r = M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=cfg.nbhd),
                     M.Options(sv_side=a.sv_side or cfg.sv_side, zero_skip=a.zero_skip,
-                              batch_svs=a.batch_svs, cluster=a.cluster))
+                              batch_svs=a.batch_svs, cluster=a.cluster, quantize_A=a.quantize))
 r.set_sinogram(y, w)
 print(json.dumps(r.sizes()))
 for rep in range(2):
@@ -38,3 +39,4 @@ for rep in range(2):
                   f"t {s['seconds'] * 1e3:8.2f} ms  kernel {s['kernel_seconds'] * 1e3:8.2f} ms  "
                   f"ns/upd {1e9 * s['kernel_seconds'] / max(s['updates'], 1):7.2f}  "
                   f"us/visit {1e6 * s['kernel_seconds'] / max(s['sv_visits'], 1) * 148:8.2f}")
+r.close()
