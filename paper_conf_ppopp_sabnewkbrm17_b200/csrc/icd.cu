@@ -678,11 +678,10 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
         const unsigned char* g_code = (const unsigned char*)(U8 ? (const void*)P.A.codes : (const void*)P.A.vals) +
                                       ((size_t)arec * P.A.VA + vbase + tpm * VPT) * CB;
         const unsigned char* g_off = P.A.off + (size_t)arec * P.A.VA + vbase + tpm * VPT;
-        auto copy_record = [&](int j, int tp) {
-            (void)tp;
+        // record of voxel j (slot v = list[j]) into ring stage `stg`
+        auto copy_record_to = [&](int j, int stg, int v) {
             if (j < nact) {
-                unsigned char* st = astage + ((gseq + (uint32_t)j) % R) * L.stage_bytes;
-                const int v = list[j];
+                unsigned char* st = astage + stg * L.stage_bytes;
                 const unsigned char* gc = g_code + (size_t)v * (P.A.VA * CB);
                 if (U8) {
                     if (VPT == 4)
@@ -700,6 +699,11 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     cp_async4(st + L.off_in_stage + tpm * VPT, g_off + (size_t)v * P.A.VA);
             }
             cp_async_commit();
+        };
+        const int sbase = (int)(gseq % (uint32_t)R);  // ring stage of this visit's voxel 0
+        auto copy_record = [&](int j, int tp) {
+            (void)tp;
+            copy_record_to(j, (sbase + j) % R, j < nact ? list[j] : 0);
         };
         // prior warp, lane 0 (development switch MBIR_DBG bit 0): L2 warm-up of voxel j's record
         auto prefetch_record = [&](int j) {
@@ -855,6 +859,8 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 uint32_t ca[VPT][CW], cb[VPT][CW];
                 float2 wa[VPT][2], wb[VPT][2];
                 float hh;
+                int sj;      // ring stage of voxel j (the pair's first voxel)
+                int lv[2];   // list[j + R], list[j + 1 + R]: the records copied into its stages
             };
             // A values of a record as channel pairs
             auto avals = [&](const uint32_t (&c)[CW], float2 (&f)[2]) {
@@ -879,8 +885,13 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 if (VPT != 4) __syncwarp();  // offset words copied by another lane of the warp
                 if (PROF && P.tprof && lane == 0)   // development aid: A-stream wait
                     atomicAdd(P.tprof + 22 + (j >= R), (unsigned long long)(clock64() - tf0));
-                const unsigned char* sta = astage + ((gseq + (uint32_t)j) % R) * L.stage_bytes;
-                const unsigned char* stb = astage + ((gseq + (uint32_t)j + 1) % R) * L.stage_bytes;
+                const int sb1 = ps.sj + 1 == R ? 0 : ps.sj + 1;
+                const unsigned char* sta = astage + ps.sj * L.stage_bytes;
+                const unsigned char* stb = astage + sb1 * L.stage_bytes;
+                // the slots of the records that will refill these stages (read early: the copy
+                // after the scatter then needs no shared-memory round trip)
+                ps.lv[0] = j + R < nact ? list[j + R] : 0;
+                ps.lv[1] = j + 1 + R < nact ? list[j + 1 + R] : 0;
                 load_words<VPT, CW>(sta, L.off_in_stage, tp, ps.ca, ps.oa);
                 load_words<VPT, CW>(stb, L.off_in_stage, tp, ps.cb, ps.ob);
                 ps.ob = hb ? ps.ob : ps.oa;
@@ -965,6 +976,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 1 : 9);
                 if (CL == 1) asm volatile("bar.arrive 1, %0;" ::"r"(npair_threads) : "memory");
                 // ---- meanwhile: the next pair's e-independent state
+                nxt.sj = cur.sj + 2 >= R ? cur.sj + 2 - R : cur.sj + 2;
                 if (idx + 2 < nact) prep(idx + 2, idx + 3 < nact, nxt);
                 if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 2 : 10);
                 // ---- barrier B: the deltas are published
@@ -1003,14 +1015,18 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 4 : 12);
                 // the next pair's stages are consumed (its state is in registers): refill them
                 // with the records R voxels ahead
-                copy_record(idx + 2 + R, tp);
-                copy_record(idx + 3 + R, tp);
+                {
+                    const int s1 = nxt.sj + 1 == R ? 0 : nxt.sj + 1;
+                    copy_record_to(idx + 2 + R, nxt.sj, nxt.lv[0]);
+                    copy_record_to(idx + 3 + R, s1, nxt.lv[1]);
+                }
             };
             // the A records of the first R voxels (every stage is free: the previous visit ended
             // with a CTA-wide barrier), then the first pair's state; its stages are refilled.
             // The pair loop is unrolled by two so the two states swap roles without copies.
             PairState st0, st1;
             for (int i = 0; i < R; ++i) copy_record(i, tp);
+            st0.sj = sbase;
             prep(0, 1 < nact, st0);
             copy_record(R, tp);
             copy_record(R + 1, tp);
