@@ -5,8 +5,11 @@
 // for GPU load balance); the chosen set is split into 4 checkerboard groups whose members share
 // no boundary (Fig. 3).  Reading R14: the update amount is sum |delta| of the SV's
 // most recent visit, the selection is made per slice, ties go to the lower SV index, and the
-// random subset is uniform without replacement from a counter-based hash of
-// (seed, iteration, slice, SV).
+// random subset (and iteration 1's random order) is uniform without replacement from a
+// counter-based hash of (seed, iteration, SV) -- the same for every slice, so the flat task list
+// (rank r of every slice, then r + 1, ...) runs one SV at all slices of a phase back to back and
+// the concurrently running CTAs share that SV's A records through L2 (A is slice-invariant in
+// parallel beam, cross-slice A reuse).
 //
 // One CTA per slice: keys in shared memory -> bitonic sort -> the first nsel keys are the
 // selection, in key order -> a block-wide scan of 4 packed 16-bit colour counters places every
@@ -30,7 +33,7 @@ __global__ void __launch_bounds__(kSelThreads) k_select(const SchedParams S)
 {
     extern __shared__ unsigned long long keys[];  // [nsv_pad]
     __shared__ unsigned long long wscan[kSelThreads / 32];
-    const int z = blockIdx.x, zg = S.z_offset + z;
+    const int z = blockIdx.x;
     const int n = S.nsv_pad;
     for (int i = threadIdx.x; i < n; i += blockDim.x) {
         unsigned long long key = ~0ull;
@@ -42,8 +45,7 @@ __global__ void __launch_bounds__(kSelThreads) k_select(const SchedParams S)
             } else if (S.mode == 3) {
                 key = (unsigned long long)i;
             } else {
-                const uint64_t h = mix64s(S.seed ^ 0x5bd1e995ULL ^
-                                          mix64s(((uint64_t)S.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)i));
+                const uint64_t h = mix64s(S.seed ^ 0x5bd1e995ULL ^ mix64s(((uint64_t)S.iter << 40) ^ (uint64_t)i));
                 key = ((unsigned long long)(uint32_t)(h >> 32) << 32) | (unsigned)i;
             }
         }
