@@ -80,8 +80,10 @@ typedef struct mbir_prior {
 typedef struct mbir_options {
     int sv_side;           /* SuperVoxel side s; tiles of s x s voxels, default 9   */
     double sv_fraction;    /* fraction of SVs per iteration >= 2, default 0.25  */
-    int batch_svs;         /* BATCH_SIZE: SVs per slice per launch (Alg3:25); 0 = a whole
-                              checkerboard colour group per launch (no threshold), default 0   */
+    int batch_svs;         /* BATCH_SIZE: SVs per slice per launch (Alg3:25); 0 = auto: a whole
+                              checkerboard colour group per launch when the phase spans enough
+                              slices that <= 32 SVs of one slice run at once, else batches of
+                              32 SVs per slice (no threshold); default 0                          */
     int batch_threshold;   /* Alg3:26-27: drop a group's remainder smaller than this; -1 =
                               batch_svs/4; ignored when batch_svs == 0                   */
     int zero_skip;         /* P:115, default 1 (never in iteration 1; reading R9)               */

@@ -276,7 +276,15 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         ++launches;
         // ---- flat task lists + batch ranges per (z-parity, colour) phase (Alg3:24-27)
         const bool det = h->o.deterministic != 0;
-        const int B = (det || h->o.batch_svs <= 0) ? h->max_group : h->o.batch_svs;
+        // batch_svs = 0 (auto): a whole colour group per launch, unless the phase has so few slices
+        // that more than kAutoBatch SVs of one slice would run at once -- then batches of
+        // kAutoBatch SVs per slice, each launch seeing the previous one's write-backs.  Same-colour
+        // SVs updated concurrently fit the same residual along shared rays; with ~148 of them in
+        // one 2-D slice the first sweeps from x0 = 0 overshoot, clip whole SVs to 0 and zero-skip
+        // then freezes them (reading R22).
+        const int slices_in_phase = std::max(1, h->g.nz_local / parities);
+        const bool auto_batch = !det && h->o.batch_svs == 0 && target_ctas > kAutoBatch * slices_in_phase;
+        const int B = auto_batch ? kAutoBatch : (det || h->o.batch_svs <= 0) ? h->max_group : h->o.batch_svs;
         const int thr = (det || h->o.batch_svs <= 0) ? 0 : (h->o.batch_threshold >= 0 ? h->o.batch_threshold : B / 4);
         const int nb = (h->max_group + B - 1) / B;
         CK(launch_flatten(h->d_task_list, h->d_task_count, h->g.nz_local, h->g.z_offset, parities,

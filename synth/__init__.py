@@ -16,4 +16,5 @@ from .phantom import (  # noqa: F401
     shepp_logan_2d,
     shepp_logan_3d,
     sinogram,
+    sweep_configs,
 )

@@ -244,6 +244,40 @@ def test_converged_3d_matches_oracle(zero_skip, tol_hu, tol_cost):
     assert abs(cg - co) <= tol_cost * abs(co)
 
 
+SWEEP_SMALL = [  # (phantom, baggage seed, lambda0, views, SV side): BASELINE configs[4]'s axes at N = 64
+    ("shepp_logan", 0, 1e3, 180, 5),
+    ("baggage", 0, 1e4, 90, 7),
+    ("baggage", 1, 1e5, 360, 9),
+    ("shepp_logan", 0, 1e5, 90, 9),
+]
+
+
+@pytest.mark.parametrize("case", SWEEP_SMALL, ids=[f"{c[0]}{c[1]}-l{int(c[2])}-v{c[3]}-s{c[4]}" for c in SWEEP_SMALL])
+def test_sweep_cases_converge_to_oracle(case):
+    """The sweep's variety (BASELINE.json configs[4]: phantom incl. baggage-like scenes with a
+    large air fraction, dose, view count, SV side; M = 2N as in the paper) at a size the oracle
+    converges in seconds: converged image within 1 HU and cost within 1e-4 of the oracle's."""
+    ph, bseed, lam, v, side = case
+    cfg = WorkloadConfig("sweep-small", 64, 1, v, 128, side, 8, 0.002, phantom=ph, lambda0=lam)
+    c = make_case(cfg, 100 + bseed)
+    g, og = geoms(cfg)
+    A = O.sysmatrix(og)
+    _, _, Aq = O.quantize(A)
+    pr = O.Prior(sigma=cfg.sigma, nbhd=8)
+    x = np.zeros(cfg.n * cfg.n)
+    e = O.error_sinogram(og, Aq, c.y.astype(np.float64), x)
+    O.icd_run(og, pr, Aq, c.w, x, e, 150, seed=3000, zero_skip=False)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=8),
+                         M.Options(sv_side=side, zero_skip=0)) as r:
+        r.set_sinogram(c.y, c.w)
+        r.reconstruct(300)
+        xg = r.image().ravel().astype(np.float64)
+    assert O.rmse_hu(xg, x) < 1.0, O.rmse_hu(xg, x)
+    cg = O.cost(og, pr, Aq, c.y, c.w, xg)
+    co = O.cost(og, pr, Aq, c.y, c.w, x)
+    assert abs(cg - co) <= 1e-4 * abs(co), (cg, co)
+
+
 # ------------------------------------------------------------------ scheduler + accounting
 def test_iteration_accounting_and_selection_fractions(cfg1):
     """Alg3:17-22: iteration 1 visits every SV of every slice; later iterations
