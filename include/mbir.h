@@ -164,6 +164,14 @@ int mbir_set_sinogram(mbir_handle* h, const float* y, const float* w, int where)
  * if a sinogram is loaded.  Errors: EINVAL (negative values with positivity), ECUDA. */
 int mbir_set_image(mbir_handle* h, const float* x0, int where);
 
+/* Set the image to the filtered back-projection of the loaded sinogram y (Ram-Lak filter by
+ * direct convolution, linearly interpolated back-projection, clipped at 0 with positivity;
+ * Kak & Slaney ch. 3) and recompute e = y - A x.  An initial image only: the paper does not
+ * state one (reading R23) and ICD converges to the same MAP point from any start.
+ * Collective across ranks (halo exchange).  Uses a temporary [nz_local][nviews][nchannels]
+ * device buffer.  Errors: ESTATE (no sinogram), ENOMEM, ECUDA, ENCCL. */
+int mbir_init_fbp(mbir_handle* h);
+
 /* Run whole iterations of GPU-ICD (Alg. 3 lines 16-31) until at least `equits` equits of
  * executed updates have been done by this call (one equit = nx*ny*nz_total updates).
  * Collective across ranks.  st may be NULL.  Errors: ESTATE (no sinogram), ENUMERIC, ECUDA,

@@ -280,3 +280,38 @@ def rmse_hu(a, b, mu_water: float = MU_WATER) -> float:
     a = np.ascontiguousarray(a, np.float64).ravel()
     b = np.ascontiguousarray(b, np.float64).ravel()
     return lib().orc_rmse_hu(_p(a, C.c_double), _p(b, C.c_double), a.size, mu_water)
+
+
+def fbp(g: Geometry, y, positivity: bool = True) -> np.ndarray:
+    """Filtered back-projection of y [nz][V][M] (the optional initial image of mbir_init_fbp;
+    not part of the paper's method, reading R23), in float64, written from the textbook
+    definition (Kak & Slaney, ch. 3, eqs. 61-63): q_k = dc * (h * p_k) with the band-limited ramp
+    h(0) = 1/(4 dc^2), h(n dc) = -1/(pi^2 n^2 dc^2) for odd n, 0 for even n != 0 (full linear
+    convolution, np.convolve); f(x, y) = (pi / V) sum_k q_k(x cos th_k + y sin th_k), linear
+    interpolation between channel centres t0 + (m + 1/2) dc, zero outside the detector.
+    Returns [nz][ny][nx], clipped at 0 when positivity."""
+    y = np.asarray(y, np.float64)
+    V, M = g.nviews, g.nchannels
+    dc = g.dchannel
+    n = np.arange(-(M - 1), M)
+    h = np.zeros(n.size)
+    h[n == 0] = 1.0 / (4 * dc * dc)
+    odd = n % 2 != 0
+    h[odd] = -1.0 / (np.pi ** 2 * n[odd].astype(np.float64) ** 2 * dc * dc)
+    th = np.asarray(g.angles, np.float64) if g.angles is not None else np.arange(V) * np.pi / V
+    t0 = -0.5 * M * dc + g.center_offset * dc
+    xc = (np.arange(g.nx) - 0.5 * (g.nx - 1)) * g.dxy
+    yc = (np.arange(g.ny) - 0.5 * (g.ny - 1)) * g.dxy
+    X, Y = np.meshgrid(xc, yc)  # [iy][ix]
+    out = np.zeros((y.shape[0], g.ny, g.nx))
+    for z in range(y.shape[0]):
+        for k in range(V):
+            q = dc * np.convolve(y[z, k], h)[M - 1: 2 * M - 1]
+            u = (X * np.cos(th[k]) + Y * np.sin(th[k]) - t0) / dc - 0.5
+            m = np.floor(u).astype(np.int64)
+            f = u - m
+            qa = np.where((m >= 0) & (m < M), q[np.clip(m, 0, M - 1)], 0.0)
+            qb = np.where((m + 1 >= 0) & (m + 1 < M), q[np.clip(m + 1, 0, M - 1)], 0.0)
+            out[z] += qa + f * (qb - qa)
+    out *= np.pi / V
+    return np.maximum(out, 0.0) if positivity else out

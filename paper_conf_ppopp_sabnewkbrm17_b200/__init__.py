@@ -22,6 +22,7 @@ from .api import (  # noqa: F401
     mbir_reconstruct,
     mbir_rmse_hu,
     mbir_set_image,
+    mbir_init_fbp,
     mbir_set_sinogram,
 )
 from ._lib import LIB_PATH, MbirError, load  # noqa: F401

@@ -23,7 +23,7 @@ MBIR_DEVICE = 1
 # every symbol include/mbir.h declares (checked by tests/test_abi.py)
 EXPORTS = (
     "mbir_default_options", "mbir_default_prior", "mbir_create", "mbir_set_sinogram",
-    "mbir_set_image", "mbir_reconstruct", "mbir_iterate", "mbir_get_image",
+    "mbir_set_image", "mbir_init_fbp", "mbir_reconstruct", "mbir_iterate", "mbir_get_image",
     "mbir_get_error_sinogram", "mbir_rmse_hu", "mbir_query_sizes", "mbir_get_sysmatrix",
     "mbir_get_sysmatrix_columns",
     "mbir_probe_update", "mbir_nccl_unique_id", "mbir_halo_plan", "mbir_destroy",
@@ -110,6 +110,8 @@ def load(path: str = LIB_PATH):
     L.mbir_set_sinogram.argtypes = [H, vp, vp, C.c_int]
     L.mbir_set_image.restype = C.c_int
     L.mbir_set_image.argtypes = [H, vp, C.c_int]
+    L.mbir_init_fbp.restype = C.c_int
+    L.mbir_init_fbp.argtypes = [H]
     L.mbir_reconstruct.restype = C.c_int
     L.mbir_reconstruct.argtypes = [H, C.c_double, C.POINTER(mbir_stats)]
     L.mbir_iterate.restype = C.c_int

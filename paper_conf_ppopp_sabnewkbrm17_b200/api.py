@@ -146,6 +146,10 @@ def mbir_set_image(h, g: Geometry, x0=None):
     L.check(L.load().mbir_set_image(h, px, where), h, "mbir_set_image")
 
 
+def mbir_init_fbp(h):
+    L.check(L.load().mbir_init_fbp(h), h, "mbir_init_fbp")
+
+
 def mbir_reconstruct(h, equits: float) -> dict:
     st = L.mbir_stats()
     L.check(L.load().mbir_reconstruct(h, float(equits), C.byref(st)), h, "mbir_reconstruct")
@@ -263,6 +267,10 @@ class Reconstructor:
 
     def set_image(self, x0=None):
         mbir_set_image(self.h, self.g, x0)
+
+    def init_fbp(self):
+        """x0 = FBP of the loaded sinogram (mbir_init_fbp)."""
+        mbir_init_fbp(self.h)
 
     def reconstruct(self, equits: float) -> dict:
         return mbir_reconstruct(self.h, equits)

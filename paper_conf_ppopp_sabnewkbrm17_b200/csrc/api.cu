@@ -822,6 +822,28 @@ int mbir_set_image(mbir_handle* h, const float* x0, int where)
     return MBIR_OK;
 }
 
+int mbir_init_fbp(mbir_handle* h)
+{
+    if (!h) return MBIR_EINVAL;
+    if (!h->have_sino) return fail(h, MBIR_ESTATE, "mbir_set_sinogram has not been called");
+    const size_t pl = plane_elems(h), ns = sino_elems(h);
+    float* q = nullptr;
+    if (cudaMallocAsync((void**)&q, ns * sizeof(float), h->st) != cudaSuccess)
+        return fail(h, MBIR_ENOMEM, "cudaMallocAsync (FBP filtered sinogram)");
+    cudaError_t e = launch_fbp(h->g, h->d_cs, h->d_y, q, h->d_x + pl, h->pr.positivity, h->st);
+    cudaFreeAsync(q, h->st);
+    if (e != cudaSuccess) return fail(h, MBIR_ECUDA, std::string("FBP: ") + cudaGetErrorString(e));
+    h->x_zero = false;
+    int r = exchange_halo(h, -1);
+    if (r) return r;
+    r = refresh_error(h, false);
+    if (r) return r;
+    CK(cudaMemsetAsync(h->d_amount, 0, sizeof(float) * h->g.nz_local * h->nsv, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    h->iter = 0;
+    return MBIR_OK;
+}
+
 int mbir_reconstruct(mbir_handle* h, double equits, mbir_stats* st)
 {
     if (!h || !(equits >= 0)) return MBIR_EINVAL;

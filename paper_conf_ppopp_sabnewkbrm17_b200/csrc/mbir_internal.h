@@ -129,6 +129,9 @@ cudaError_t launch_select(const SchedParams& sp, cudaStream_t st);
 cudaError_t launch_flatten(const int* task_list, const int* task_count, int nz_local, int z_offset,
                            int parities, int max_group, int batch, int thr, int nb, int* flat,
                            int* brange, cudaStream_t st);
+// FBP initial image (fbp.cu): q = ramp-filtered y (scratch [nz][V][M]), x = clip(backprojection)
+cudaError_t launch_fbp(const mbir_geometry& g, const double* d_cs, const float* y, float* q, float* x,
+                       int positivity, cudaStream_t st);
 cudaError_t launch_rmse_partial(const float* x, const float* g, int64_t n, double* acc,
                                 cudaStream_t st);
 cudaError_t launch_check_finite(const float* a, int64_t n, int nonneg, int* flag, cudaStream_t st);

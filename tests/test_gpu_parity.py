@@ -423,3 +423,44 @@ def test_cluster_option_validation():
     assert ei.value.code == -1
     with M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side)) as r:
         assert r.sizes()["cluster"] == 1
+
+
+# ------------------------------------------------------------------ FBP initial image (R23)
+def test_fbp_init_matches_reference_and_converges(cfg1):
+    """mbir_init_fbp: the device FBP equals the float64 textbook reference (oracle.fbp) to fp32
+    accuracy, e is reset to y - A x, and ICD from it reaches the same MAP point as the oracle."""
+    cfg, case, g, og, A, codes, amax, Aq = cfg1
+    ref = O.fbp(og, case.y)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=8),
+                         M.Options(sv_side=cfg.sv_side, zero_skip=0)) as r:
+        r.set_sinogram(case.y, case.w)
+        r.init_fbp()
+        x0 = r.image().astype(np.float64)
+        e0 = r.error_sinogram()
+        assert np.abs(x0 - ref).max() <= 2e-5 * np.abs(ref).max(), np.abs(x0 - ref).max()
+        eo = O.error_sinogram(og, Aq, case.y.astype(np.float64), x0.ravel())
+        assert np.abs(e0.ravel() - eo.ravel()).max() < 1e-4 * np.abs(case.y).max()
+        r.reconstruct(300)
+        xg = r.image().ravel().astype(np.float64)
+    pr = O.Prior(sigma=cfg.sigma, nbhd=8)
+    x = np.zeros(cfg.n * cfg.n)
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+    O.icd_run(og, pr, Aq, case.w, x, e, 150, seed=3000, zero_skip=False)
+    assert O.rmse_hu(xg, x) < 1.0
+    cg = O.cost(og, pr, Aq, case.y, case.w, xg)
+    co = O.cost(og, pr, Aq, case.y, case.w, x)
+    assert abs(cg - co) <= 1e-4 * abs(co)
+
+
+def test_fbp_init_3d_slab_and_state_errors():
+    cfg = small3d()
+    case = make_case(cfg)
+    g, og = geoms(cfg)
+    ref = O.fbp(og, case.y)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26), M.Options(sv_side=cfg.sv_side)) as r:
+        with pytest.raises(M.MbirError):
+            r.init_fbp()  # no sinogram yet: MBIR_ESTATE
+        r.set_sinogram(case.y, case.w)
+        r.init_fbp()
+        x0 = r.image().astype(np.float64)
+    assert np.abs(x0 - ref).max() <= 2e-5 * np.abs(ref).max()
