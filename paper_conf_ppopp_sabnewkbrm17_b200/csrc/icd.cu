@@ -978,6 +978,14 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 // ---- meanwhile: the next pair's e-independent state
                 nxt.sj = cur.sj + 2 >= R ? cur.sj + 2 - R : cur.sj + 2;
                 if (idx + 2 < nact) prep(idx + 2, idx + 3 < nact, nxt);
+                // the next pair's stages are consumed (prep has used its records): refill them
+                // with the records R voxels ahead while the deltas are being derived (one commit
+                // group per voxel, empty past the visit's end, keeps the wait counts fixed)
+                {
+                    const int s1 = nxt.sj + 1 == R ? 0 : nxt.sj + 1;
+                    copy_record_to(idx + 2 + R, nxt.sj, nxt.lv[0]);
+                    copy_record_to(idx + 3 + R, s1, nxt.lv[1]);
+                }
                 if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 2 : 10);
                 // ---- barrier B: the deltas are published
                 {
@@ -1013,13 +1021,6 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                     }
                 }
                 if (lane == 0 && (vw == 0 || vw == 5)) stamp(idx >> 1, vw == 0 ? 4 : 12);
-                // the next pair's stages are consumed (its state is in registers): refill them
-                // with the records R voxels ahead
-                {
-                    const int s1 = nxt.sj + 1 == R ? 0 : nxt.sj + 1;
-                    copy_record_to(idx + 2 + R, nxt.sj, nxt.lv[0]);
-                    copy_record_to(idx + 3 + R, s1, nxt.lv[1]);
-                }
             };
             // the A records of the first R voxels (every stage is free: the previous visit ended
             // with a CTA-wide barrier), then the first pair's state; its stages are refilled.
