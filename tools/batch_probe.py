@@ -12,6 +12,9 @@ ap.add_argument("--batches", default="0,8,16,32,64")
 ap.add_argument("--golden-equits", type=float, default=100)
 ap.add_argument("--zero-skip", type=int, default=1)
 ap.add_argument("--det", type=int, default=0)
+ap.add_argument("--fbp", type=int, default=0)
+ap.add_argument("--cluster", type=int, default=0)
+ap.add_argument("--max-equits", type=float, default=150)
 a = ap.parse_args()
 if a.case in CONFIGS:
     cfg, cid = CONFIGS[a.case], 0
@@ -27,8 +30,10 @@ with M.Reconstructor(g, pr, M.Options(sv_side=cfg.sv_side, deterministic=1, zero
     gold = torch.from_numpy(r.image().copy()).cuda()
 print(cfg.name, cfg.n, cfg.nviews, "golden max", float(gold.max()))
 for b in [int(x) for x in a.batches.split(",")]:
-    with M.Reconstructor(g, pr, M.Options(sv_side=cfg.sv_side, batch_svs=b, batch_threshold=0, zero_skip=a.zero_skip, deterministic=a.det)) as r:
+    with M.Reconstructor(g, pr, M.Options(sv_side=cfg.sv_side, batch_svs=b, batch_threshold=0, zero_skip=a.zero_skip, deterministic=a.det, cluster=a.cluster)) as r:
         r.set_sinogram(y, w)
+        if a.fbp:
+            r.init_fbp()
         t = eq = 0.0
         hist = []
         for it in range(400):
@@ -36,5 +41,5 @@ for b in [int(x) for x in a.batches.split(",")]:
             t += st["seconds"]; eq += st["equits"]
             hu = r.rmse_hu(gold)
             if it < 4: hist.append(round(hu, 1))
-            if hu < 10 or eq > 150: break
+            if hu < 10 or eq > a.max_equits: break
         print(f"batch {b:4d}: iters {it+1:4d} equits {eq:7.2f} device {t*1e3:8.2f} ms  final HU {hu:8.2f}  first HU {hist}")
