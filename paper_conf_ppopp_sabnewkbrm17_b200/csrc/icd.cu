@@ -1292,7 +1292,7 @@ __global__ void k_forward(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
     float* acc = (float*)smem;  // [rows][Vs]
-    const int sv = blockIdx.x, z = blockIdx.y;
+    const int z = blockIdx.x, sv = blockIdx.y;
     const int bx = sv % P.nsvx, by = sv / P.nsvx;
     const int gx0 = bx * P.side, gy0 = by * P.side;
     const int tw = min(P.side, P.nx - gx0), th = min(P.side, P.ny - gy0);
@@ -1542,7 +1542,7 @@ cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cu
     auto k = quantize ? k_forward<true> : k_forward<false>;
     e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    k<<<dim3(p.nsv, p.nz_local), 256, smem, st>>>(p);
+    k<<<dim3(p.nz_local, p.nsv), 256, smem, st>>>(p);  // slices of one SV adjacent: A from L2
     return cudaGetLastError();
 }
 
