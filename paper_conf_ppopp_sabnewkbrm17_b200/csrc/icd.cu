@@ -5,23 +5,23 @@
 // intra-voxel, intra-SV and inter-SV parallelism over SV buffers
 // created before and written back after the update.
 //
-// B200 design: one CTA owns one (slice, SV) task at a time
-// (persistent over the phase's task list).  Its threads own VIEWS: warp w, lane l owns views
-// (w*VPT + t)*32 + l, t < VPT.  The SV buffer (e and w over the SV's sinogram band) lives in
-// shared memory as [row = channel offset in band][view] with a view stride that is a multiple
-// of 32, so a warp's 32 lanes always hit 32 distinct banks whatever the voxel's per-view
-// offsets (conflict-free gather and scatter without atomics: a thread is the only writer of
-// its views).  Voxels of the SV are updated one after another in a random order, exactly as
-// sequential ICD within the SV: per voxel, every view thread gathers its part of
-// theta1 = -sum w A e from shared memory (A streamed from HBM, prefetched RING voxels ahead),
-// a warp-shuffle reduction and ONE __syncthreads hand the partial sums to every warp, a
-// dedicated prior warp has meanwhile computed the q-GGMRF surrogate terms over the voxel's
-// neighbourhood from a shared-memory x tile, and every warp derives the same delta and
-// scatters e -= A delta into its own views.  theta2 = A^T W A is fixed by w and is
-// precomputed per (slice, voxel) when the sinogram is loaded.  The SVB is packed and written
-// back with coalesced 128-byte row accesses transposed through warp shuffles; the write-back
-// adds the band's delta e atomically (red.global.add.f32) because same-colour SVs of a batch
-// share sinogram entries.
+// B200 design: one CTA per SM owns one (slice, SV) task at a time,
+// persistent over the phase's task list.  Its view threads own VIEWS: view warp w, lane l owns
+// views (w*VPT + t)*32 + l, t < VPT.  The SV buffer (e and w over the SV's sinogram band) lives
+// in shared memory as [row = channel offset in band][view] with a view stride that is a multiple
+// of 32, so a warp's 32 lanes always hit 32 distinct banks whatever the voxels' per-view offsets
+// (conflict-free gather and scatter without atomics: a thread is the only writer of its views).
+// Voxels of the SV are updated in a random order exactly as sequential ICD, two per step: the
+// view warps gather both voxels' theta1 partials from the same e (their overlap H = sum w A_b A_a
+// and w A were prepared in the previous step), warp-reduce and arrive on a named barrier; the
+// prior warp derives delta_a, then theta1_b corrected by a's change and delta_b (q-GGMRF
+// surrogate, reading R1), publishes them on a second barrier and computes the next pair's
+// surrogate sums from a shared-memory x tile; the view warps scatter e -= A delta into their own
+// views.  A records (uint8 codes + band offsets) are streamed R voxels ahead by per-thread
+// cp.async.  theta2 = A^T W A is fixed by w and precomputed per (slice, voxel).  The SVB is
+// packed from 16-byte-aligned band windows transposed through per-warp staging tiles, and written
+// back as delta e = final - e_init with red.global.add.v4.f32, because same-colour SVs share
+// sinogram entries.
 #include "mbir_internal.h"
 
 #include <cstdio>
@@ -59,29 +59,6 @@ __device__ __forceinline__ float dq(uint32_t word, int i)
 {
     const uint32_t b = __byte_perm(word, 0x4B000000u, 0x7440u | (uint32_t)i);
     return __uint_as_float(b) - 8388608.f;
-}
-
-// In-register 32x32 transpose across a warp: on return lane l holds in r[i] what lane i held
-// in r[l].  5 butterfly stages of 16 shuffles.
-__device__ __forceinline__ void transpose32(float (&r)[32], int lane)
-{
-#pragma unroll
-    for (int s = 4; s >= 0; --s) {
-        const int b = 1 << s;
-        const bool upper = (lane & b) != 0;
-#pragma unroll
-        for (int i = 0; i < 32; ++i) {
-            if ((i & b) == 0) {
-                const int j = i | b;
-                const float send = upper ? r[i] : r[j];
-                const float recv = __shfl_xor_sync(kFull, send, b);
-                if (upper)
-                    r[i] = recv;
-                else
-                    r[j] = recv;
-            }
-        }
-    }
 }
 
 __device__ __forceinline__ void red_add_f32(float* p, float v)
@@ -170,45 +147,6 @@ __device__ __forceinline__ void shifted(uint32_t cw, const float2 (&a)[2], int d
     }
     r[0] = make_float2(q[0], q[1]);
     r[1] = make_float2(q[2], q[3]);
-}
-
-// this thread's VPT adjacent A records (apos) from a stage: code words + dequantised values as
-// channel pairs, and (VPT 2, 4) the band offsets packed in one word
-template <int VPT, bool U8>
-__device__ __forceinline__ void load_records(const unsigned char* stg, int off_in_stage, int tp,
-                                             uint32_t (&cw)[VPT], float2 (&f)[VPT][2], uint32_t& ob)
-{
-    if (U8) {
-        if (VPT == 4) {
-            const uint4 c4 = ((const uint4*)stg)[tp];
-            cw[0] = c4.x;
-            cw[VPT > 1 ? 1 : 0] = c4.y;
-            cw[VPT > 2 ? 2 : 0] = c4.z;
-            cw[VPT > 3 ? 3 : 0] = c4.w;
-        } else if (VPT == 2) {
-            const uint2 c2 = ((const uint2*)stg)[tp];
-            cw[0] = c2.x;
-            cw[VPT > 1 ? 1 : 0] = c2.y;
-        } else {
-#pragma unroll
-            for (int t = 0; t < VPT; ++t) cw[t] = ((const uint32_t*)stg)[tp * VPT + t];
-        }
-#pragma unroll
-        for (int t = 0; t < VPT; ++t) {
-            f[t][0] = dq2(cw[t], 0);
-            f[t][1] = dq2(cw[t], 2);
-        }
-    } else {
-#pragma unroll
-        for (int t = 0; t < VPT; ++t) {
-            const float4 v = ((const float4*)stg)[tp * VPT + t];
-            f[t][0] = make_float2(v.x, v.y);
-            f[t][1] = make_float2(v.z, v.w);
-            cw[t] = 0u;
-        }
-    }
-    if (VPT == 4) ob = ((const uint32_t*)(stg + off_in_stage))[tp];
-    if (VPT == 2) ob = ((const uint16_t*)(stg + off_in_stage))[tp];
 }
 
 // this thread's VPT adjacent records (apos) from a stage as raw words (CW = 1: a uint8 code word
@@ -305,7 +243,7 @@ __device__ __forceinline__ void prior_pair(const int* tof, int i0, int nact, con
     }
 }
 
-// ---- TMA (cp.async.bulk) + mbarrier helpers for the A-record ring ----
+// ---- mbarrier, cp.async and L2-prefetch helpers ----
 __device__ __forceinline__ uint32_t smem_u32(const void* p)
 {
     return (uint32_t)__cvta_generic_to_shared(p);
@@ -314,24 +252,9 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count)
 {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes)
-{
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar)
 {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
-{
-    asm volatile(
-        "{\n\t.reg .pred p;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
-        "r"(parity)
-        : "memory");
 }
 // per-thread asynchronous global -> shared copies (LDGSTS), tracked per thread by commit groups
 __device__ __forceinline__ void cp_async16(void* dst, const void* src)
@@ -356,14 +279,6 @@ __device__ __forceinline__ void cp_async_wait()
 __device__ __forceinline__ void l2_prefetch_bulk(const void* src, uint32_t bytes)
 {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar)
-{
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-            smem_u32(dst)),
-        "l"(src), "r"(bytes), "r"(smem_u32(bar))
-        : "memory");
 }
 
 // ---- thread-block-cluster helpers (CL = 2: the two CTAs of a cluster split an SV's views) ----
