@@ -431,3 +431,17 @@ def test_fbp_reproduces_uniform_disk():
     sel = x2 > 0.5 * mu
     assert abs(X[sel].mean() - 30.0) < 1.0 and abs(Y[sel].mean() + 20.0) < 1.0
     assert abs(sel.sum() * 4.0 / (math.pi * 12.0 * 8.0) - 1) < 0.15  # the ellipse's area
+
+
+def test_sweep_configs_grid():
+    """BASELINE configs[4]: 200 distinct seeded cases over the documented axes, M = 2N (paper
+    ratio, dc = dxy/2), SV sides the update kernel supports at that pitch, deterministic."""
+    from synth import sweep_configs
+    a, b = sweep_configs(), sweep_configs()
+    assert len(a) == 200 and [(c.name, i) for c, i in a] == [(c.name, i) for c, i in b]
+    keys = {(c.phantom, i, c.lambda0, c.nviews, c.sv_side, c.n) for c, i in a}
+    assert len(keys) == 200
+    for c, _ in a:
+        assert c.nchannels == 2 * c.n and abs(c.dchannel - c.dxy / 2) < 1e-12
+        assert c.sv_side in (5, 7, 9) and c.nviews in (90, 180, 360, 720) and c.lambda0 in (1e3, 1e4, 1e5)
+    assert {c.phantom for c, _ in a} == {"shepp_logan", "baggage"}
