@@ -282,9 +282,12 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         // SVs updated concurrently fit the same residual along shared rays; with ~148 of them in
         // one 2-D slice the first sweeps from x0 = 0 overshoot, clip whole SVs to 0 and zero-skip
         // then freezes them (reading R22).
+        // A ray crosses ~sqrt(G) SVs of a colour group of G, so with C of them in flight per slice
+        // it meets ~C / sqrt(G) concurrently updated SVs; the cap keeps that near kAutoRayLoad.
         const int slices_in_phase = std::max(1, h->g.nz_local / parities);
-        const bool auto_batch = !det && h->o.batch_svs == 0 && target_ctas > kAutoBatch * slices_in_phase;
-        const int B = auto_batch ? kAutoBatch : (det || h->o.batch_svs <= 0) ? h->max_group : h->o.batch_svs;
+        const int ray_cap = std::max(8, (int)(kAutoRayLoad * std::sqrt(0.25 * h->nsv)));
+        const bool auto_batch = !det && h->o.batch_svs == 0 && target_ctas > ray_cap * slices_in_phase;
+        const int B = auto_batch ? ray_cap : (det || h->o.batch_svs <= 0) ? h->max_group : h->o.batch_svs;
         const int thr = (det || h->o.batch_svs <= 0) ? 0 : (h->o.batch_threshold >= 0 ? h->o.batch_threshold : B / 4);
         const int nb = (h->max_group + B - 1) / B;
         CK(launch_flatten(h->d_task_list, h->d_task_count, h->g.nz_local, h->g.z_offset, parities,
