@@ -265,7 +265,8 @@ def main():
     ksec = sum(s["kernel_seconds"] for s in stats)
     klaunch = sum(s["kernel_launches"] for s in stats)
     local_updates = updates / world
-    local_visits = sum(s["sv_visits"] for s in stats) / world
+    # SV-buffer traffic only for visits that updated something (fully zero-skipped ones move none)
+    local_visits = sum(s["sv_visits"] - s["sv_visits_empty"] for s in stats) / world
     bytes_per_update = nnz_avg * 1 + cfg.nviews * 1 + 4  # u8 codes of the nnz, offsets, scale
     alg_bytes = local_updates * bytes_per_update + local_visits * 16 * band_avg
     achieved = alg_bytes / ksec / 1e9

@@ -124,6 +124,8 @@ typedef struct mbir_stats {
     double kernel_seconds; /* summed device time of the fused update-kernel launches,
                               CUDA events on the handle's stream around each launch     */
     int64_t kernel_launches; /* fused update-kernel launches                           */
+    int64_t sv_visits_empty; /* of sv_visits: tasks whose every voxel was zero-skipped (no
+                                SV-buffer traffic; reading R9)                           */
 } mbir_stats;
 
 /* Sizes of the internal layout (for tests, benchmarks and buffer allocation). */

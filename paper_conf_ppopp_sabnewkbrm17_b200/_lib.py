@@ -65,7 +65,7 @@ class mbir_stats(C.Structure):
         ("updates", C.c_int64), ("skipped", C.c_int64), ("sv_visits", C.c_int64),
         ("iterations", C.c_int64), ("equits", C.c_double), ("seconds", C.c_double),
         ("sum_abs_delta", C.c_double), ("launches", C.c_int64),
-        ("kernel_seconds", C.c_double), ("kernel_launches", C.c_int64),
+        ("kernel_seconds", C.c_double), ("kernel_launches", C.c_int64), ("sv_visits_empty", C.c_int64),
     ]
 
     def as_dict(self):

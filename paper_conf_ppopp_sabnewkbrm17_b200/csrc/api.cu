@@ -90,11 +90,12 @@ struct mbir_handle {
     static constexpr int kNPerm = 64;
     int *d_task_list = nullptr, *d_task_count = nullptr;
     int *d_flat = nullptr, *d_brange = nullptr, *d_fetch = nullptr;
-    unsigned long long* d_counters = nullptr;  // [updates, skipped, visits]
+    int* d_keep = nullptr;  // zero-skip pre-filter flags of the current phase list
+    unsigned long long* d_counters = nullptr;  // [updates, skipped, visits, empty visits]
     double* d_sum_delta = nullptr;
     int* d_flag = nullptr;
     double* d_acc = nullptr;
-    unsigned long long* h_counters = nullptr;  // pinned [4] (3 counters + sum_delta bits)
+    unsigned long long* h_counters = nullptr;  // pinned [5] (4 counters + sum_delta bits)
     bool have_sino = false;
     bool x_zero = true;  // the image is known to be all zero (then e = y needs no projection)
     int iter = 0;
@@ -236,7 +237,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
     const int nnb = h->pr.neighborhood;
     const int parities = (nnb == 26 && h->g.nz_total > 1) ? 2 : 1;
     const int target_ctas = h->nsm * h->blocks_per_sm;
-    int64_t updates = 0, skipped = 0, visits = 0, iters = 0, launches = 0, klaunches = 0;
+    int64_t updates = 0, skipped = 0, visits = 0, empty = 0, iters = 0, launches = 0, klaunches = 0;
     double ksec = 0.0;
     double sum_delta = 0.0;
     CK(cudaEventRecord(h->ev0, h->st));
@@ -246,7 +247,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         h->iter += 1;
         h->x_zero = false;
         h->kev_used = 0;
-        CK(cudaMemsetAsync(h->d_counters, 0, 3 * sizeof(unsigned long long), h->st));
+        CK(cudaMemsetAsync(h->d_counters, 0, 4 * sizeof(unsigned long long), h->st));
         CK(cudaMemsetAsync(h->d_sum_delta, 0, sizeof(double), h->st));
         // ---- SV selection (Alg3:17-23)
         SchedParams sp{};
@@ -300,10 +301,21 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         // deterministic: one CTA (or one cluster) walks the phase list in order (sequential ICD,
         // known order)
         const int grid = det ? h->cl : target_ctas;
+        // iterations >= 2 without batching: the tasks whose whole tile is zero are flagged per
+        // phase (sched.cu k_zero_flags) and skipped at task fetch by the update kernel
+        const bool prefilter = p.zero_skip_active && nb == 1 && !det && !(p.dbg & 4);
         for (int zp = 0; zp < parities; ++zp) {
             for (int colour = 0; colour < 4; ++colour) {
                 const int ph = zp * 4 + colour;
                 p.flat = h->d_flat + ph * cap;
+                p.keep = nullptr;
+                if (prefilter) {
+                    CK(launch_zero_flags(h->d_flat + ph * cap, h->d_brange + ph * (nb + 1), h->d_x, h->g.nx,
+                                         h->g.ny, h->g.nz_local, h->g.z_offset, h->g.nz_total, h->side, h->nsvx,
+                                         nnb, (int)cap, h->d_keep, h->st));
+                    ++launches;
+                    p.keep = h->d_keep;
+                }
                 for (int b = 0; b < nb; ++b) {
                     p.brange = h->d_brange + ph * (nb + 1) + b;
                     p.fetch = h->d_fetch + ph * nb + b;
@@ -318,12 +330,12 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
             }
         }
         if (h->nranks > 1) {
-            CKN(nccl().AllReduce(h->d_counters, h->d_counters, 3, ncclUint64, ncclSum, h->comm, h->st));
+            CKN(nccl().AllReduce(h->d_counters, h->d_counters, 4, ncclUint64, ncclSum, h->comm, h->st));
             CKN(nccl().AllReduce(h->d_sum_delta, h->d_sum_delta, 1, ncclFloat64, ncclSum, h->comm, h->st));
         }
-        CK(cudaMemcpyAsync(h->h_counters, h->d_counters, 3 * sizeof(unsigned long long),
+        CK(cudaMemcpyAsync(h->h_counters, h->d_counters, 4 * sizeof(unsigned long long),
                            cudaMemcpyDeviceToHost, h->st));
-        CK(cudaMemcpyAsync(h->h_counters + 3, h->d_sum_delta, sizeof(double), cudaMemcpyDeviceToHost,
+        CK(cudaMemcpyAsync(h->h_counters + 4, h->d_sum_delta, sizeof(double), cudaMemcpyDeviceToHost,
                            h->st));
         CK(cudaStreamSynchronize(h->st));
         for (int i = 0; i < h->kev_used; ++i) {
@@ -335,8 +347,9 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         updates += (int64_t)h->h_counters[0];
         skipped += (int64_t)h->h_counters[1];
         visits += (int64_t)h->h_counters[2];
+        empty += (int64_t)h->h_counters[3];
         double sd;
-        memcpy(&sd, h->h_counters + 3, sizeof(double));
+        memcpy(&sd, h->h_counters + 4, sizeof(double));
         if (!isfinite(sd)) return fail(h, MBIR_ENUMERIC, "non-finite update amount");
         sum_delta += sd;
         ++iters;
@@ -353,6 +366,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         st->updates = updates;
         st->skipped = skipped;
         st->sv_visits = visits;
+        st->sv_visits_empty = empty;
         st->iterations = iters;
         st->equits = (double)updates / nvox_total;
         st->seconds = ms * 1e-3;
@@ -481,7 +495,7 @@ void mbir_destroy(mbir_handle* h)
     void* ptrs[] = {h->A.codes, h->A.vals, h->A.off, h->A.count, h->A.scale, h->A.band_start,
                     h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
                     h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count,
-                    h->d_flat, h->d_brange, h->d_fetch, h->d_perm, h->d_counters, h->d_sum_delta,
+                    h->d_flat, h->d_brange, h->d_fetch, h->d_keep, h->d_perm, h->d_counters, h->d_sum_delta,
                     h->d_flag, h->d_acc, h->d_tprof, h->d_trace};
     if (h->d_trace && getenv("MBIR_TRACE")) {  // development aid: raw clock stamps (tools/trace_visit.py)
         std::vector<unsigned long long> t(1024);
@@ -680,6 +694,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_task_count, (size_t)G.nz_local * 4))) return bail(r);
     if ((r = dalloc(h, &h->d_flat, (size_t)8 * G.nz_local * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_brange, (size_t)8 * (h->max_group + 1)))) return bail(r);
+    if ((r = dalloc(h, &h->d_keep, (size_t)G.nz_local * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_fetch, (size_t)8 * h->max_group))) return bail(r);
     {
         // random voxel visiting orders within an SV ("randomized order"; reading R10):
@@ -700,7 +715,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         if ((r = dalloc(h, &h->d_perm, perm.size()))) return bail(r);
         if (cudaMemcpy(h->d_perm, perm.data(), perm.size(), cudaMemcpyHostToDevice) != cudaSuccess) return bail(MBIR_ECUDA);
     }
-    if ((r = dalloc(h, &h->d_counters, 3))) return bail(r);
+    if ((r = dalloc(h, &h->d_counters, 4))) return bail(r);
     if ((r = dalloc(h, &h->d_sum_delta, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_flag, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_acc, 1))) return bail(r);
@@ -712,7 +727,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         if ((r = dalloc(h, &h->d_tprof, 32))) return bail(r);
         cudaMemset(h->d_tprof, 0, 32 * sizeof(unsigned long long));
     }
-    if (cudaMallocHost((void**)&h->h_counters, 4 * sizeof(unsigned long long)) != cudaSuccess) return bail(MBIR_ENOMEM);
+    if (cudaMallocHost((void**)&h->h_counters, 5 * sizeof(unsigned long long)) != cudaSuccess) return bail(MBIR_ENOMEM);
     cudaMemsetAsync(h->d_x, 0, sizeof(float) * pl * (G.nz_local + 2), h->st);
     cudaMemsetAsync(h->d_amount, 0, sizeof(float) * G.nz_local * h->nsv, h->st);
     if (cudaEventCreate(&h->ev0) != cudaSuccess || cudaEventCreate(&h->ev1) != cudaSuccess) return bail(MBIR_ECUDA);

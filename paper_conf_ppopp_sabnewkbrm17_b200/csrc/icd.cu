@@ -493,7 +493,23 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
         if (CL == 2) st_peer_u32(peer_addr(s_task + i, 1), (uint32_t)v);
     };
     if (CL == 2) cluster_sync_all();  // peer smem (mbarriers, red) initialised before any remote access
-    if (threadIdx.x == 0 && crank == 0) publish_task(0, tstart + atomicAdd(P.fetch, 1));
+    // the next task of the launch's list; with the zero-skip pre-filter (P.keep), tasks whose
+    // whole tile is zero are accounted as skipped visits here and never reach a CTA's pipeline
+    auto fetch_task = [&]() {
+        int q = tstart + atomicAdd(P.fetch, 1);
+        while (P.keep && q < tend && !P.keep[q]) {
+            const int tkq = P.flat[q];
+            const int zq = tkq >> 14, svq = tkq & 16383;
+            const int twq = min(side, P.nx - (svq % P.nsvx) * side), thq = min(side, P.ny - (svq / P.nsvx) * side);
+            P.sv_amount[(size_t)zq * P.nsv + svq] = 0.f;
+            atomicAdd(P.counters + 1, (unsigned long long)(twq * thq));
+            atomicAdd(P.counters + 2, 1ull);
+            atomicAdd(P.counters + 3, 1ull);
+            q = tstart + atomicAdd(P.fetch, 1);
+        }
+        return q;
+    };
+    if (threadIdx.x == 0 && crank == 0) publish_task(0, fetch_task());
     if (CL == 2) cluster_sync_all(); else __syncthreads();
     int q = s_task[0];
     if (q < tend) band_info(P, P.flat[q], binfo, vbase, VL, threadIdx.x, blockDim.x);
@@ -571,7 +587,8 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
                 atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
                 atomicAdd(P.counters + 2, 1ull);
-                publish_task(nslot, tstart + atomicAdd(P.fetch, 1));
+                atomicAdd(P.counters + 3, 1ull);
+                publish_task(nslot, fetch_task());
             }
             if (CL == 2) cluster_sync_all(); else __syncthreads();
             if (s_task[nslot] < tend)
@@ -657,7 +674,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 // CL = 2 hands it to rank 1 through DSMEM + an mbarrier arrival)
                 for (int i = R; i < 2 * R && i < nact; ++i) prefetch_record(i);
                 if (crank == 0) {
-                    publish_task(nslot, tstart + atomicAdd(P.fetch, 1));
+                    publish_task(nslot, fetch_task());
                     if (CL == 2) mbar_arrive_peer(peer_addr(taskbar, 1));
                 }
             }

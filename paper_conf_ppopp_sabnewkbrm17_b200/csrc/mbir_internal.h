@@ -82,6 +82,7 @@ struct IcdParams {
     const int* flat;         // phase task list, entries (local slice << 14) | SV
     const int* brange;       // [2]: this launch's batch = flat[brange[0] .. brange[1])
     int* fetch;              // task counter of this launch (zeroed per iteration)
+    const int* keep;         // optional [list]: 0 = the task's whole tile is zero (zero-skip pre-filter)
     unsigned long long* counters;  // [0] updates [1] skipped [2] sv visits
     double* sum_delta;
     uint64_t seed;
@@ -132,6 +133,10 @@ cudaError_t launch_flatten(const int* task_list, const int* task_count, int nz_l
 // FBP initial image (fbp.cu): q = ramp-filtered y (scratch [nz][V][M]), x = clip(backprojection)
 cudaError_t launch_fbp(const mbir_geometry& g, const double* d_cs, const float* y, float* q, float* x,
                        int positivity, cudaStream_t st);
+// zero-skip pre-filter of a phase list (sched.cu): keep[t] = 0 iff task t's whole tile is zero
+cudaError_t launch_zero_flags(const int* flat, const int* brange, const float* x, int nx, int ny,
+                              int nz_local, int z_offset, int nz_total, int side, int nsvx, int nnb,
+                              int max_tasks, int* keep, cudaStream_t st);
 cudaError_t launch_rmse_partial(const float* x, const float* g, int64_t n, double* acc,
                                 cudaStream_t st);
 cudaError_t launch_check_finite(const float* a, int64_t n, int nonneg, int* flag, cudaStream_t st);

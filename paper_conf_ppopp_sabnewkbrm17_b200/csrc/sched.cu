@@ -161,6 +161,36 @@ __global__ void k_flatten(const int* __restrict__ task_list, const int* __restri
     }
 }
 
+// Zero-skip pre-filter of one phase's task list (iterations >= 2, no batching).  An SV visit is
+// fully skipped (reading R9) iff every in-volume x of its tile -- the SV, its 1-voxel ring
+// and, with the 26-neighbourhood, the slices z +- 1 -- is 0.  During a phase only SVs of its colour
+// (and z parity) change and none of them is in another's tile, so the phase-start answer equals
+// the visit-start one.  The update kernel's task fetch then accounts flagged tasks exactly as a
+// skipped visit (k_icd_sv fetch_task) without loading their tiles.  A warp per task (grid-stride).
+__global__ void k_zero_flags(const int* __restrict__ flat, const int* __restrict__ brange,
+                             const float* __restrict__ x, int nx, int ny, int nz_local, int z_offset,
+                             int nz_total, int side, int nsvx, int nnb, int* __restrict__ keep)
+{
+    const int lane = threadIdx.x & 31;
+    const int nwarps = gridDim.x * (blockDim.x >> 5), n = brange[1];
+    for (int t = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); t < n; t += nwarps) {
+    const int tk = flat[t];
+    const int z = tk >> 14, sv = tk & 16383;
+    const int gx0 = (sv % nsvx) * side - 1, gy0 = (sv / nsvx) * side - 1;
+    const int TW = side + 2, nzt = nnb == 26 ? 3 : 1;
+    const size_t plane = (size_t)nx * ny;
+    bool nz = false;
+    for (int i = lane; i < nzt * TW * TW && !nz; i += 32) {
+        const int tz = nzt == 3 ? i / (TW * TW) - 1 : 0, r = i % (TW * TW);
+        const int gx = gx0 + r % TW, gy = gy0 + r / TW, gz = z_offset + z + tz;
+        if (gx < 0 || gx >= nx || gy < 0 || gy >= ny || gz < 0 || gz >= nz_total) continue;
+        nz = x[(size_t)(z + 1 + tz) * plane + (size_t)gy * nx + gx] != 0.f;
+    }
+    nz = __any_sync(0xffffffffu, nz);
+    if (lane == 0) keep[t] = nz ? 1 : 0;
+    }
+}
+
 __global__ void k_rmse(const float* __restrict__ x, const float* __restrict__ g, int64_t n,
                        double* acc)
 {
@@ -202,6 +232,16 @@ cudaError_t launch_flatten(const int* task_list, const int* task_count, int nz_l
 {
     k_flatten<<<parities * 4, 256, 0, st>>>(task_list, task_count, nz_local, z_offset, parities,
                                             max_group, batch, thr, nb, flat, brange);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_zero_flags(const int* flat, const int* brange, const float* x, int nx, int ny,
+                              int nz_local, int z_offset, int nz_total, int side, int nsvx, int nnb,
+                              int max_tasks, int* keep, cudaStream_t st)
+{
+    if (max_tasks <= 0) return cudaSuccess;
+    k_zero_flags<<<min((max_tasks + 7) / 8, 296), 256, 0, st>>>(flat, brange, x, nx, ny, nz_local, z_offset,
+                                                                nz_total, side, nsvx, nnb, keep);
     return cudaGetLastError();
 }
 
