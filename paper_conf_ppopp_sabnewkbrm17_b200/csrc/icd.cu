@@ -1188,7 +1188,7 @@ template <bool U8>
 __global__ void k_theta2(const IcdParams P)
 {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const int sv = blockIdx.x, z = blockIdx.y;
+    const int z = blockIdx.x, sv = blockIdx.y;
     const float* wz = P.w + (size_t)z * P.V * P.M;
     const int vpt = P.A.vpt;
     for (int slot = warp; slot < P.S2; slot += nw) {
@@ -1461,7 +1461,7 @@ cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int 
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st)
 {
     auto k = quantize ? k_theta2<true> : k_theta2<false>;
-    k<<<dim3(p.nsv, p.nz_local), 512, 0, st>>>(p);
+    k<<<dim3(p.nz_local, p.nsv), 512, 0, st>>>(p);  // slices of one SV adjacent: A from L2
     return cudaGetLastError();
 }
 
