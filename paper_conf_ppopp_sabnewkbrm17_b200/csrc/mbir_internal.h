@@ -17,7 +17,7 @@ constexpr int kMaxNbr = 26;       // 3-D neighbourhood (reading R2)
 constexpr int kRingDepth = 4;     // A-record prefetch depth (voxels) in the update kernel
 constexpr int kMaxSvbRows = 32;   // SV-buffer rows held by one 32-lane transpose tile
 constexpr int kMaxThreads = 1024;
-constexpr double kAutoRayLoad = 2.5;  // batch_svs = 0: concurrently updated SVs one ray meets (R22)
+constexpr double kAutoRayLoad = 1.5;  // batch_svs = 0: concurrently updated SVs one ray meets (R22)
 
 // ---- prior constants in __constant__ memory (set by set_prior_constants) ----
 struct PriorConst {
