@@ -487,3 +487,36 @@ def test_2d_slice_with_many_svs_does_not_collapse():
     # both runs zero-skip, whose fixed point is order-dependent (reading R9; 5.9 HU measured at
     # this low dose): within the paper's own convergence criterion, 10 HU
     assert O.rmse_hu(xg, x) < 10.0, O.rmse_hu(xg, x)
+
+
+def test_zero_skip_prefilter_path_matches_oracle():
+    """Iterations >= 2 without batching flag fully zero-skipped SV visits per phase and account
+    them at task fetch (api.cu / sched.cu k_zero_flags).  A whole-group batch on a 3-D baggage case
+    (large air fraction) exercises it: empty visits are reported, the accounting stays consistent
+    and the converged image matches the oracle's zero-skip run (reading R9 bound)."""
+    cfg = WorkloadConfig("mini3d-bag", 40, 4, 60, 64, 7, 26, 0.002, phantom="baggage")
+    case = make_case(cfg, 101)
+    g, og = geoms(cfg)
+    _, _, Aq = O.quantize(O.sysmatrix(og))
+    pr = O.Prior(sigma=cfg.sigma, nbhd=26)
+    x = np.zeros(cfg.nz * cfg.n * cfg.n)
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+    O.icd_run(og, pr, Aq, case.w, x, e, 120, seed=3000, zero_skip=True)
+    nvox = cfg.nz * cfg.n * cfg.n
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
+                         M.Options(sv_side=cfg.sv_side, batch_svs=1000, batch_threshold=0)) as r:
+        r.set_sinogram(case.y, case.w)
+        st1 = r.iterate(1)
+        assert st1["updates"] == nvox and st1["sv_visits_empty"] == 0  # no skipping in iteration 1
+        empty = 0
+        for _ in range(30):
+            st = r.iterate(1)
+            assert st["sv_visits_empty"] <= st["sv_visits"]
+            empty += st["sv_visits_empty"]
+        assert empty > 0
+        r.reconstruct(200)
+        xg = r.image().ravel().astype(np.float64)
+    assert O.rmse_hu(xg, x) < 2.0, O.rmse_hu(xg, x)
+    cg = O.cost(og, pr, Aq, case.y, case.w, xg)
+    co = O.cost(og, pr, Aq, case.y, case.w, x)
+    assert abs(cg - co) <= 5e-4 * abs(co)
