@@ -91,8 +91,10 @@ struct IcdParams {
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
     unsigned long long* trace;  // optional per-pair clock trace of one SV visit (env MBIR_TRACE)
-    int dbg;                 // development switches (env MBIR_DBG): bit 0 no A-record L2 warm-up,
-                             // bit 1 no band-row L2 warm-up
+    int dbg;                 // development switches (env MBIR_DBG): bit 0 A-record L2 warm-up on,
+                             // bit 1 band-row L2 warm-up off, bit 2 zero-skip pre-filter off;
+                             // timing ablations with wrong results: bit 4 no scatter, bit 5 no
+                             // prior terms, bit 7 no e_init store
     SmemLayout lay;          // update-kernel smem layout (filled by launch_icd)
 };
 
