@@ -1195,10 +1195,10 @@ __global__ void k_theta2(const IcdParams P)
         const size_t ab = ((size_t)sv * P.S2 + slot) * P.A.VA;
         const float sc = P.A.scale[(size_t)sv * P.S2 + slot];
         float acc = 0.f;
-        for (int pk = lane; pk < P.A.VA; pk += 32) {  // record positions, coalesced
+#pragma unroll 4
+        for (int pk = lane; pk < P.A.VA; pk += 32) {  // record positions, coalesced (4 in flight)
             const int qq = pk / vpt, t = pk % vpt;     // inverse of apos()
-            const int k = ((qq >> 5) * vpt + t) * 32 + (qq & 31);
-            if (k >= P.V) continue;
+            const int k = min(((qq >> 5) * vpt + t) * 32 + (qq & 31), P.V - 1);  // padded: count 0
             const int n = P.A.count[ab + pk];
             const int o = P.A.band_start[(size_t)sv * P.V + k] + P.A.off[ab + pk];
             float a[4];
