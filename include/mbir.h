@@ -97,10 +97,19 @@ typedef struct mbir_options {
                               1 = one CTA owns a task; 2 = a 2-CTA thread-block cluster splits
                               the task's views (two tasks per SM; EINVAL where not possible).
                               The arithmetic is the same either way.                             */
+    int zero_skip_period;  /* with zero_skip: iterations 1 + k*zero_skip_period, k >= 1 (numbers
+                              counted from the last set_sinogram / set_image) run
+                              WITHOUT zero-skipping on a random sv_fraction of the SVs, so voxels
+                              frozen at 0 are re-examined and the fixed point stays the MAP
+                              estimate; 0 = the plain heuristic of P:115, whose fixed point can
+                              differ from the MAP (reading R9).  Default 4                      */
 } mbir_options;
 
 /* Placement and (optional) multi-GPU slab partition.  device: CUDA ordinal.  stream: a
- * cudaStream_t (NULL = the library creates its own).  For nranks > 1, nccl_unique_id points to
+ * cudaStream_t on which every call orders its device work (NULL = the library creates its own
+ * blocking stream, implicitly ordered with the legacy default stream).  Device buffers passed
+ * to any call must be complete with respect to that stream (pass the stream that produced
+ * them; the Python binding passes torch's current stream).  For nranks > 1, nccl_unique_id points to
  * the 128-byte ncclUniqueId produced by mbir_nccl_unique_id() on rank 0 and broadcast by the
  * caller (e.g. over a torch.distributed process group); rank r must own slices
  * [z_offset, z_offset + nz_local) with slabs contiguous in rank order. */
@@ -141,10 +150,11 @@ typedef struct mbir_sizes {
     int64_t nnz;                    /* total non-zeros of the slice-plane system matrix    */
     int64_t a_bytes;                /* device bytes of the compressed A                   */
     int64_t band_entries;           /* sum over (SV, view) of band widths                  */
+    int max_group;                  /* SVs of one checkerboard colour per slice (max)     */
 } mbir_sizes;
 
 /* Fill defaults: sv_side 9, sv_fraction 0.25, batch_svs 0, batch_threshold -1, zero_skip 1,
- * quantize_A 1, seed 3000, deterministic 0, cluster 0 (auto). */
+ * quantize_A 1, seed 3000, deterministic 0, cluster 0 (auto), zero_skip_period 4. */
 void mbir_default_options(mbir_options* o);
 /* p 1.2, q 2, T 1, sigma 0.005, neighborhood 26, positivity 1. */
 void mbir_default_prior(mbir_prior* p);
@@ -215,6 +225,28 @@ int mbir_get_sysmatrix_columns(mbir_handle* h, const int64_t* voxels, int n, int
  * floats, computed on the device from the library's A representation, e, w and x. */
 int mbir_probe_update(mbir_handle* h, const int64_t* voxels, int n, float* theta1,
                       float* theta2, float* delta);
+
+/* Test hook: record every voxel update the fused update kernel executes from now on -- the
+ * (theta1, theta2, delta) of Alg. 1 steps 3-8 exactly as the kernel's delta chain
+ * used them (theta1 of the second voxel of a pair includes the first one's update of e, so it
+ * equals sequential ICD's theta1 at that update).  capacity = entries kept (0 = off; frees the
+ * buffer).  Pairs are recorded first voxel first; in deterministic mode (one CTA) the record
+ * is the exact update sequence.  Errors: EINVAL, ENOMEM. */
+int mbir_set_update_dump(mbir_handle* h, int64_t capacity);
+
+/* Copy up to cap recorded updates into host arrays (voxels: local flat (z*ny + y)*nx + x;
+ * theta1, theta2, delta float32), set *n to the number recorded since the last call (which
+ * can exceed cap and the capacity: then the record was truncated), and restart the record.
+ * Errors: EINVAL, ESTATE (no dump buffer), ECUDA. */
+int mbir_get_update_dump(mbir_handle* h, int64_t cap, int64_t* voxels, float* theta1,
+                         float* theta2, float* delta, int64_t* n);
+
+/* Test hook (scheduler, P:203-225 / Alg3:17-23): copy the SV selection of the most recent
+ * iteration and the update amounts (host buffers, each may be NULL).  task_list int32
+ * [nz_local][4 colours][max_group] (SV indices of the colour group in selection order; entries
+ * past task_count are stale), task_count int32 [nz_local][4], amount float32 [nz_local][nsv]
+ * (sum |delta| of each SV's most recent visit, the key of the next "top" selection). */
+int mbir_get_schedule(mbir_handle* h, int32_t* task_list, int32_t* task_count, float* amount);
 
 /* Multi-GPU bootstrap: write a fresh 128-byte ncclUniqueId into id (call on rank 0 only).
  * Returns ENOTSUP if libnccl.so.2 cannot be loaded. */

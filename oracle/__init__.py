@@ -81,8 +81,11 @@ def lib():
                                        C.c_int, dp, dp, dp]
         L.orc_icd_run.restype = C.c_int64
         L.orc_icd_run.argtypes = [G, P, C.c_int, ip, ip, dp, dp, dp, dp, C.c_int, C.c_int,
-                                  C.c_uint64, C.c_int, lp, C.c_int64, dp, C.c_int64,
+                                  C.c_uint64, C.c_int, C.c_int, lp, C.c_int64, dp, C.c_int64,
                                   C.POINTER(_Stats)]
+        L.orc_icd_run_zpar.restype = C.c_int
+        L.orc_icd_run_zpar.argtypes = [G, P, C.c_int, ip, ip, dp, dp, dp, dp, C.c_int, C.c_int,
+                                       C.c_uint64, C.c_int, C.c_int, C.c_int, C.POINTER(_Stats)]
         L.orc_error_sinogram.restype = None
         L.orc_error_sinogram.argtypes = [G, C.c_int, ip, ip, dp, dp, dp, dp]
         L.orc_cost.restype = C.c_double
@@ -241,9 +244,10 @@ def voxel_update(g: Geometry, pr: Prior, A: SysMatrix, w, x, e, j: int, apply: b
 
 
 def icd_run(g: Geometry, pr: Prior, A: SysMatrix, w, x, e, n_equits: int, *, first_sweep=1,
-            seed=3000, zero_skip=True, order=None, dump=0):
+            seed=3000, zero_skip=True, zero_skip_period=0, order=None, dump=0):
     """Sequential ICD.  x, e (float64, contiguous) updated in place.
-    Returns (stats dict, dump array [n,4] of (j, theta1, theta2, delta))."""
+    zero_skip_period > 0: sweeps numbered by a multiple of it run without zero-skipping
+    (reading R9).  Returns (stats dict, dump array [n,4] of (j, theta1, theta2, delta))."""
     assert x.dtype == np.float64 and x.flags.c_contiguous
     assert e.dtype == np.float64 and e.flags.c_contiguous
     w = np.ascontiguousarray(w, np.float64)
@@ -256,7 +260,7 @@ def icd_run(g: Geometry, pr: Prior, A: SysMatrix, w, x, e, n_equits: int, *, fir
     n = lib().orc_icd_run(C.byref(gc), C.byref(pc), A.K, _p(A.first, C.c_int32),
                           _p(A.count, C.c_int32), _p(A.vals, C.c_double), _p(w, C.c_double),
                           _p(x, C.c_double), _p(e, C.c_double), n_equits, first_sweep,
-                          C.c_uint64(seed), int(zero_skip),
+                          C.c_uint64(seed), int(zero_skip), int(zero_skip_period),
                           _p(order_arr, C.c_int64) if order_arr is not None else None,
                           len(order_arr) if order_arr is not None else 0,
                           _p(dbuf, C.c_double) if dump else None, dump, C.byref(st))
@@ -264,6 +268,27 @@ def icd_run(g: Geometry, pr: Prior, A: SysMatrix, w, x, e, n_equits: int, *, fir
         raise MemoryError("oracle icd_run")
     return ({"updates": st.updates, "skipped": st.skipped, "sum_abs_delta": st.sum_abs_delta},
             dbuf[:n] if dump else None)
+
+
+def icd_run_zpar(g: Geometry, pr: Prior, A: SysMatrix, w, x, e, n_equits: int, *, first_sweep=1,
+                 seed=3000, zero_skip=False, zero_skip_period=0, threads=None):
+    """Sequential ICD with the slices of one z-parity on several host threads (an exact
+    serialisation, see oracle.h orc_icd_run_zpar).  x, e updated in place.  Returns stats."""
+    assert x.dtype == np.float64 and x.flags.c_contiguous
+    assert e.dtype == np.float64 and e.flags.c_contiguous
+    w = np.ascontiguousarray(w, np.float64)
+    st = _Stats()
+    gc, pc = g.c(), pr.c()
+    nt = threads or (os.cpu_count() or 1)
+    r = lib().orc_icd_run_zpar(C.byref(gc), C.byref(pc), A.K, _p(A.first, C.c_int32),
+                               _p(A.count, C.c_int32), _p(A.vals, C.c_double), _p(w, C.c_double),
+                               _p(x, C.c_double), _p(e, C.c_double), n_equits, first_sweep,
+                               C.c_uint64(seed), int(zero_skip), int(zero_skip_period), nt,
+                               C.byref(st))
+    if r < 0:
+        raise MemoryError("oracle icd_run_zpar")
+    return {"updates": st.updates, "skipped": st.skipped, "sum_abs_delta": st.sum_abs_delta,
+            "threads": nt}
 
 
 def cost(g: Geometry, pr: Prior, A: SysMatrix, y, w, x) -> float:

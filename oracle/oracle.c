@@ -10,6 +10,7 @@
 #include <math.h>
 #include <stdlib.h>
 #include <string.h>
+#include <pthread.h>
 
 #define ORC_PI 3.14159265358979323846
 #define ORC_EPS 1e-9 /* channel-index guard, reading R5 */
@@ -276,10 +277,18 @@ static int all_zero_nbhd(const orc_geom* g, int nbhd, const double* x, int64_t j
     return 1;
 }
 
+/* zero-skip in this 1-based sweep?  P:115 skips from the second sweep on (reading R9); with a
+ * re-admission period P > 0 every P-th sweep runs without skipping, so a voxel frozen at 0 is
+ * re-examined and a fixed point of the iteration is a fixed point of plain ICD (the MAP). */
+static int skip_sweep(int zero_skip, int period, int sweep)
+{
+    return zero_skip && sweep > 1 && !(period > 0 && sweep % period == 0);
+}
+
 int64_t orc_icd_run(const orc_geom* g, const orc_prior* pr, int K,
                     const int32_t* first, const int32_t* count, const double* vals,
                     const double* w, double* x, double* e,
-                    int n_equits, int first_sweep, uint64_t seed, int zero_skip,
+                    int n_equits, int first_sweep, uint64_t seed, int zero_skip, int zero_skip_period,
                     const int64_t* order, int64_t order_len,
                     double* dump, int64_t dump_cap, orc_stats* st)
 {
@@ -314,7 +323,7 @@ int64_t orc_icd_run(const orc_geom* g, const orc_prior* pr, int K,
         }
         for (int64_t q = 0; q < n; ++q) {
             int64_t j = seq[q];
-            if (zero_skip && sweep > 1 && all_zero_nbhd(g, pr->nbhd, x, j)) {
+            if (skip_sweep(zero_skip, zero_skip_period, sweep) && all_zero_nbhd(g, pr->nbhd, x, j)) {
                 if (st) st->skipped++;
                 continue;
             }
@@ -337,6 +346,115 @@ int64_t orc_icd_run(const orc_geom* g, const orc_prior* pr, int K,
     }
     free(perm);
     return ndump;
+}
+
+/* Sequential ICD in slice-parity halves (golden runs of 3-D volumes): per sweep,
+ * for parity 0 then 1, every slice z of that parity runs one pass over its own voxels in a
+ * fresh random order (splitmix64 Fisher-Yates seeded from (seed, sweep, z)).  Slices of one
+ * parity share no sinogram entry (each slice has its own e, parallel beam) and no prior edge
+ * (the 26-neighbourhood links z to z +- 1 only), so running them on several threads at once is
+ * exactly the sequential ICD of their concatenated orders: an exact serialisation, not an
+ * approximation.  POSIX threads pull slices from a shared counter. */
+typedef struct {
+    const orc_geom* g;
+    const orc_prior* pr;
+    int K;
+    const int32_t *first, *count;
+    const double *vals, *w;
+    double *x, *e;
+    uint64_t seed;
+    int sweep, parity, skip;
+    int next; /* next slice index of this parity to take (guarded by the mutex) */
+    pthread_mutex_t mu;
+    int64_t upd, skp;
+    double sad;
+    int fail;
+} zpar_job;
+
+static void zpar_slice(zpar_job* J, int z, int64_t* perm, int64_t* upd, int64_t* skp, double* sad)
+{
+    const orc_geom* g = J->g;
+    const int64_t plane = (int64_t)g->nx * g->ny;
+    uint64_t st64 = J->seed ^ ((uint64_t)J->sweep * 0xD1B54A32D192ED03ULL) ^ ((uint64_t)(z + 1) * 0x9E3779B97F4A7C15ULL);
+    for (int64_t i = 0; i < plane; ++i) perm[i] = i;
+    for (int64_t i = plane - 1; i > 0; --i) {
+        int64_t r = (int64_t)(splitmix64(&st64) % (uint64_t)(i + 1));
+        int64_t t = perm[i];
+        perm[i] = perm[r];
+        perm[r] = t;
+    }
+    for (int64_t q = 0; q < plane; ++q) {
+        const int64_t jj = perm[q], j = (int64_t)z * plane + jj;
+        if (J->skip && all_zero_nbhd(g, J->pr->nbhd, J->x, j)) {
+            (*skp)++;
+            continue;
+        }
+        double dl;
+        orc_voxel_update(g, J->pr, J->K, J->first + jj * g->nviews, J->count + jj * g->nviews,
+                         J->vals + jj * g->nviews * J->K, J->w, J->x, J->e, j, 1, NULL, NULL, &dl);
+        (*upd)++;
+        *sad += fabs(dl);
+    }
+}
+
+static void* zpar_worker(void* arg)
+{
+    zpar_job* J = (zpar_job*)arg;
+    const int64_t plane = (int64_t)J->g->nx * J->g->ny;
+    int64_t* perm = (int64_t*)malloc(sizeof(int64_t) * (size_t)plane);
+    int64_t upd = 0, skp = 0;
+    double sad = 0.0;
+    for (;;) {
+        pthread_mutex_lock(&J->mu);
+        const int z = J->next;
+        J->next += 2;
+        pthread_mutex_unlock(&J->mu);
+        if (z >= J->g->nz || !perm) break;
+        zpar_slice(J, z, perm, &upd, &skp, &sad);
+    }
+    pthread_mutex_lock(&J->mu);
+    J->upd += upd;
+    J->skp += skp;
+    J->sad += sad;
+    if (!perm) J->fail = 1;
+    pthread_mutex_unlock(&J->mu);
+    free(perm);
+    return NULL;
+}
+
+int orc_icd_run_zpar(const orc_geom* g, const orc_prior* pr, int K, const int32_t* first,
+                     const int32_t* count, const double* vals, const double* w, double* x,
+                     double* e, int n_equits, int first_sweep, uint64_t seed, int zero_skip,
+                     int zero_skip_period, int nthreads, orc_stats* st)
+{
+    zpar_job J;
+    memset(&J, 0, sizeof(J));
+    J.g = g; J.pr = pr; J.K = K; J.first = first; J.count = count; J.vals = vals; J.w = w;
+    J.x = x; J.e = e; J.seed = seed;
+    pthread_mutex_init(&J.mu, NULL);
+    if (nthreads < 1) nthreads = 1;
+    if (nthreads > 256) nthreads = 256;
+    pthread_t th[256];
+    for (int s = 0; s < n_equits && !J.fail; ++s) {
+        J.sweep = first_sweep + s;
+        J.skip = skip_sweep(zero_skip, zero_skip_period, J.sweep);
+        for (int parity = 0; parity < 2; ++parity) {
+            J.parity = parity;
+            J.next = parity;
+            int started = 0;
+            for (int t = 0; t < nthreads; ++t)
+                if (pthread_create(&th[t], NULL, zpar_worker, &J) == 0) ++started;
+            if (started == 0) zpar_worker(&J);
+            for (int t = 0; t < started; ++t) pthread_join(th[t], NULL);
+        }
+    }
+    pthread_mutex_destroy(&J.mu);
+    if (st) {
+        st->updates += J.upd;
+        st->skipped += J.skp;
+        st->sum_abs_delta += J.sad;
+    }
+    return J.fail ? -1 : 0;
 }
 
 void orc_error_sinogram(const orc_geom* g, int K, const int32_t* first, const int32_t* count,

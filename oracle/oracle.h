@@ -19,8 +19,8 @@
  *   - The MAP cost f(x) = 1/2 (y-Ax)^T W (y-Ax) + sum_{pairs} b_jr rho(x_j - x_r)
  *     (Eq. 1 at P:351, with the 1/2 implied by Alg. 1's thetas; reading R7).
  *
- * All arithmetic is IEEE double, single thread, no blocking/fusion/reordering beyond
- * the definitions above.  Pins (tests/test_oracle_pins.py) tie it to closed forms,
+ * All arithmetic is IEEE double, single thread (orc_icd_run_zpar: one thread per slice of a
+ * z-parity on POSIX threads, an exact serialisation), no blocking/fusion/reordering beyond the definitions above.  Pins (tests/test_oracle_pins.py) tie it to closed forms,
  * brute force, paper-printed values and invariants.
  *
  * Parity status per function:
@@ -113,16 +113,26 @@ void orc_voxel_update(const orc_geom* g, const orc_prior* pr, int K,
  * in `order` (if non-NULL, `order_len` voxel indices per sweep) or a fresh random
  * permutation (splitmix64 Fisher-Yates seeded from (seed, sweep number)).  Zero-skip
  * (reading R9): when zero_skip != 0 and the 1-based sweep number (first_sweep + s) > 1,
- * skip voxel j iff x_j and all its neighbours are exactly 0.
+ * skip voxel j iff x_j and all its neighbours are exactly 0 -- except in sweeps whose number
+ * is a multiple of zero_skip_period (> 0), which re-examine every voxel.
  * e must equal y - A x on entry (use orc_error_sinogram).  If dump != NULL it receives
  * (j, theta1, theta2, delta) for every executed update, in order (dump_cap entries max).
  * Returns number of dump entries written. */
 int64_t orc_icd_run(const orc_geom* g, const orc_prior* pr, int K,
                     const int32_t* first, const int32_t* count, const double* vals,
                     const double* w, double* x, double* e,
-                    int n_equits, int first_sweep, uint64_t seed, int zero_skip,
+                    int n_equits, int first_sweep, uint64_t seed, int zero_skip, int zero_skip_period,
                     const int64_t* order, int64_t order_len,
                     double* dump, int64_t dump_cap, orc_stats* st);
+
+/* The same ICD with slices of one z-parity run concurrently on nthreads POSIX threads:
+ * per sweep, parity 0 slices then parity 1 slices, each slice in its own random order.  An
+ * exact serialisation of sequential ICD (same-parity slices share no data; see oracle.c).
+ * Returns 0, or -1 on allocation failure.  Stats are accumulated into *st. */
+int orc_icd_run_zpar(const orc_geom* g, const orc_prior* pr, int K, const int32_t* first,
+                     const int32_t* count, const double* vals, const double* w, double* x,
+                     double* e, int n_equits, int first_sweep, uint64_t seed, int zero_skip,
+                     int zero_skip_period, int nthreads, orc_stats* st);
 
 /* e = y - A x for the whole volume (per slice, same A). */
 void orc_error_sinogram(const orc_geom* g, int K, const int32_t* first, const int32_t* count,

@@ -26,7 +26,8 @@ EXPORTS = (
     "mbir_set_image", "mbir_init_fbp", "mbir_reconstruct", "mbir_iterate", "mbir_get_image",
     "mbir_get_error_sinogram", "mbir_rmse_hu", "mbir_query_sizes", "mbir_get_sysmatrix",
     "mbir_get_sysmatrix_columns",
-    "mbir_probe_update", "mbir_nccl_unique_id", "mbir_halo_plan", "mbir_destroy",
+    "mbir_probe_update", "mbir_set_update_dump", "mbir_get_update_dump", "mbir_get_schedule",
+    "mbir_nccl_unique_id", "mbir_halo_plan", "mbir_destroy",
     "mbir_strerror", "mbir_last_error",
 )
 
@@ -52,6 +53,7 @@ class mbir_options(C.Structure):
         ("sv_side", C.c_int), ("sv_fraction", C.c_double), ("batch_svs", C.c_int),
         ("batch_threshold", C.c_int), ("zero_skip", C.c_int), ("quantize_A", C.c_int),
         ("seed", C.c_uint64), ("deterministic", C.c_int), ("cluster", C.c_int),
+        ("zero_skip_period", C.c_int),
     ]
 
 
@@ -77,7 +79,7 @@ class mbir_sizes(C.Structure):
         ("nsv_x", C.c_int), ("nsv_y", C.c_int), ("nsv", C.c_int), ("K", C.c_int),
         ("band_max", C.c_int), ("svb_rows", C.c_int), ("threads_per_cta", C.c_int), ("cluster", C.c_int), ("resident_ctas", C.c_int),
         ("smem_bytes", C.c_int), ("nnz", C.c_int64), ("a_bytes", C.c_int64),
-        ("band_entries", C.c_int64),
+        ("band_entries", C.c_int64), ("max_group", C.c_int),
     ]
 
     def as_dict(self):
@@ -130,6 +132,12 @@ def load(path: str = LIB_PATH):
     L.mbir_get_sysmatrix_columns.argtypes = [H, vp, C.c_int, vp, vp, vp, vp, vp]
     L.mbir_probe_update.restype = C.c_int
     L.mbir_probe_update.argtypes = [H, vp, C.c_int, vp, vp, vp]
+    L.mbir_set_update_dump.restype = C.c_int
+    L.mbir_set_update_dump.argtypes = [H, C.c_int64]
+    L.mbir_get_update_dump.restype = C.c_int
+    L.mbir_get_update_dump.argtypes = [H, C.c_int64, vp, vp, vp, vp, C.POINTER(C.c_int64)]
+    L.mbir_get_schedule.restype = C.c_int
+    L.mbir_get_schedule.argtypes = [H, vp, vp, vp]
     L.mbir_nccl_unique_id.restype = C.c_int
     L.mbir_nccl_unique_id.argtypes = [vp]
     L.mbir_halo_plan.restype = C.c_int

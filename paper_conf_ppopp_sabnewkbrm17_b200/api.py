@@ -17,7 +17,7 @@ __all__ = [
     "Geometry", "Prior", "Options", "mbir_create", "mbir_set_sinogram", "mbir_set_image",
     "mbir_reconstruct", "mbir_iterate", "mbir_get_image", "mbir_get_error_sinogram",
     "mbir_rmse_hu", "mbir_query_sizes", "mbir_get_sysmatrix", "mbir_get_sysmatrix_columns",
-    "mbir_probe_update",
+    "mbir_probe_update", "mbir_set_update_dump", "mbir_get_update_dump", "mbir_get_schedule",
     "mbir_nccl_unique_id", "mbir_destroy", "Reconstructor",
 ]
 
@@ -73,11 +73,12 @@ class Options:
     seed: int = 3000
     deterministic: int = 0
     cluster: int = 0  # update-kernel CTAs per SV task: 0 auto, 1, 2 (same arithmetic)
+    zero_skip_period: int = 4  # every n-th iteration without zero-skip (reading R9); 0 = never
 
     def c(self) -> L.mbir_options:
         return L.mbir_options(self.sv_side, self.sv_fraction, self.batch_svs,
                               self.batch_threshold, self.zero_skip, self.quantize_A, self.seed,
-                              self.deterministic, self.cluster)
+                              self.deterministic, self.cluster, self.zero_skip_period)
 
 
 def _buf(a, n: int | None = None, dtype=np.float32, writable=False):
@@ -106,10 +107,24 @@ def mbir_nccl_unique_id() -> bytes:
     return bytes(buf)
 
 
+def _torch_current_stream(device: int):
+    """torch's current CUDA stream on `device` (as a cudaStream_t), if torch is already in use
+    with CUDA: the library then orders its work after the torch kernels that produced its device
+    inputs (mbir.h: device buffers must be ready on the handle's stream).  None otherwise (the
+    library creates its own stream)."""
+    import sys
+    torch = sys.modules.get("torch")
+    if torch is None or not torch.cuda.is_available():
+        return None
+    return torch.cuda.current_stream(device).cuda_stream or None
+
+
 def mbir_create(g: Geometry, p: Prior | None = None, o: Options | None = None, *, device: int = 0,
                 stream: int | None = None, rank: int = 0, nranks: int = 1,
                 nccl_id: bytes | None = None):
     lib = L.load()
+    if stream is None:
+        stream = _torch_current_stream(device)
     gc = g.c()
     pc = (p or Prior()).c()
     oc = (o or Options()).c()
@@ -233,6 +248,33 @@ def mbir_probe_update(h, voxels):
     return t1, t2, dl
 
 
+def mbir_set_update_dump(h, capacity: int):
+    L.check(L.load().mbir_set_update_dump(h, int(capacity)), h, "mbir_set_update_dump")
+
+
+def mbir_get_update_dump(h, cap: int):
+    """Returns (voxels int64, theta1, theta2, delta float32, n_recorded)."""
+    vox = np.empty(cap, np.int64)
+    t1 = np.empty(cap, np.float32)
+    t2 = np.empty(cap, np.float32)
+    dl = np.empty(cap, np.float32)
+    n = C.c_int64()
+    L.check(L.load().mbir_get_update_dump(h, cap, vox.ctypes.data, t1.ctypes.data, t2.ctypes.data,
+                                          dl.ctypes.data, C.byref(n)), h, "mbir_get_update_dump")
+    m = min(n.value, cap)
+    return vox[:m], t1[:m], t2[:m], dl[:m], n.value
+
+
+def mbir_get_schedule(h, g: Geometry, sizes: dict):
+    """(task_list [nz][4][max_group] int32, task_count [nz][4] int32, amount [nz][nsv] float32)."""
+    tl = np.empty((g.nz_local, 4, sizes["max_group"]), np.int32)
+    tc = np.empty((g.nz_local, 4), np.int32)
+    am = np.empty((g.nz_local, sizes["nsv"]), np.float32)
+    L.check(L.load().mbir_get_schedule(h, tl.ctypes.data, tc.ctypes.data, am.ctypes.data), h,
+            "mbir_get_schedule")
+    return tl, tc, am
+
+
 def mbir_destroy(h):
     if h:
         L.load().mbir_destroy(h)
@@ -298,3 +340,12 @@ class Reconstructor:
 
     def probe(self, voxels):
         return mbir_probe_update(self.h, voxels)
+
+    def set_update_dump(self, capacity: int):
+        mbir_set_update_dump(self.h, capacity)
+
+    def update_dump(self, cap: int):
+        return mbir_get_update_dump(self.h, cap)
+
+    def schedule(self):
+        return mbir_get_schedule(self.h, self.g, self.sizes())

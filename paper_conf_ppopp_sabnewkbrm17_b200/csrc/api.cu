@@ -105,6 +105,11 @@ struct mbir_handle {
     int kev_used = 0;
     unsigned long long* d_tprof = nullptr;  // phase cycle counters (env MBIR_PHASE_PROFILE)
     unsigned long long* d_trace = nullptr;  // per-pair clock trace of one visit (env MBIR_TRACE)
+    PriorConst pc{};  // q-GGMRF constants and neighbourhood, passed to every kernel by value
+    // per-update record (test hook mbir_set_update_dump): [cap][4] = (voxel, theta1, theta2, delta)
+    float* d_dump = nullptr;
+    unsigned long long* d_dump_count = nullptr;
+    int64_t dump_cap = 0;
     std::string err;
 };
 
@@ -165,7 +170,10 @@ IcdParams make_params(mbir_handle* h)
     p.deterministic = h->o.deterministic;
     p.tprof = h->d_tprof;
     p.trace = h->d_trace;
-    p.dbg = getenv("MBIR_DBG") ? atoi(getenv("MBIR_DBG")) : 0;
+    p.pc = h->pc;
+    p.dump = h->d_dump;
+    p.dump_count = h->d_dump_count;
+    p.dump_cap = h->dump_cap;
     return p;
 }
 
@@ -238,6 +246,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
     const int parities = (nnb == 26 && h->g.nz_total > 1) ? 2 : 1;
     const int target_ctas = h->nsm * h->blocks_per_sm;
     int64_t updates = 0, skipped = 0, visits = 0, empty = 0, iters = 0, launches = 0, klaunches = 0;
+    int zero_iters = 0;  // consecutive iterations without an executed update
     double ksec = 0.0;
     double sum_delta = 0.0;
     CK(cudaEventRecord(h->ev0, h->st));
@@ -263,6 +272,12 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         sp.sv_amount = h->d_amount;
         sp.task_list = h->d_task_list;
         sp.task_count = h->d_task_count;
+        // zero-skip re-admission iteration (reading R9): no zero-skipping, and a RANDOM subset, so
+        // that SVs frozen at 0 (update amount 0, never among the "top" ones) are re-examined
+        // (iterations 1 + k P, k >= 1: with an even period these are random-subset iterations
+        // anyway, so the top-amount iterations stay as Alg. 3 has them)
+        const bool readmit = h->o.zero_skip && h->o.zero_skip_period > 0 && h->iter > 1 &&
+                             h->iter % h->o.zero_skip_period == 1 % h->o.zero_skip_period;
         if (h->o.deterministic) {
             sp.mode = 3;
             sp.nsel = h->nsv;
@@ -270,7 +285,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
             sp.mode = 0;
             sp.nsel = h->nsv;
         } else {
-            sp.mode = (h->iter % 2 == 0) ? 1 : 2;
+            sp.mode = (h->iter % 2 == 0 && !readmit) ? 1 : 2;
             sp.nsel = std::min(h->nsv, std::max(1, (int)ceil(h->o.sv_fraction * h->nsv - 1e-9)));
         }
         CK(launch_select(sp, h->st));
@@ -296,14 +311,15 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         ++launches;
         CK(cudaMemsetAsync(h->d_fetch, 0, sizeof(int) * 8 * nb, h->st));
         IcdParams p = make_params(h);
-        p.zero_skip_active = (h->o.zero_skip && h->iter > 1) ? 1 : 0;
+        // zero-skip from iteration 2 on, except in re-admission iterations
+        p.zero_skip_active = (h->o.zero_skip && h->iter > 1 && !readmit) ? 1 : 0;
         const size_t cap = (size_t)h->g.nz_local * h->max_group;
         // deterministic: one CTA (or one cluster) walks the phase list in order (sequential ICD,
         // known order)
         const int grid = det ? h->cl : target_ctas;
         // iterations >= 2 without batching: the tasks whose whole tile is zero are flagged per
         // phase (sched.cu k_zero_flags) and skipped at task fetch by the update kernel
-        const bool prefilter = p.zero_skip_active && nb == 1 && !det && !(p.dbg & 4);
+        const bool prefilter = p.zero_skip_active && nb == 1 && !det;
         for (int zp = 0; zp < parities; ++zp) {
             for (int colour = 0; colour < 4; ++colour) {
                 const int ph = zp * 4 + colour;
@@ -353,9 +369,17 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         if (!isfinite(sd)) return fail(h, MBIR_ENUMERIC, "non-finite update amount");
         sum_delta += sd;
         ++iters;
-        if (n_iter < 0 && h->h_counters[0] == 0 && h->h_counters[2] > 0 && h->o.zero_skip) {
-            // everything zero-skipped: the image is all zero and stays so; stop
-            break;
+        if (n_iter < 0) {
+            if (h->h_counters[2] == 0)  // nothing was scheduled: the loop could never progress
+                return fail(h, MBIR_ESTATE, "an iteration scheduled no SuperVoxel (batch threshold "
+                                            "drops every task: lower batch_threshold or batch_svs)");
+            // no executed update: either every visited voxel was zero-skipped (a random subset
+            // can be all zero while the image is not), or the image is all zero.  Stop only when
+            // an iteration that visited every SV without zero-skipping executed nothing (then the
+            // image is all zero and stays so), or after 16 consecutive such iterations
+            zero_iters = h->h_counters[0] == 0 ? zero_iters + 1 : 0;
+            const bool visited_all = (h->iter == 1 || h->o.deterministic) && !p.zero_skip_active;
+            if (h->h_counters[0] == 0 && (visited_all || zero_iters >= 16)) break;
         }
     }
     CK(cudaEventRecord(h->ev1, h->st));
@@ -421,6 +445,8 @@ void mbir_default_options(mbir_options* o)
     o->quantize_A = 1;
     o->seed = 3000;
     o->deterministic = 0;
+    o->cluster = 0;
+    o->zero_skip_period = 4;
 }
 
 void mbir_default_prior(mbir_prior* p)
@@ -496,7 +522,7 @@ void mbir_destroy(mbir_handle* h)
                     h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
                     h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count,
                     h->d_flat, h->d_brange, h->d_fetch, h->d_keep, h->d_perm, h->d_counters, h->d_sum_delta,
-                    h->d_flag, h->d_acc, h->d_tprof, h->d_trace};
+                    h->d_flag, h->d_acc, h->d_tprof, h->d_trace, h->d_dump, h->d_dump_count};
     if (h->d_trace && getenv("MBIR_TRACE")) {  // development aid: raw clock stamps (tools/trace_visit.py)
         std::vector<unsigned long long> t(1024);
         cudaMemcpy(t.data(), h->d_trace, 1024 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
@@ -556,8 +582,16 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         (P.neighborhood != 8 && P.neighborhood != 26))
         return bail(MBIR_EINVAL);
     if (h->o.sv_side < 1 || h->o.sv_side > 16 || !(h->o.sv_fraction > 0 && h->o.sv_fraction <= 1) ||
-        h->o.batch_svs < 0)
+        h->o.batch_svs < 0 || h->o.zero_skip_period < 0)
         return bail(MBIR_EINVAL);
+    {
+        // the phase task lists (sched.cu k_flatten) gather at most kMaxPhaseSlices slices of one
+        // z-parity: reject larger slabs instead of leaving slices unscheduled
+        const int parities = (P.neighborhood == 26 && h->g.nz_total > 1) ? 2 : 1;
+        if ((G.nz_local + parities - 1) / parities > kMaxPhaseSlices)
+            return (fail(h, MBIR_EINVAL, "nz_local too large: at most " + std::to_string(kMaxPhaseSlices) +
+                                             " slices per z-parity phase per rank"), bail(MBIR_EINVAL));
+    }
     if (h->nranks > 1 && (!d || !d->nccl_unique_id || h->rank < 0 || h->rank >= h->nranks))
         return bail(MBIR_EINVAL);
     if (G.angles) h->angles.assign(G.angles, G.angles + G.nviews);
@@ -565,7 +599,10 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
 
     if (cudaSetDevice(h->device) != cudaSuccess) return bail(MBIR_ECUDA);
     if (!h->st) {
-        if (cudaStreamCreateWithFlags(&h->st, cudaStreamNonBlocking) != cudaSuccess) return bail(MBIR_ECUDA);
+        // a BLOCKING stream: its work is ordered after (and before) work on the legacy default
+        // stream, so device inputs produced there (e.g. torch tensors on torch's default stream)
+        // are complete before the library reads them
+        if (cudaStreamCreateWithFlags(&h->st, cudaStreamDefault) != cudaSuccess) return bail(MBIR_ECUDA);
         h->own_stream = true;
     }
     int r;
@@ -756,7 +793,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         pc.qmp = (float)(P.q - P.p);
         pc.inv_Ts = (float)(1.0 / (P.T * P.sigma));
         pc.positivity = P.positivity;
-        if (set_prior_constants(pc) != cudaSuccess) return bail(MBIR_ECUDA);
+        h->pc = pc;
     }
 
     // ---- multi-GPU communicator (z-slab partition)
@@ -814,15 +851,25 @@ int mbir_set_image(mbir_handle* h, const float* x0, int where)
     if (!h) return MBIR_EINVAL;
     const size_t pl = plane_elems(h);
     if (x0) {
-        CK(cudaMemcpyAsync(h->d_x + pl, x0, pl * h->g.nz_local * 4, kind_in(where), h->st));
+        // validate in a temporary buffer first: on rejection the image, e and the scheduler
+        // state stay untouched (e = y - A x keeps holding).  The verdict is agreed across ranks
+        // before anyone returns, so a rejecting rank cannot leave the others in the collective
+        // halo exchange below.
+        const size_t n = pl * h->g.nz_local;
+        float* tmp = nullptr;
+        CK(cudaMallocAsync((void**)&tmp, n * 4, h->st));
+        CK(cudaMemcpyAsync(tmp, x0, n * 4, kind_in(where), h->st));
         CK(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->st));
-        CK(launch_check_finite(h->d_x + pl, (int64_t)(pl * h->g.nz_local), h->pr.positivity, h->d_flag, h->st));
+        CK(launch_check_finite(tmp, (int64_t)n, h->pr.positivity, h->d_flag, h->st));
+        if (h->nranks > 1) CKN(nccl().AllReduce(h->d_flag, h->d_flag, 1, ncclInt32, ncclMax, h->comm, h->st));
         int flag = 0;
         CK(cudaMemcpyAsync(&flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost, h->st));
         CK(cudaStreamSynchronize(h->st));
+        if (!flag) CK(cudaMemcpyAsync(h->d_x + pl, tmp, n * 4, cudaMemcpyDeviceToDevice, h->st));
+        CK(cudaFreeAsync(tmp, h->st));
         if (flag) {
-            cudaMemsetAsync(h->d_x + pl, 0, pl * h->g.nz_local * 4, h->st);
-            return fail(h, MBIR_EINVAL, "x0 must be finite (and >= 0 with positivity)");
+            CK(cudaStreamSynchronize(h->st));
+            return fail(h, MBIR_EINVAL, "x0 must be finite (and >= 0 with positivity) on every rank");
         }
     } else {
         CK(cudaMemsetAsync(h->d_x + pl, 0, pl * h->g.nz_local * 4, h->st));
@@ -929,6 +976,7 @@ int mbir_query_sizes(const mbir_handle* h, mbir_sizes* s)
     s->nnz = h->nnz;
     s->a_bytes = h->a_bytes;
     s->band_entries = h->band_entries;
+    s->max_group = h->max_group;
     return MBIR_OK;
 }
 
@@ -985,6 +1033,62 @@ int mbir_get_sysmatrix_columns(mbir_handle* h, const int64_t* voxels, int n, int
     for (int i = 0; i < n; ++i)
         if (voxels[i] < 0 || voxels[i] >= (int64_t)plane_elems(h)) return fail(h, MBIR_EINVAL, "voxel index out of range");
     return export_sysmatrix(h, voxels, n, first, count, values, codes, scales);
+}
+
+int mbir_set_update_dump(mbir_handle* h, int64_t capacity)
+{
+    if (!h || capacity < 0) return MBIR_EINVAL;
+    CK(cudaStreamSynchronize(h->st));
+    if (h->d_dump) cudaFree(h->d_dump);
+    if (h->d_dump_count) cudaFree(h->d_dump_count);
+    h->d_dump = nullptr;
+    h->d_dump_count = nullptr;
+    h->dump_cap = 0;
+    if (capacity == 0) return MBIR_OK;
+    int r;
+    if ((r = dalloc(h, &h->d_dump, (size_t)capacity * 4))) return r;
+    if ((r = dalloc(h, &h->d_dump_count, 1))) return r;
+    CK(cudaMemsetAsync(h->d_dump_count, 0, sizeof(unsigned long long), h->st));
+    CK(cudaStreamSynchronize(h->st));
+    h->dump_cap = capacity;
+    return MBIR_OK;
+}
+
+int mbir_get_update_dump(mbir_handle* h, int64_t cap, int64_t* voxels, float* theta1, float* theta2,
+                         float* delta, int64_t* n)
+{
+    if (!h || cap < 0 || !n || (cap > 0 && (!voxels || !theta1 || !theta2 || !delta))) return MBIR_EINVAL;
+    if (!h->d_dump) return fail(h, MBIR_ESTATE, "mbir_set_update_dump has not been called");
+    unsigned long long cnt = 0;
+    CK(cudaMemcpyAsync(&cnt, h->d_dump_count, sizeof(cnt), cudaMemcpyDeviceToHost, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    const int64_t m = std::min<int64_t>({(int64_t)cnt, cap, h->dump_cap});
+    std::vector<float> buf((size_t)m * 4);
+    if (m > 0) CK(cudaMemcpy(buf.data(), h->d_dump, (size_t)m * 16, cudaMemcpyDeviceToHost));
+    for (int64_t i = 0; i < m; ++i) {
+        uint32_t v;
+        memcpy(&v, &buf[4 * i], 4);
+        voxels[i] = (int64_t)v;
+        theta1[i] = buf[4 * i + 1];
+        theta2[i] = buf[4 * i + 2];
+        delta[i] = buf[4 * i + 3];
+    }
+    *n = (int64_t)cnt;
+    CK(cudaMemsetAsync(h->d_dump_count, 0, sizeof(unsigned long long), h->st));
+    CK(cudaStreamSynchronize(h->st));
+    return MBIR_OK;
+}
+
+int mbir_get_schedule(mbir_handle* h, int32_t* task_list, int32_t* task_count, float* amount)
+{
+    if (!h) return MBIR_EINVAL;
+    const size_t nz = h->g.nz_local;
+    if (task_list)
+        CK(cudaMemcpyAsync(task_list, h->d_task_list, nz * 4 * h->max_group * 4, cudaMemcpyDeviceToHost, h->st));
+    if (task_count) CK(cudaMemcpyAsync(task_count, h->d_task_count, nz * 4 * 4, cudaMemcpyDeviceToHost, h->st));
+    if (amount) CK(cudaMemcpyAsync(amount, h->d_amount, nz * h->nsv * 4, cudaMemcpyDeviceToHost, h->st));
+    CK(cudaStreamSynchronize(h->st));
+    return MBIR_OK;
 }
 
 int mbir_probe_update(mbir_handle* h, const int64_t* voxels, int n, float* theta1, float* theta2,

@@ -29,29 +29,22 @@
 
 namespace mbir {
 
-__constant__ PriorConst c_prior;
-
-cudaError_t set_prior_constants(const PriorConst& pc)
-{
-    return cudaMemcpyToSymbol(c_prior, &pc, sizeof(pc));
-}
-
 namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 
 // phi(D) = rho'(D)/(2D) for the q-GGMRF potential with q = 2 (reading R1):
 //   phi = c_phi * (q/p + u) / (1 + u)^2,  u = |D/(T sigma)|^(q-p)   (|D|^(q-2) = 1)
-__device__ __forceinline__ float phi_f(float d)
+__device__ __forceinline__ float phi_f(const PriorConst& pc, float d)
 {
     const float ad = fabsf(d);
     float u;
-    if (c_prior.qmp == 0.f)
+    if (pc.qmp == 0.f)
         u = 1.f;
     else
-        u = (ad == 0.f) ? 0.f : exp2f(c_prior.qmp * __log2f(ad * c_prior.inv_Ts));
+        u = (ad == 0.f) ? 0.f : exp2f(pc.qmp * __log2f(ad * pc.inv_Ts));
     const float opu = 1.f + u;
-    return __fdividef(c_prior.c_phi * (c_prior.pq + u), opu * opu);
+    return __fdividef(pc.c_phi * (pc.pq + u), opu * opu);
 }
 
 // uint8 code i of a packed word -> float, via the 2^23 magic (PRMT + FADD, no I2F)
@@ -207,7 +200,7 @@ __device__ __forceinline__ void prior_pair(const int* tof, int i0, int nact, con
         const int gx = gx0 + lx + nb.dx[k], gy = gy0 + ly + nb.dy[k], gz = zg + nb.dz[k];
         if (nb.w[k] != 0.f && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total) {
             const float xr = xt[c0 + nb.dt[k]];
-            const float bt = nb.w[k] * phi_f(v - xr);
+            const float bt = nb.w[k] * phi_f(P.pc, v - xr);
             sb += bt;
             sx += bt * xr;
             if (nb.dz[k] == 0 && nb.dx[k] == dxa && nb.dy[k] == dya) {
@@ -274,11 +267,6 @@ template <int N>
 __device__ __forceinline__ void cp_async_wait()
 {
     asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-// warm L2 with a global block (bulk prefetch; no completion tracking)
-__device__ __forceinline__ void l2_prefetch_bulk(const void* src, uint32_t bytes)
-{
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
 }
 
 // ---- thread-block-cluster helpers (CL = 2: the two CTAs of a cluster split an SV's views) ----
@@ -471,11 +459,11 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
 #pragma unroll
     for (int k = 0; k < 2; ++k) {
         const int r = (lane & 15) + 16 * k;
-        const bool ok = r < c_prior.nnb;
-        nb.dx[k] = ok ? c_prior.dx[r] : 0;
-        nb.dy[k] = ok ? c_prior.dy[r] : 0;
-        nb.dz[k] = ok ? c_prior.dz[r] : 0;
-        nb.w[k] = ok ? c_prior.b[r] : 0.f;
+        const bool ok = r < P.pc.nnb;
+        nb.dx[k] = ok ? P.pc.dx[r] : 0;
+        nb.dy[k] = ok ? P.pc.dy[r] : 0;
+        nb.dz[k] = ok ? P.pc.dz[r] : 0;
+        nb.w[k] = ok ? P.pc.b[r] : 0.f;
         nb.dt[k] = (nb.dz[k] * (side + 2) + nb.dy[k]) * (side + 2) + nb.dx[k];
     }
 
@@ -571,11 +559,11 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 keep = 1;
                 if (P.zero_skip_active) {
                     keep = xt[(zc * TW + ly + 1) * TW + lx + 1] != 0.f;
-                    for (int r = 0; r < c_prior.nnb && !keep; ++r) {
-                        const int gx = gx0 + lx + c_prior.dx[r], gy = gy0 + ly + c_prior.dy[r];
-                        const int gz = zg + c_prior.dz[r];
+                    for (int r = 0; r < P.pc.nnb && !keep; ++r) {
+                        const int gx = gx0 + lx + P.pc.dx[r], gy = gy0 + ly + P.pc.dy[r];
+                        const int gz = zg + P.pc.dz[r];
                         if (gx < 0 || gx >= P.nx || gy < 0 || gy >= P.ny || gz < 0 || gz >= P.nz_total) continue;
-                        keep = xt[((zc + c_prior.dz[r]) * TW + ly + 1 + c_prior.dy[r]) * TW + lx + 1 + c_prior.dx[r]] != 0.f;
+                        keep = xt[((zc + P.pc.dz[r]) * TW + ly + 1 + P.pc.dy[r]) * TW + lx + 1 + P.pc.dx[r]] != 0.f;
                     }
                 }
             }
@@ -637,13 +625,6 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
             (void)tp;
             copy_record_to(j, (sbase + j) % R, j < nact ? list[j] : 0);
         };
-        // prior warp, lane 0 (development switch MBIR_DBG bit 0): L2 warm-up of voxel j's record
-        auto prefetch_record = [&](int j) {
-            if (!(P.dbg & 1)) return;
-            const size_t rec = (arec + list[j]) * (size_t)P.A.VA + vbase;
-            l2_prefetch_bulk(U8 ? (const void*)(P.A.codes + rec) : (const void*)(P.A.vals + rec), VL * (U8 ? 4 : 16));
-            l2_prefetch_bulk(P.A.off + rec, VL);
-        };
         if (is_prior) {
             // one of NPERM host-drawn random permutations of the tile, chosen per
             // (seed, iteration, slice, SV) visit; identity (raster order) in deterministic mode
@@ -670,9 +651,8 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
             }
             __syncwarp();
             if (lane == 0) {
-                // the L2 warm-up of the records R .. 2R-1, and the next task (rank 0 fetches it;
-                // CL = 2 hands it to rank 1 through DSMEM + an mbarrier arrival)
-                for (int i = R; i < 2 * R && i < nact; ++i) prefetch_record(i);
+                // the next task (rank 0 fetches it; CL = 2 hands it to rank 1 through DSMEM + an
+                // mbarrier arrival)
                 if (crank == 0) {
                     publish_task(nslot, fetch_task());
                     if (CL == 2) mbar_arrive_peer(peer_addr(taskbar, 1));
@@ -726,7 +706,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 const uint32_t bi = vbase + kk < V ? binfo[tb * VL + kk] : 0u;
                 const int bwt = (int)(bi & 31u), sk = (int)(bi >> 5) & 3;
                 const uint32_t bmask = ((1u << bwt) - 1u) << sk;  // band's window positions
-                if (!isw && !(P.dbg & 128)) {  // (dbg 128: timing ablation)
+                if (!isw) {
 #pragma unroll
                     for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), v4[m]);
                 }
@@ -932,7 +912,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 //      entries the two voxels share with the full value, so A_b is never needed on
                 //      a's channels
                 const float sda = dslot[(pn & 1) * 2], sdb = dslot[(pn & 1) * 2 + 1];
-                if ((sda != 0.f || sdb != 0.f) && !(P.dbg & 16)) {  // (dbg 16: timing ablation)
+                if (sda != 0.f || sdb != 0.f) {
                     const float2 nda = make_float2(-sda, -sda), ndb = make_float2(-sdb, -sdb);
                     auto put2 = [&](float* p, float2 v0, float2 v1) {
                         p[0] = v0.x;
@@ -992,43 +972,53 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 const PriPair pp = pri[buf];
                 const float scale_a = vscale[idx];
                 float ua = pp.va;
+                const float theta1a = -scale_a * sa;  // Alg1:5
+                const float theta2a = vth2[idx];      // Alg1:6 (precomputed)
                 {
-                    const float theta1 = -scale_a * sa;  // Alg1:5
-                    const float theta2 = vth2[idx];      // Alg1:6 (precomputed)
-                    const float num = theta2 * pp.va - theta1 + 2.f * pp.sxa;
-                    const float den = theta2 + 2.f * pp.sa;
+                    const float num = theta2a * pp.va - theta1a + 2.f * pp.sxa;
+                    const float den = theta2a + 2.f * pp.sa;
                     if (den > 0.f) ua = __fdividef(num, den);
-                    if (c_prior.positivity) ua = fmaxf(ua, 0.f);
+                    if (P.pc.positivity) ua = fmaxf(ua, 0.f);
                 }
                 const float da = ua - pp.va;  // Alg1:7-8
-                float ub = pp.vb, db = 0.f, scale_b = 0.f;
+                float ub = pp.vb, db = 0.f, scale_b = 0.f, theta1b = 0.f, theta2b = 0.f;
                 if (hasb) {
                     scale_b = vscale[idx + 1];
                     // e after a's update: sum w A_b e' = s_b (S_b - s_a delta_a H)
-                    const float theta1 = -scale_b * fmaf(-scale_a * da, sh, sbs);
-                    const float theta2 = vth2[idx + 1];
+                    const float theta1 = theta1b = -scale_b * fmaf(-scale_a * da, sh, sbs);
+                    const float theta2 = theta2b = vth2[idx + 1];
                     float psb = pp.sb, psx = pp.sxb;
                     if (pp.bab != 0.f) {  // a is b's neighbour: its term with a's new value
-                        const float bn = pp.bab * phi_f(pp.vb - ua);
+                        const float bn = pp.bab * phi_f(P.pc, pp.vb - ua);
                         psb += bn - pp.btab;
                         psx += bn * ua - pp.btab * pp.va;
                     }
                     const float num = theta2 * pp.vb - theta1 + 2.f * psx;
                     const float den = theta2 + 2.f * psb;
                     if (den > 0.f) ub = __fdividef(num, den);
-                    if (c_prior.positivity) ub = fmaxf(ub, 0.f);
+                    if (P.pc.positivity) ub = fmaxf(ub, 0.f);
                     db = ub - pp.vb;
                 }
                 if (lane == 0) {
                     dslot[(pn & 1) * 2] = scale_a * da;
                     dslot[(pn & 1) * 2 + 1] = scale_b * db;
                 }
+                if (P.dump && lane == 0) {
+                    // test hook (mbir_set_update_dump): the pair's (voxel, theta1, theta2, delta)
+                    // exactly as the delta chain used them (b's theta1 includes a's update), a then b
+                    const unsigned long long slot = atomicAdd(P.dump_count, hasb ? 2ull : 1ull);
+                    for (int u = 0; u < (hasb ? 2 : 1); ++u) {
+                        const int tv = tof[idx + u];
+                        const uint32_t vox = (uint32_t)(((size_t)z * P.ny + gy0 + (tv >> 8)) * P.nx + gx0 + (tv & 255));
+                        if (slot + u < (unsigned long long)P.dump_cap)
+                            *(float4*)(P.dump + 4 * (slot + u)) = make_float4(
+                                __uint_as_float(vox), u ? theta1b : theta1a, u ? theta2b : theta2a, u ? db : da);
+                    }
+                }
                 if (lane == 0) stamp(idx >> 1, 7);
                 asm volatile("bar.arrive 2, %0;" ::"r"(npair_threads) : "memory");  // barrier B
                 // the pair's new values, then the next pair's surrogate terms
                 if (lane == 0) {
-                    if (idx + 2 * R < nact) prefetch_record(idx + 2 * R);
-                    if (idx + 1 + 2 * R < nact) prefetch_record(idx + 1 + 2 * R);
                     const int ta = tof[idx];
                     xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
                     if (hasb) {
@@ -1039,7 +1029,7 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                 }
                 __syncwarp();
                 const long long tr0 = (PROF && P.tprof) ? clock64() : 0;
-                if (idx + 2 < nact && !(P.dbg & 32))  // (dbg 32: timing ablation)
+                if (idx + 2 < nact)
                     prior_pair(tof, idx + 2, nact, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
                                pri + (pn + 1) % kPairBufs);
                 if (PROF && P.tprof && lane == 0) atomicAdd(P.tprof + 24, (unsigned long long)(clock64() - tr0));
@@ -1153,7 +1143,6 @@ __global__ void __launch_bounds__(CL == 2 ? (VPT == 2 ? 224 : 128) : (VPT == 2 ?
                         if (k < kend) {
                             const int r = k * M + bs[i], r1 = r + max(bwd[i], 1) - 1;
                             dst[k] = ((uint32_t)r << 5) | (uint32_t)bwd[i];
-                            if (P.dbg & 2) continue;
                             asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
                             asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
                             asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
@@ -1324,17 +1313,17 @@ __global__ void k_probe(const IcdParams P, const int64_t* vox, float* out3)
         const float v = P.x[(size_t)(z + 1) * plane + (size_t)iy * P.nx + ix];
         float sbv = 0.f, sbx = 0.f;
         const int zg = P.z_offset + z;
-        for (int r = 0; r < c_prior.nnb; ++r) {
-            const int gx = ix + c_prior.dx[r], gy = iy + c_prior.dy[r], gz = zg + c_prior.dz[r];
+        for (int r = 0; r < P.pc.nnb; ++r) {
+            const int gx = ix + P.pc.dx[r], gy = iy + P.pc.dy[r], gz = zg + P.pc.dz[r];
             if (gx < 0 || gx >= P.nx || gy < 0 || gy >= P.ny || gz < 0 || gz >= P.nz_total) continue;
-            const float xr = P.x[(size_t)(z + 1 + c_prior.dz[r]) * plane + (size_t)gy * P.nx + gx];
-            const float bt = c_prior.b[r] * phi_f(v - xr);
+            const float xr = P.x[(size_t)(z + 1 + P.pc.dz[r]) * plane + (size_t)gy * P.nx + gx];
+            const float bt = P.pc.b[r] * phi_f(P.pc, v - xr);
             sbv += bt;
             sbx += bt * xr;
         }
         const float num = T2 * v - T1 + 2.f * sbx, den = T2 + 2.f * sbv;
         float u = den > 0.f ? num / den : v;
-        if (c_prior.positivity) u = fmaxf(u, 0.f);
+        if (P.pc.positivity) u = fmaxf(u, 0.f);
         out3[3 * q] = T1;
         out3[3 * q + 1] = T2;
         out3[3 * q + 2] = u - v;

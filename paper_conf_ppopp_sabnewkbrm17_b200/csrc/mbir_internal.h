@@ -14,12 +14,11 @@ namespace mbir {
 
 constexpr int kK = 4;             // max channels per (voxel, view) (reading R5; K=4 for dc > 0.4714 dxy)
 constexpr int kMaxNbr = 26;       // 3-D neighbourhood (reading R2)
-constexpr int kRingDepth = 4;     // A-record prefetch depth (voxels) in the update kernel
 constexpr int kMaxSvbRows = 32;   // SV-buffer rows held by one 32-lane transpose tile
-constexpr int kMaxThreads = 1024;
+constexpr int kMaxPhaseSlices = 1024;  // slices of one (z-parity, colour) phase (sched.cu k_flatten)
 constexpr double kAutoRayLoad = 1.5;  // batch_svs = 0: concurrently updated SVs one ray meets (R22)
 
-// ---- prior constants in __constant__ memory (set by set_prior_constants) ----
+// ---- prior constants, per handle: passed by value in the kernels' parameter blocks ----
 struct PriorConst {
     int nnb;                 // 8 or 26
     int dx[kMaxNbr], dy[kMaxNbr], dz[kMaxNbr];
@@ -91,10 +90,10 @@ struct IcdParams {
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
     unsigned long long* trace;  // optional per-pair clock trace of one SV visit (env MBIR_TRACE)
-    int dbg;                 // development switches (env MBIR_DBG): bit 0 A-record L2 warm-up on,
-                             // bit 1 band-row L2 warm-up off, bit 2 zero-skip pre-filter off;
-                             // timing ablations with wrong results: bit 4 no scatter, bit 5 no
-                             // prior terms, bit 7 no e_init store
+    PriorConst pc;           // q-GGMRF constants and neighbourhood of this handle (reading R1-R2)
+    float* dump;             // optional [dump_cap][4] (voxel bits, theta1, theta2, delta) per update
+    unsigned long long* dump_count;
+    long long dump_cap;
     SmemLayout lay;          // update-kernel smem layout (filled by launch_icd)
 };
 
@@ -112,7 +111,6 @@ struct SchedParams {
 };
 
 // kernels / launchers (sysmatrix.cu, icd.cu, sched.cu, aux.cu)
-cudaError_t set_prior_constants(const PriorConst& pc);
 cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, int side, int nsvx,
                             int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxoff,
                             cudaStream_t st);

@@ -114,17 +114,17 @@ __global__ void __launch_bounds__(kSelThreads) k_select(const SchedParams S)
 // batches from the first one with fewer than thr SVs left are dropped ("break", reading R15).
 // Kept tasks are interleaved round-robin over slices (rank r of every slice, then r+1, ...),
 // so each batch is a contiguous range and concurrent CTAs work on different slices.
-constexpr int kMaxSlices = 1024;
+// (mbir_create rejects volumes with more than kMaxPhaseSlices slices in one phase)
 __global__ void k_flatten(const int* __restrict__ task_list, const int* __restrict__ task_count,
                           int nz_local, int z_offset, int parities, int max_group, int B, int thr,
                           int nb, int* __restrict__ flat, int* __restrict__ brange)
 {
-    __shared__ int zl[kMaxSlices], K[kMaxSlices];
+    __shared__ int zl[kMaxPhaseSlices], K[kMaxPhaseSlices];
     __shared__ int s_n, s_maxK;
     const int ph = blockIdx.x, parity = ph / 4, colour = ph % 4;
     if (threadIdx.x == 0) {
         int n = 0, mk = 0;
-        for (int z = 0; z < nz_local && n < kMaxSlices; ++z) {
+        for (int z = 0; z < nz_local && n < kMaxPhaseSlices; ++z) {
             if (parities == 2 && ((z_offset + z) & 1) != parity) continue;
             const int cnt = task_count[z * 4 + colour];
             int k = cnt;

@@ -196,9 +196,19 @@ __global__ void k_export(int nx, int ny, double d, int V, int M, double dc, doub
             for (int i = 0; i < kK; ++i) codes[o * kK + i] = (uint8_t)(wd >> (8 * i));
         }
         if (vals) {
-            const double2 a = cs[k];
-            const Col col = column_entry(nx, ny, d, M, dc, center_offset, a.x, a.y, ix, iy);
-            for (int i = 0; i < kK; ++i) vals[o * kK + i] = (float)col.v[i];
+            // the values the update kernel uses: the stored fp32 entries, or (uint8 A) the
+            // dequantised codes code * scale
+            if (quantize) {
+                const uint32_t wd = A.codes[base + apos(k, A.vpt)];
+                const float sc = A.scale[(size_t)sv * A.S2 + slot];
+                for (int i = 0; i < kK; ++i) vals[o * kK + i] = (float)((wd >> (8 * i)) & 255u) * sc;
+            } else {
+                const float4 v = A.vals[base + apos(k, A.vpt)];
+                vals[o * kK + 0] = v.x;
+                vals[o * kK + 1] = v.y;
+                vals[o * kK + 2] = v.z;
+                vals[o * kK + 3] = v.w;
+            }
         }
     }
     if (scales && threadIdx.x == 0) scales[jo] = A.scale[(size_t)sv * A.S2 + slot];

@@ -43,11 +43,25 @@ def test_sysmatrix_bit_exact_index_structure(cfg1, quant):
     np.testing.assert_array_equal(count, A.count)
     m = A.count > 0
     np.testing.assert_array_equal(first[m], A.first[m])
-    np.testing.assert_allclose(vals, A.vals.astype(np.float32), rtol=2e-7, atol=1e-7 * A.vals.max())
     assert sz["nnz"] == int(A.count.sum())
     if quant:
+        # the buffers the update kernel reads: codes bit-exact, scale = fp32(amax/255), and the
+        # exported values are the dequantised code * scale it computes with
         np.testing.assert_array_equal(gcodes, codes)
-        np.testing.assert_allclose(scales, (amax / 255).astype(np.float32), rtol=1e-7)
+        np.testing.assert_array_equal(scales, (amax / 255).astype(np.float32))
+        np.testing.assert_array_equal(vals, codes.astype(np.float32) * scales[:, None, None])
+        np.testing.assert_allclose(vals, Aq.vals, rtol=2.5e-7, atol=0)
+    else:
+        # the stored fp32 values (read back from the buffer the kernel uses) against the oracle's
+        # polygon-clipping areas: two double-precision formulations of the same strip integral,
+        # each rounded once to fp32 (R5): within 1 ulp of fp32 of the value, plus an
+        # absolute term for near-empty sliver entries, whose double-precision difference is
+        # dominated by cancellation in either formulation (measured <= 1e-13 of the column max)
+        d = np.abs(vals.astype(np.float64) - A.vals)
+        ulp = np.spacing(np.abs(A.vals).astype(np.float32)).astype(np.float64)
+        amaxc = A.vals.max(axis=(1, 2), keepdims=True)
+        print("max |dA| / ulp:", (d / np.maximum(ulp, 1e-45)).max(), " max |dA| / column max:", (d / amaxc).max())
+        assert np.all(d <= ulp + 1e-12 * amaxc)
 
 
 def test_sysmatrix_paper_geometry_sampled():
@@ -69,10 +83,10 @@ def test_sysmatrix_paper_geometry_sampled():
         assert mc <= 4
         np.testing.assert_array_equal(count[q], c)
         np.testing.assert_array_equal(first[q][c > 0], f[c > 0])
-        np.testing.assert_allclose(vals[q], v.astype(np.float32), rtol=2e-7, atol=1e-7 * v.max())
         cd, am = O.quantize_column(v, c)
         np.testing.assert_array_equal(gcodes[q], cd)
         assert scales[q] == np.float32(am / 255)
+        np.testing.assert_array_equal(vals[q], cd.astype(np.float32) * scales[q])
 
 
 # ------------------------------------------------------------------ fixed-state probe (a4, a5)
@@ -191,16 +205,17 @@ def test_deterministic_equit_tracks_sequential_oracle_3d():
 
 
 # ------------------------------------------------------------------ converged parity
-@pytest.mark.parametrize("zero_skip,tol_hu,tol_cost", [(0, 1.0, 1e-4), (1, 2.0, 5e-4)])
+@pytest.mark.parametrize("zero_skip,tol_hu,tol_cost", [(0, 1.0, 1e-4), (1, 1.0, 1e-4)])
 def test_converged_image_and_cost_match_oracle_cfg1(cfg1, zero_skip, tol_hu, tol_cost):
     """Asynchronous parallel ICD is nondeterministic, but the MAP point is unique: the
     converged GPU image is within 1 HU RMSE of the oracle's and the cost within 1e-4.  With
-    zero-skipping the fixed point is order-dependent (reading R9), hence the looser bound."""
+    zero-skipping and its periodic re-admission (reading R9) the fixed point is still the
+    MAP, so the same bound holds against the oracle's no-skip run."""
     cfg, case, g, og, A, codes, amax, Aq = cfg1
     pr = O.Prior(sigma=cfg.sigma, nbhd=8)
     x = np.zeros(cfg.n * cfg.n)
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
-    O.icd_run(og, pr, Aq, case.w, x, e, 150, seed=3000, zero_skip=bool(zero_skip))
+    O.icd_run(og, pr, Aq, case.w, x, e, 150, seed=3000, zero_skip=False)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=8),
                          M.Options(sv_side=cfg.sv_side, zero_skip=zero_skip)) as r:
         r.set_sinogram(case.y, case.w)
@@ -218,12 +233,11 @@ def test_converged_image_and_cost_match_oracle_cfg1(cfg1, zero_skip, tol_hu, tol
     assert np.abs(eg.ravel() - eo.ravel()).max() < 1e-3 * np.abs(case.y).max()
 
 
-@pytest.mark.parametrize("zero_skip,tol_hu,tol_cost", [(0, 1.0, 1e-4), (1, 2.0, 5e-4)])
+@pytest.mark.parametrize("zero_skip,tol_hu,tol_cost", [(0, 1.0, 1e-4), (1, 1.0, 1e-4)])
 def test_converged_3d_matches_oracle(zero_skip, tol_hu, tol_cost):
-    """Without zero-skipping the MAP point is unique: 1 HU / 1e-4 (BASELINE.json).  With it
-    (P:115), a voxel whose whole neighbourhood reached 0 is frozen, so the fixed point depends on
-    the update order (reading R9: the oracle's own zero-skip and no-skip runs differ by 2.6e-4
-    in cost on this case); the looser bound covers that path dependence."""
+    """The MAP point is unique: 1 HU / 1e-4 (BASELINE.json) against the oracle's no-skip run,
+    with or without zero-skipping, whose periodic re-admission (reading R9) keeps the
+    MAP as the fixed point."""
     cfg = small3d()
     case = make_case(cfg)
     g, og = geoms(cfg)
@@ -232,7 +246,7 @@ def test_converged_3d_matches_oracle(zero_skip, tol_hu, tol_cost):
     pr = O.Prior(sigma=cfg.sigma, nbhd=26)
     x = np.zeros(cfg.nz * cfg.n * cfg.n)
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
-    O.icd_run(og, pr, Aq, case.w, x, e, 120, seed=3000, zero_skip=bool(zero_skip))
+    O.icd_run(og, pr, Aq, case.w, x, e, 120, seed=3000, zero_skip=False)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
                          M.Options(sv_side=cfg.sv_side, zero_skip=zero_skip)) as r:
         r.set_sinogram(case.y, case.w)
@@ -478,22 +492,21 @@ def test_2d_slice_with_many_svs_does_not_collapse():
     pr = O.Prior(sigma=cfg.sigma, nbhd=8)
     x = np.zeros(cfg.n * cfg.n)
     e = O.error_sinogram(og, Aq, c.y.astype(np.float64), x)
-    O.icd_run(og, pr, Aq, c.w, x, e, 80, seed=3000, zero_skip=True)
+    O.icd_run(og, pr, Aq, c.w, x, e, 120, seed=3000, zero_skip=False)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=8), M.Options(sv_side=5)) as r:
         r.set_sinogram(c.y, c.w)
-        r.reconstruct(80)
+        r.reconstruct(160)
         xg = r.image().ravel().astype(np.float64)
     assert xg.max() > 0.5 * x.max()
-    # both runs zero-skip, whose fixed point is order-dependent (reading R9; 5.9 HU measured at
-    # this low dose): within the paper's own convergence criterion, 10 HU
-    assert O.rmse_hu(xg, x) < 10.0, O.rmse_hu(xg, x)
+    # zero-skip with re-admission (reading R9) reaches the no-skip MAP
+    assert O.rmse_hu(xg, x) < 1.0, O.rmse_hu(xg, x)
 
 
 def test_zero_skip_prefilter_path_matches_oracle():
     """Iterations >= 2 without batching flag fully zero-skipped SV visits per phase and account
     them at task fetch (api.cu / sched.cu k_zero_flags).  A whole-group batch on a 3-D baggage case
     (large air fraction) exercises it: empty visits are reported, the accounting stays consistent
-    and the converged image matches the oracle's zero-skip run (reading R9 bound)."""
+    and the converged image matches the oracle's MAP (1 HU / 1e-4)."""
     cfg = WorkloadConfig("mini3d-bag", 40, 4, 60, 64, 7, 26, 0.002, phantom="baggage")
     case = make_case(cfg, 101)
     g, og = geoms(cfg)
@@ -501,7 +514,7 @@ def test_zero_skip_prefilter_path_matches_oracle():
     pr = O.Prior(sigma=cfg.sigma, nbhd=26)
     x = np.zeros(cfg.nz * cfg.n * cfg.n)
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
-    O.icd_run(og, pr, Aq, case.w, x, e, 120, seed=3000, zero_skip=True)
+    O.icd_run(og, pr, Aq, case.w, x, e, 120, seed=3000, zero_skip=False)
     nvox = cfg.nz * cfg.n * cfg.n
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
                          M.Options(sv_side=cfg.sv_side, batch_svs=1000, batch_threshold=0)) as r:
@@ -516,10 +529,11 @@ def test_zero_skip_prefilter_path_matches_oracle():
         assert empty > 0
         r.reconstruct(200)
         xg = r.image().ravel().astype(np.float64)
-    assert O.rmse_hu(xg, x) < 2.0, O.rmse_hu(xg, x)
+    # the pre-filtered zero-skip path with re-admission (reading R9) reaches the no-skip MAP
+    assert O.rmse_hu(xg, x) < 1.0, O.rmse_hu(xg, x)
     cg = O.cost(og, pr, Aq, case.y, case.w, xg)
     co = O.cost(og, pr, Aq, case.y, case.w, x)
-    assert abs(cg - co) <= 5e-4 * abs(co)
+    assert abs(cg - co) <= 1e-4 * abs(co)
 
 
 @pytest.mark.parametrize("name", ["cfg3", "cfg4"])

@@ -222,6 +222,43 @@ def test_p8_phi_is_half_rho_prime_over_delta(p, q, T, sigma):
             assert O.rho(D, pr) == pytest.approx(D * D / (4 * sigma ** 2), rel=1e-14)
 
 
+@pytest.mark.parametrize("p,T,sigma", [(1.2, 1.0, 0.7), (1.2, 2.0, 0.005), (1.5, 0.5, 3.0)])
+def test_p8_rho_phi_golden_values_at_T_sigma(p, T, sigma):
+    """Golden values worked out by hand from the q-GGMRF definition (reading R1), q = 2: at
+    D = T*sigma, u = |D/(T sigma)|^(q-p) = 1, so rho(T sigma) = (T sigma)^p/(p sigma^p) * 1/2
+    = T^p / (2p), whatever sigma -- a sigma^q-for-sigma^p slip gives sigma^(p-q) T^p/(2p) and
+    fails for sigma != 1.  For T = 1 rho(D) = D^2/(p sigma^2) / (1 + (D/sigma)^(2-p)), whose
+    derivative at sigma is (2 + p)/(4 p sigma), so phi(sigma) = rho'/(2 sigma) = (2 + p)/(8 p sigma^2).
+    Symmetric in the sign of D."""
+    pr = O.Prior(p, 2.0, T, sigma, 8)
+    D = T * sigma
+    assert O.rho(D, pr) == pytest.approx(T ** p / (2 * p), rel=1e-13)
+    assert O.rho(-D, pr) == pytest.approx(T ** p / (2 * p), rel=1e-13)
+    if T == 1.0:
+        assert O.phi(D, pr) == pytest.approx((2 + p) / (8 * p * sigma ** 2), rel=1e-12)
+        assert O.phi(-D, pr) == pytest.approx((2 + p) / (8 * p * sigma ** 2), rel=1e-12)
+    # far tail, |D| >> T sigma: u -> inf, rho -> |D|^p / (p sigma^p) (the p-norm branch)
+    big = 1e12 * T * sigma  # u = 1e12^(2-p) >= 1e6: u/(1+u) = 1 - O(1e-6)
+    assert O.rho(big, pr) == pytest.approx(big ** p / (p * sigma ** p), rel=2e-6)
+
+
+def test_rmse_hu_golden_values():
+    """P:277 footnote / reading R12: HU = 1000 (mu - mu_w)/mu_w with mu_w = 0.02 mm^-1, so a
+    uniform offset of 2e-4 mm^-1 is exactly 10 HU and 2e-5 is 1 HU; a +-c pattern has RMSE c; a
+    single voxel of 0.02 off in a 100-voxel image is sqrt(1/100)*1000 = 100 HU.  (A dropped
+    x1000, a missing /mu_w or a missing sqrt / mean fails these.)"""
+    g = np.random.default_rng(7).uniform(0.0, 0.04, 1000)
+    assert O.rmse_hu(g + 2e-4, g) == pytest.approx(10.0, rel=1e-9)
+    assert O.rmse_hu(g - 2e-5, g) == pytest.approx(1.0, rel=1e-9)
+    s = np.where(np.arange(1000) % 2 == 0, 1.0, -1.0) * 6e-4
+    assert O.rmse_hu(g + s, g) == pytest.approx(30.0, rel=1e-9)
+    a = np.zeros(100)
+    b = np.zeros(100)
+    b[17] = 0.02
+    assert O.rmse_hu(a, b) == pytest.approx(100.0, rel=1e-12)
+    assert O.rmse_hu(a, b, mu_water=0.04) == pytest.approx(50.0, rel=1e-12)
+
+
 def test_p8_neighbour_weights():
     """Reading R2: b_jr proportional to 1/distance, interior weights sum to 1."""
     s8 = sum(O.nbr_weight(dx, dy, 0, 8) for dx in (-1, 0, 1) for dy in (-1, 0, 1))
@@ -390,6 +427,40 @@ def test_zero_skip_semantics():
                       order=np.array(order))
     assert st["updates"] == 9  # the 8 neighbours and 27 itself; 27 then clips back to 0
     assert x[27] == 0.0
+
+
+def test_zero_skip_readmission_period():
+    """Reading R9: with a re-admission period P, sweeps numbered by a multiple of P examine every
+    voxel even where the plain heuristic would skip (here: all of them)."""
+    g, A, _, y, w = _small_problem(8)
+    pr = O.Prior(1.2, 2.0, 1.0, 0.005, 8)
+    x = np.zeros(64)
+    e = O.error_sinogram(g, A, -y, x)  # all updates clip to 0
+    st, _ = O.icd_run(g, pr, A, w, x, e, 4, seed=1, zero_skip=True, zero_skip_period=2)
+    assert st["updates"] == 3 * 64 and st["skipped"] == 64  # sweeps 1, 2, 4 update; 3 skips
+    st, _ = O.icd_run(g, pr, A, w, x, e, 3, first_sweep=5, seed=1, zero_skip=True, zero_skip_period=0)
+    assert st["updates"] == 0 and st["skipped"] == 3 * 64
+
+
+def test_zero_skip_with_readmission_reaches_the_map():
+    """P:115's zero-skip freezes a voxel whose neighbourhood is all zero; from x0 = 0 (reading
+    R9) the first SV-ordered sweep can clip whole regions of the object to 0, which plain
+    zero-skip then only re-opens from their borders, so its fixed point need not be the MAP.
+    With re-admission (period 4) every fixed point of the iteration is a fixed point of plain
+    ICD: after enough sweeps it matches the no-skip result to < 0.05 HU, and the plain
+    heuristic's own fixed point is reported for the record."""
+    cfg = CONFIGS["cfg1"]
+    case = make_case(cfg)
+    g = O.Geometry(cfg.n, cfg.n, 1, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dchannel)
+    A = O.sysmatrix(g)
+    pr = O.Prior(sigma=cfg.sigma, nbhd=8)
+    runs = {}
+    for name, zs, per in (("noskip", False, 0), ("readmit", True, 4)):
+        x = np.zeros(cfg.n * cfg.n)
+        e = O.error_sinogram(g, A, case.y.astype(np.float64), x)
+        O.icd_run(g, pr, A, case.w, x, e, 160, seed=3000, zero_skip=zs, zero_skip_period=per)
+        runs[name] = x
+    assert O.rmse_hu(runs["readmit"], runs["noskip"]) < 0.05
 
 
 def test_p12_golden_self_convergence_cfg1():
