@@ -21,6 +21,12 @@
 
 using namespace mbir;
 
+// views per lane of the update kernel for > 128 views (build-time choice: 4 = six view warps,
+// 2 = twelve)
+#ifndef MBIR_WIDE_VPT
+#define MBIR_WIDE_VPT 4
+#endif
+
 namespace {
 
 // ---- NCCL through dlopen (only needed when nranks > 1) ----
@@ -104,7 +110,6 @@ struct mbir_handle {
     std::vector<cudaEvent_t> kev;  // per-launch event pairs of the update kernel (one iteration)
     int kev_used = 0;
     unsigned long long* d_tprof = nullptr;  // phase cycle counters (env MBIR_PHASE_PROFILE)
-    unsigned long long* d_trace = nullptr;  // per-pair clock trace of one visit (env MBIR_TRACE)
     PriorConst pc{};  // q-GGMRF constants and neighbourhood, passed to every kernel by value
     // per-update record (test hook mbir_set_update_dump): [cap][4] = (voxel, theta1, theta2, delta)
     float* d_dump = nullptr;
@@ -169,7 +174,6 @@ IcdParams make_params(mbir_handle* h)
     p.iter = h->iter;
     p.deterministic = h->o.deterministic;
     p.tprof = h->d_tprof;
-    p.trace = h->d_trace;
     p.pc = h->pc;
     p.dump = h->d_dump;
     p.dump_count = h->d_dump_count;
@@ -218,7 +222,8 @@ int timed_icd(mbir_handle* h, const IcdParams& p, int nnb, bool q, int gx, int g
         }
     }
     CK(cudaEventRecord(h->kev[2 * h->kev_used], h->st));
-    CK(launch_icd(p, h->vpt, nnb, q, h->cl, gx, gy, h->st));
+    (void)gy;
+    CK(launch_svicd(p, h->vpt, nnb, q, gx, h->st));
     CK(cudaEventRecord(h->kev[2 * h->kev_used + 1], h->st));
     h->kev_used++;
     return MBIR_OK;
@@ -316,7 +321,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         const size_t cap = (size_t)h->g.nz_local * h->max_group;
         // deterministic: one CTA (or one cluster) walks the phase list in order (sequential ICD,
         // known order)
-        const int grid = det ? h->cl : target_ctas;
+        const int grid = det ? 1 : target_ctas;
         // iterations >= 2 without batching: the tasks whose whole tile is zero are flagged per
         // phase (sched.cu k_zero_flags) and skipped at task fetch by the update kernel
         const bool prefilter = p.zero_skip_active && nb == 1 && !det;
@@ -406,17 +411,8 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         const double v = (double)(t[5] ? t[5] : 1);
         fprintf(stderr,
                 "[mbir phase] visits %llu voxels %llu | cycles/visit: order %.0f pack %.0f loop %.0f "
-                "writeback %.0f | loop cycles/voxel %.1f | warp0 own pack %.0f (tile0: issue %.0f "
-                "land %.0f stage %.0f)\n",
-                t[5], t[4], t[0] / v, t[1] / v, t[2] / v, t[3] / v, t[2] / (double)(t[4] ? t[4] : 1),
-                t[6] / v, t[7] / v, t[8] / v, t[9] / v);
-        fprintf(stderr, "[mbir phase] barrier wait cycles/visit by warp:");
-        for (int i = 0; i < 8; ++i) fprintf(stderr, " %.0f", t[10 + i] / v);
-        fprintf(stderr, " | producer loop %.0f | view full-wait (records < R, >= R) %.0f %.0f | prior_pair %.0f",
-                t[21] / v, t[22] / v, t[23] / v, t[24] / v);
-        fprintf(stderr, " | TMA issue->ready: blocked waits %llu avg latency %.0f, unblocked %llu avg lead %.0f",
-                t[26], t[25] / (double)(t[26] ? t[26] : 1), t[28], t[27] / (double)(t[28] ? t[28] : 1));
-        fprintf(stderr, "\n");
+                "writeback %.0f | loop cycles/voxel %.1f\n",
+                t[5], t[4], t[0] / v, t[1] / v, t[2] / v, t[3] / v, t[2] / (double)(t[4] ? t[4] : 1));
     }
     return MBIR_OK;
 }
@@ -522,15 +518,7 @@ void mbir_destroy(mbir_handle* h)
                     h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
                     h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count,
                     h->d_flat, h->d_brange, h->d_fetch, h->d_keep, h->d_perm, h->d_counters, h->d_sum_delta,
-                    h->d_flag, h->d_acc, h->d_tprof, h->d_trace, h->d_dump, h->d_dump_count};
-    if (h->d_trace && getenv("MBIR_TRACE")) {  // development aid: raw clock stamps (tools/trace_visit.py)
-        std::vector<unsigned long long> t(1024);
-        cudaMemcpy(t.data(), h->d_trace, 1024 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
-        if (FILE* f = fopen(getenv("MBIR_TRACE"), "wb")) {
-            fwrite(t.data(), sizeof(unsigned long long), t.size(), f);
-            fclose(f);
-        }
-    }
+                    h->d_flag, h->d_acc, h->d_tprof, h->d_dump, h->d_dump_count};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     if (h->h_counters) cudaFreeHost(h->h_counters);
@@ -639,13 +627,12 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     h->A.S2 = h->S2;
     h->A.V = G.nviews;
     // ---- update-kernel shape: fat view warps (4 views per lane, <= 6 warps) keep the per-voxel
-    // per-warp overhead (reduction, barrier, delta) small; tiny view counts use 1 per lane
-    // (2 views per lane in 12 view warps was measured too: 13 warps leave 128 registers per
-    // thread and the gather spills)
-    h->vpt = G.nviews > 128 ? 4 : 1;
+    // per-warp overhead (reduction, barrier, delta) small; <= 128 views use 1 view per lane
+    // (<= 4 warps)
+    h->vpt = G.nviews > 128 ? MBIR_WIDE_VPT : 1;
     h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
     if (h->nvw * h->vpt > 24) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
-    h->Vs = h->nvw * 32 * h->vpt;
+    h->Vs = (h->nvw * 32 * h->vpt + 127) / 128 * 128;  // record stride: whole 128-view tiles
     h->A.vpt = h->vpt;
     h->A.VA = h->Vs;  // thread-major record positions (apos); a multiple of 32 -> TMA-sized
     const size_t nA = (size_t)h->nsv * h->S2 * h->A.VA;
@@ -691,29 +678,20 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
     {
-        // cluster variant (two tasks per SM, each split over a 2-CTA cluster): uint8 A, 4 views
-        // per lane, an even number of view warps, and two CTAs' shared memory fitting one SM
+        // the fused update kernel: nvw view warps + the delta warp + the prior warp, one CTA per SM
         IcdParams p = make_params(h);
-        const int want = h->o.cluster;
-        if (want < 0 || want > 2) return (fail(h, MBIR_EINVAL, "cluster must be 0, 1 or 2"), bail(MBIR_EINVAL));
-        const int smem2 = icd_smem_bytes(p, h->vpt, P.neighborhood, quant, 2);
-        const bool ok2 = quant && h->vpt == 4 && h->nvw % 2 == 0 && h->nvw >= 2 &&
-                         h->S2 <= 32 * (h->nvw / 2 + 1) &&
-                         2 * (smem2 + 1024) <= (int)prop.sharedMemPerMultiprocessor;
-        if (want == 2 && !ok2)
-            return (fail(h, MBIR_EINVAL, "cluster = 2 needs uint8 A, > 128 views in an even number of 128-view warps and two SV buffers per SM"), bail(MBIR_EINVAL));
-        // auto = 1: measured on cfg4, the cluster variant's per-pair DSMEM exchange lengthens the
-        // voxel chain more than splitting the views shortens it
-        h->cl = want == 2 ? 2 : 1;
-        h->threads = 32 * (h->nvw / h->cl + 1);  // view warps + the prior (and A-stream producer) warp
-        if (h->S2 > h->threads) return (fail(h, MBIR_EINVAL, "sv_side^2 exceeds the update kernel's block size"), bail(MBIR_EINVAL));
-        h->smem = icd_smem_bytes(p, h->vpt, P.neighborhood, quant, h->cl);
+        if (h->o.cluster < 0 || h->o.cluster > 1)
+            return (fail(h, MBIR_EINVAL, "cluster must be 0 (auto) or 1: one CTA per SV task"), bail(MBIR_EINVAL));
+        h->cl = 1;
+        h->threads = 32 * (h->nvw + 2);
+        h->smem = svicd_smem_bytes(p, h->vpt, P.neighborhood, quant);
         if (h->smem > (int)prop.sharedMemPerBlockOptin)
             return (fail(h, MBIR_EINVAL, "SV buffer (" + std::to_string(h->smem) + " B) exceeds shared memory: reduce sv_side"), bail(MBIR_EINVAL));
         h->blocks_per_sm = std::max(1, std::min((int)(prop.sharedMemPerMultiprocessor / (h->smem + 1024)),
                                                 (int)(2048 / h->threads)));
-        if (h->cl == 2) h->blocks_per_sm = 2;  // two clusters' CTAs per SM (grid = 2 x 148)
-        h->resident = icd_resident_ctas(p, h->vpt, P.neighborhood, quant, h->cl);
+        h->resident = svicd_resident_ctas(p, h->vpt, P.neighborhood, quant);
+        if (h->resident <= 0) return (fail(h, MBIR_ECUDA, "update kernel does not fit on the device"), bail(MBIR_ECUDA));
+        h->blocks_per_sm = std::max(1, h->resident / h->nsm);
     }
 
     // ---- state buffers
@@ -726,7 +704,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_theta2, (size_t)G.nz_local * h->nsv * h->S2))) return bail(r);
     if ((r = dalloc(h, &h->d_amount, (size_t)G.nz_local * h->nsv))) return bail(r);
     // e_init tiles of the concurrently running SV visits: one per CTA of the largest grid
-    if ((r = dalloc(h, &h->d_scratch, (size_t)h->nsm * h->blocks_per_sm * h->Vs * 32))) return bail(r);
+    if ((r = dalloc(h, &h->d_scratch, (size_t)h->nsm * h->blocks_per_sm * svicd_scratch_floats(h->vpt)))) return bail(r);
     if ((r = dalloc(h, &h->d_task_list, (size_t)G.nz_local * 4 * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_task_count, (size_t)G.nz_local * 4))) return bail(r);
     if ((r = dalloc(h, &h->d_flat, (size_t)8 * G.nz_local * h->max_group))) return bail(r);
@@ -756,10 +734,6 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_sum_delta, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_flag, 1))) return bail(r);
     if ((r = dalloc(h, &h->d_acc, 1))) return bail(r);
-    if (getenv("MBIR_TRACE")) {  // development aid: dumped to the file MBIR_TRACE names by mbir_destroy
-        if ((r = dalloc(h, &h->d_trace, 1024))) return bail(r);
-        cudaMemset(h->d_trace, 0, 1024 * sizeof(unsigned long long));
-    }
     if (getenv("MBIR_PHASE_PROFILE")) {
         if ((r = dalloc(h, &h->d_tprof, 32))) return bail(r);
         cudaMemset(h->d_tprof, 0, 32 * sizeof(unsigned long long));

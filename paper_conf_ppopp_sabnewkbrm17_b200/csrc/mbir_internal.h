@@ -89,12 +89,11 @@ struct IcdParams {
     int zero_skip_active;
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
-    unsigned long long* trace;  // optional per-pair clock trace of one SV visit (env MBIR_TRACE)
     PriorConst pc;           // q-GGMRF constants and neighbourhood of this handle (reading R1-R2)
     float* dump;             // optional [dump_cap][4] (voxel bits, theta1, theta2, delta) per update
     unsigned long long* dump_count;
     long long dump_cap;
-    SmemLayout lay;          // update-kernel smem layout (filled by launch_icd)
+    SmemLayout lay;          // update-kernel smem layout (filled by launch_svicd)
 };
 
 struct SchedParams {
@@ -114,12 +113,12 @@ struct SchedParams {
 cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, int side, int nsvx,
                             int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxoff,
                             cudaStream_t st);
-// cl: CTAs per SV task (1, or 2 = a thread-block cluster splitting the views; uint8 A, vpt 4,
-// an even number of view warps)
-int icd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
-int icd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
-cudaError_t launch_icd(const IcdParams& p, int vpt, int nnb, bool quantize, int cl, int grid_x,
-                       int grid_y, cudaStream_t st);
+// the fused update kernel (svicd.cu): nvw view warps + the delta warp + the prior warp per CTA,
+// vpt = 4 (or 1 for <= 128 views) views per lane
+int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize);
+int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize);
+int svicd_scratch_floats(int vpt);  // per-CTA e_init scratch tile
+cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid, cudaStream_t st);
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st);
 cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cudaStream_t st);
 cudaError_t launch_probe(const IcdParams& p, bool quantize, int nnb, const int64_t* vox, int n,

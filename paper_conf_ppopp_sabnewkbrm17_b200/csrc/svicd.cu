@@ -1,0 +1,1029 @@
+// The fused SuperVoxel ICD update kernel for sm_100a.
+//
+// Paper: Alg. 1 is the per-voxel update; Alg. 3 runs it with
+// intra-voxel, intra-SV and inter-SV parallelism over SV buffers
+// created before and written back after the update.
+//
+// B200 design.  One CTA per SM owns one (slice, SV) task at a time and
+// pulls tasks from the phase list (persistent grid).  Its warps have three roles:
+//   * nvw VIEW warps: view warp w, lane l owns views (w*VPT + t)*32 + l, t < VPT.  The SV buffer
+//     (e and w over the SV's sinogram band) lives in shared memory as rows
+//     [channel offset in band] x [view], e and w rows interleaved (row r of e, then row r of w),
+//     with a row length that is a multiple of 32 views, so a warp's 32 lanes hit 32 distinct
+//     banks for any per-view offsets: conflict-free gathers and scatters, no atomics (a thread is
+//     the only writer of its views).
+//   * the DELTA warp derives the two deltas of each voxel pair (Alg1:7-8, q-GGMRF surrogate,
+//     reading R1) from the view warps' partial sums and the surrogate terms;
+//   * the PRIOR warp computes the next pair's surrogate terms from the shared-memory x tile while
+//     the current pair is in flight.
+// Voxels of the SV are updated in a random order exactly as sequential ICD, two per step: both
+// voxels' theta1 partials are gathered from the same e together with their overlap
+// H = sum w A_b A_a; the delta warp corrects b's theta1 by a's change (theta1_b' = theta1_b +
+// s_b s_a delta_a H) and b's prior if a is its neighbour.  A view thread keeps the pair's
+// dequantised A values, w*A and e in registers from preparation through gather to scatter (no
+// recomputation), and prepares the next pair while the deltas are derived.  A records (uint8
+// codes + band offsets) are streamed R voxels ahead by per-thread cp.async.  theta2 = A^T W A is
+// precomputed per (slice, voxel).  The write-back is delta e = final - e_init per aligned band
+// window with red.global.add.v4.f32 (same-colour SVs share sinogram entries).
+#include "mbir_internal.h"
+
+namespace mbir {
+
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// phi(D) = rho'(D)/(2D) for the q-GGMRF potential with q = 2 (reading R1):
+//   phi = c_phi * (q/p + u) / (1 + u)^2,  u = |D/(T sigma)|^(q-p)   (|D|^(q-2) = 1)
+__device__ __forceinline__ float phi_f(const PriorConst& pc, float d)
+{
+    const float ad = fabsf(d);
+    float u;
+    if (pc.qmp == 0.f)
+        u = 1.f;
+    else
+        u = (ad == 0.f) ? 0.f : exp2f(pc.qmp * __log2f(ad * pc.inv_Ts));
+    const float opu = 1.f + u;
+    return __fdividef(pc.c_phi * (pc.pq + u), opu * opu);
+}
+
+// dequantised codes i, i + 1 of a packed word as a channel pair, via the 2^23 magic (2 PRMT +
+// 1 FADD2, no I2F)
+__device__ __forceinline__ float2 dq2(uint32_t word, int i)
+{
+    const float2 m = make_float2(__uint_as_float(__byte_perm(word, 0x4B000000u, 0x7440u | (uint32_t)i)),
+                                 __uint_as_float(__byte_perm(word, 0x4B000000u, 0x7441u + (uint32_t)i)));
+    return __fadd2_rn(m, make_float2(-8388608.f, -8388608.f));
+}
+
+// vector atomic add of 4 consecutive floats (16-byte aligned), sm_90+
+__device__ __forceinline__ void red_add_v4(float* p, float a, float b, float c, float d)
+{
+    asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(a), "f"(b), "f"(c), "f"(d)
+                 : "memory");
+}
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z)
+{
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+// per-thread asynchronous global -> shared copies (LDGSTS), tracked per thread by commit groups
+__device__ __forceinline__ void cp_async16(void* dst, const void* src)
+{
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* dst, const void* src)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* dst, const void* src)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait()
+{
+    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+// named barriers: sync (wait for `n` threads incl. this warp) / arrive (count and go on)
+__device__ __forceinline__ void bar_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+__device__ __forceinline__ void bar_arrive(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
+// A values of a voxel re-indexed to another voxel's channels: r[i] = A[i + d] (0 outside), as
+// channel pairs
+template <bool U8>
+__device__ __forceinline__ void shifted(uint32_t cw, const float2 (&a)[2], int d, float2 (&r)[2])
+{
+    if (U8) {
+        // one PRMT: byte i of s = byte i + d of cw, or 0 (selector nibble 4 = byte 0 of the zero
+        // operand); the selector nibbles are read out of 0x444432104444 at nibble 4 + d
+        const int dc = max(-4, min(4, d));
+        const uint32_t sel = (uint32_t)(0x444432104444ull >> (16 + 4 * dc));
+        const uint32_t s = __byte_perm(cw, 0u, sel);
+        r[0] = dq2(s, 0);
+        r[1] = dq2(s, 2);
+        return;
+    }
+    const float v[4] = {a[0].x, a[0].y, a[1].x, a[1].y};
+    float q[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int j = i + d;
+        q[i] = j == 0 ? v[0] : j == 1 ? v[1] : j == 2 ? v[2] : j == 3 ? v[3] : 0.f;
+    }
+    r[0] = make_float2(q[0], q[1]);
+    r[1] = make_float2(q[2], q[3]);
+}
+
+// Neighbour slots of a prior-warp lane: half-warp h = lane >> 4 works on voxel a (h = 0) or b
+// (h = 1) of a pair; its lane i owns neighbours i and i + 16 of the neighbourhood (reading R2):
+// offset (dx, dy, dz), tile-index offset dt and weight w (0: no neighbour)
+struct NbrLane {
+    int dx[2], dy[2], dz[2], dt[2];
+    float w[2];
+};
+
+// surrogate terms of a pair of consecutive voxels (a, b): a's sums, b's sums computed with a's
+// OLD value, and -- if a is b's neighbour -- that neighbour's term (btab) and weight (bab)
+struct PriPair {
+    float sa, sxa, va, sb, sxb, vb, btab, bab;
+};
+
+// prior warp: PriPair for voxels (i0, i0+1) of the visiting order from the current x tile.
+// Alg1:7's q-GGMRF surrogate sums sb = sum_r b_r phi(v - x_r), sx = sum_r b_r phi(v - x_r) x_r
+// over the neighbourhood (free boundary: off-volume neighbours contribute nothing), voxel a on
+// lanes 0-15 and voxel b (with a's OLD value) on lanes 16-31, two neighbours per lane.
+__device__ __forceinline__ void prior_pair(const int* tof, int i0, int nact, const float* xt, int cslot,
+                                           int TW, int gx0, int gy0, int zg, const IcdParams& P,
+                                           const NbrLane& nb, int lane, PriPair* out)
+{
+    const bool hasb = i0 + 1 < nact;
+    const int ta = tof[i0], tb = hasb ? tof[i0 + 1] : ta;
+    const int tv = lane < 16 ? ta : tb;
+    const int lx = tv & 255, ly = tv >> 8;
+    const int c0 = cslot + ly * TW + lx;
+    const float v = xt[c0];
+    float sb = 0.f, sx = 0.f, btn = 0.f, bwn = 0.f;  // btn, bwn: this lane's term / weight whose
+    bool mine = false;                               // neighbour is voxel a
+    const int dxa = (ta & 255) - lx, dya = (ta >> 8) - ly;  // a relative to this half's voxel
+    float xr[2];
+    bool ok[2];
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const int gx = gx0 + lx + nb.dx[k], gy = gy0 + ly + nb.dy[k], gz = zg + nb.dz[k];
+        ok[k] = nb.w[k] != 0.f && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total;
+        xr[k] = xt[c0 + nb.dt[k]];  // always inside the tile (its ring covers the neighbourhood)
+    }
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const float bt = ok[k] ? nb.w[k] * phi_f(P.pc, v - xr[k]) : 0.f;
+        sb += bt;
+        sx += bt * xr[k];
+        if (ok[k] && nb.dz[k] == 0 && nb.dx[k] == dxa && nb.dy[k] == dya) {
+            btn = bt;
+            bwn = nb.w[k];
+            mine = true;
+        }
+    }
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) {
+        sb += __shfl_xor_sync(kFull, sb, o);
+        sx += __shfl_xor_sync(kFull, sx, o);
+    }
+    // a's neighbour term in b's sums (a and b are distinct voxels, so only lanes >= 16 can own it)
+    const unsigned who = __ballot_sync(kFull, mine && lane >= 16 && hasb);
+    const int src = who ? __ffs(who) - 1 : 0;
+    const float btab = __shfl_sync(kFull, btn, src);
+    const float bab = __shfl_sync(kFull, bwn, src);
+    const float sbb = __shfl_sync(kFull, sb, 16), sxb = __shfl_sync(kFull, sx, 16), vb = __shfl_sync(kFull, v, 16);
+    if (lane == 0) {
+        PriPair pp{sb, sx, v, 0.f, 0.f, 0.f, 0.f, 0.f};
+        if (hasb) {
+            pp.sb = sbb;
+            pp.sxb = sxb;
+            pp.vb = vb;
+            if (who) {
+                pp.btab = btab;
+                pp.bab = bab;
+            }
+        }
+        *out = pp;
+    }
+}
+
+__host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
+
+// row stride (floats) of a view warp's 32-row transpose staging tile: 16-byte rows, so a lane moves
+// 4 window positions with one STS.128 / LDS.128; every quarter-warp (one shared-memory wavefront
+// of a 128-bit access) then touches 8 distinct 4-bank groups, on the put and on the read
+constexpr int kStg = 36;
+
+// SV-buffer geometry: VS = view columns (compile-time: 4 views per lane x 6 warps, or 1 x 4),
+// rows of e and w interleaved, so e row r sits at float offset 2 r VS and w row r at (2 r + 1) VS:
+// a thread reaches all four channels of a voxel's record in both arrays with immediate offsets
+// from one address
+__host__ __device__ constexpr int svb_cols(int vpt) { return vpt == 1 ? 128 : 768; }
+
+constexpr int kNSL = 16;  // partial-sum slots per quantity in the pair exchange (>= view warps)
+
+// the pack and the write-back move 32-view tiles; tile warp w (< VA / 128: the record stride VA
+// is a multiple of 128) handles tiles 4w ... 4w + 3 whatever the voxel loop's view ownership
+// (those phases are bracketed by CTA barriers), so the staging area is sized for <= 6 tile warps
+constexpr int kTileW = 4;
+__host__ __device__ constexpr int tile_warps(int va) { return va / (32 * kTileW); }
+
+// threads per CTA: VPT 4 -> <= 6 view warps, VPT 2 -> <= 12, VPT 1 -> <= 4; + delta + prior warps
+__host__ __device__ constexpr int max_threads(int vpt) { return vpt == 2 ? 448 : 256; }
+
+// named barriers of the pair protocol (0 is __syncthreads)
+constexpr int kBarA = 1;  // view warps' partials + the prior warp's terms of a pair are ready
+constexpr int kBarB = 2;  // the delta warp has published the pair's deltas
+constexpr int kBarX = 3;  // the delta warp has written the pair's new values into the x tile
+
+// A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
+__host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, int nnb, int VA, bool u8,
+                                                   int nstage, int nvw, int vpt)
+{
+    SmemLayout L;
+    const int TW = side + 2;
+    const int nzt = nnb == 26 ? 3 : 1;
+    int o = 0;
+    L.sb_e = o;  o = align16(o + 2 * rows * svb_cols(vpt) * 4);  // e / w rows interleaved
+    L.sb_w = L.sb_e + svb_cols(vpt) * 4;
+    L.xt = o;    o = align16(o + nzt * TW * TW * 4);
+    L.list = o;  o = align16(o + S2 * 4);
+    L.flags = o; o = align16(o + S2 * 4);
+    L.tof = o;   o = align16(o + S2 * 4);
+    L.red = o;   o = align16(o + 2 * 3 * kNSL * 4);  // [2 bufs][3 quantities][kNSL view warps]
+    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriPair));
+    L.vscale = o; o = align16(o + S2 * 4);
+    L.vth2 = o;  o = align16(o + S2 * 4);
+    L.misc = o;  o = align16(o + 16 * 4);
+    L.off_in_stage = VA * (u8 ? 4 : 16);
+    L.stage_bytes = align16(L.off_in_stage + VA);
+    // the A-record ring (voxel loop) and the transpose staging tiles (pack, write-back) are never
+    // live at the same time: they share one region
+    L.astage = o;
+    L.staging = o;
+    o = align16(o + max(nstage * L.stage_bytes, tile_warps(VA) * 32 * kStg * 4));
+    L.mbar = o;  o = align16(o + 4 * 32 * 4);  // neighbour tables [dx | dy | dz | b][32]
+    L.binfo = o; o = align16(o + 2 * VA * 4);  // band (row offset << 5 | width), 2 tasks
+    L.total = o;
+    return L;
+}
+
+// band of task tk for views k = k0, k0 + stride, ... < V into dst[k] = (k*M + start) << 5 | width
+__device__ __forceinline__ void band_info(const IcdParams& P, int tk, uint32_t* dst, int k0, int stride)
+{
+    const int sv = tk & 16383;
+    for (int k = k0; k < P.V; k += stride) {
+        const int r = k * P.M + P.A.band_start[(size_t)sv * P.V + k];
+        const int wd = P.A.band_width[(size_t)sv * P.V + k];
+        dst[k] = ((uint32_t)r << 5) | (uint32_t)wd;
+    }
+}
+
+// this thread's VPT adjacent records from a stage as raw words (CW = 1: a uint8 code word per
+// view; CW = 4: fp32 values), and the band offsets packed in one word (VPT bytes)
+template <int VPT, int CW>
+__device__ __forceinline__ void load_words(const unsigned char* stg, int off_in_stage, int tp,
+                                           uint32_t (&c)[VPT][CW], uint32_t& ob)
+{
+    if (CW == 1 && VPT == 4) {
+        const uint4 c4 = ((const uint4*)stg)[tp];
+        c[0][0] = c4.x;
+        c[VPT > 1 ? 1 : 0][0] = c4.y;
+        c[VPT > 2 ? 2 : 0][0] = c4.z;
+        c[VPT > 3 ? 3 : 0][0] = c4.w;
+    } else if (CW == 1 && VPT == 2) {
+        const uint2 c2 = ((const uint2*)stg)[tp];
+        c[0][0] = c2.x;
+        c[VPT > 1 ? 1 : 0][0] = c2.y;
+    } else {
+#pragma unroll
+        for (int t = 0; t < VPT; ++t) {
+            if (CW == 4) {
+                const uint4 v = ((const uint4*)stg)[tp * VPT + t];
+                c[t][0] = v.x;
+                c[t][CW > 1 ? 1 : 0] = v.y;
+                c[t][CW > 2 ? 2 : 0] = v.z;
+                c[t][CW > 3 ? 3 : 0] = v.w;
+            } else {
+                c[t][0] = ((const uint32_t*)stg)[tp * VPT + t];
+            }
+        }
+    }
+    if (VPT == 4) ob = ((const uint32_t*)(stg + off_in_stage))[tp];
+    if (VPT == 2) ob = ((const uint16_t*)(stg + off_in_stage))[tp];
+    if (VPT == 1) ob = stg[off_in_stage + tp];
+}
+
+// The update kernel.  VPT views per lane (4, or 1 for <= 128 views), uint8 or fp32 A, 8 or 26
+// neighbours, R-voxel A-record ring; PROF adds per-phase cycle counters.
+template <int VPT, bool U8, int NNB, int R, bool PROF>
+__global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P)
+{
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int nvw = P.nvw;                 // view warps
+    const bool is_view = warp < nvw, is_delta = warp == nvw, is_prior = warp == nvw + 1;
+    const int vw = is_view ? warp : 0;
+    const int V = P.V, M = P.M, S2 = P.S2, side = P.side;
+    const int VA = P.A.VA;                 // record positions / SVB columns in use
+    constexpr int VS = svb_cols(VPT);      // SVB row length (compile-time: row offsets are immediates)
+    constexpr int RS = 2 * VS;             // float stride between consecutive e (or w) rows
+    const SmemLayout& L = P.lay;
+    float* sb = (float*)(smem + L.sb_e);   // e row r at sb + r RS, w row r at sb + r RS + VS
+    float* xt = (float*)(smem + L.xt);
+    int* list = (int*)(smem + L.list);
+    int* flags = (int*)(smem + L.flags);
+    int* tof = (int*)(smem + L.tof);       // visiting order as packed (ly << 8 | lx)
+    float* red = (float*)(smem + L.red);
+    PriPair* pri = (PriPair*)(smem + L.pri);
+    float* vscale = (float*)(smem + L.vscale);
+    float* vth2 = (float*)(smem + L.vth2);
+    unsigned char* astage = smem + L.astage;
+    float* stg_w = (float*)(smem + L.staging) + vw * 32 * kStg;
+    int* s_task = (int*)(smem + L.misc);            // [0] first task, [1 + (n & 1)] the task after n
+    float* dslot = (float*)(smem + L.misc) + 4;     // [2 pairs][2]: scale_a delta_a, scale_b delta_b
+    uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA]
+    const int TW = side + 2;
+    const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
+    const size_t plane = (size_t)P.nx * P.ny;
+    const int nab = (nvw + 2) * 32;      // barrier A: view warps + delta warp + prior warp
+    const int nb2 = (nvw + 1) * 32;      // barrier B: view warps + the delta warp
+
+    for (int i = threadIdx.x; i < 2 * 3 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
+    // the neighbourhood (reading R2) as shared-memory tables [dx | dy | dz | weight bits][32]: a
+    // by-value kernel parameter indexed by a run-time value would be copied to local memory
+    int* nbt = (int*)(smem + L.mbar);
+    for (int i = threadIdx.x; i < 32; i += blockDim.x) {
+        const bool ok = i < P.pc.nnb;
+        nbt[i] = ok ? P.pc.dx[i] : 0;
+        nbt[32 + i] = ok ? P.pc.dy[i] : 0;
+        nbt[64 + i] = ok ? P.pc.dz[i] : 0;
+        nbt[96 + i] = ok ? __float_as_int(P.pc.b[i]) : 0;
+    }
+    __syncthreads();
+    // SVB rows outside a visit's band are never packed: start them finite (zero)
+    for (int i = threadIdx.x; i < (L.xt - L.sb_e) / 16; i += blockDim.x)
+        ((float4*)(smem + L.sb_e))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    // per-thread view ownership: view warp w, lane l owns views (w*VPT + t)*32 + l
+    int kv[VPT];
+#pragma unroll
+    for (int t = 0; t < VPT; ++t) kv[t] = (vw * VPT + t) * 32 + lane;
+    uint32_t gseq = 0;  // running voxel sequence number of this CTA: A stage = gseq % R
+    uint32_t pseq = 0;  // running voxel-pair number: exchange buffers pseq & 1
+    // prior-warp lane r owns neighbour r (and r + 16): offsets and weights in registers
+    NbrLane nb;
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const int r = (lane & 15) + 16 * k;
+        nb.dx[k] = nbt[r];
+        nb.dy[k] = nbt[32 + r];
+        nb.dz[k] = nbt[64 + r];
+        nb.w[k] = __int_as_float(nbt[96 + r]);
+        nb.dt[k] = (nb.dz[k] * (side + 2) + nb.dy[k]) * (side + 2) + nb.dx[k];
+    }
+
+    // this launch's batch: flat tasks [start, end) of the phase list (sched.cu k_flatten), pulled
+    // one at a time by the persistent CTAs (dynamic distribution, Alg3:4 / T3); with the zero-skip
+    // pre-filter (P.keep), tasks whose whole tile is zero are accounted as skipped visits here
+    const int tstart = P.brange[0], tend = P.brange[1];
+    auto fetch_task = [&]() {
+        int q = tstart + atomicAdd(P.fetch, 1);
+        while (P.keep && q < tend && !P.keep[q]) {
+            const int tkq = P.flat[q];
+            const int zq = tkq >> 14, svq = tkq & 16383;
+            const int twq = min(side, P.nx - (svq % P.nsvx) * side), thq = min(side, P.ny - (svq / P.nsvx) * side);
+            P.sv_amount[(size_t)zq * P.nsv + svq] = 0.f;
+            atomicAdd(P.counters + 1, (unsigned long long)(twq * thq));
+            atomicAdd(P.counters + 2, 1ull);
+            atomicAdd(P.counters + 3, 1ull);
+            q = tstart + atomicAdd(P.fetch, 1);
+        }
+        return q;
+    };
+    if (threadIdx.x == 0) s_task[0] = fetch_task();
+    __syncthreads();
+    int q = s_task[0];
+    if (q < tend) band_info(P, P.flat[q], binfo, threadIdx.x, blockDim.x);
+    int tb = 0;     // binfo buffer of the current task
+    int nslot = 1;  // s_task slot of the next task
+    for (;; q = s_task[nslot], nslot ^= 3, tb ^= 1) {
+        if (q >= tend) break;
+        const int tk = P.flat[q];
+        const int z = tk >> 14, sv = tk & 16383;  // local slice, SV
+        const int zg = P.z_offset + z;            // global slice
+        const int gx0 = (sv % P.nsvx) * side, gy0 = (sv / P.nsvx) * side;
+        const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
+        long long tp0 = 0, tp1 = 0, tp2 = 0, tp3 = 0;
+        if (PROF && threadIdx.x == 0) tp0 = clock64();
+
+        // ---- 1. x tile (+1 halo ring, +-1 slice in 3-D) into shared memory
+        {
+            constexpr int XMAX = 2;  // tile entries per thread and round: all loads in flight
+            const int ntile = (NNB == 26 ? 3 : 1) * TW * TW;
+            for (int i0 = 0; i0 < ntile; i0 += XMAX * blockDim.x) {
+                float xv[XMAX];
+                bool inb[XMAX];
+#pragma unroll
+                for (int u = 0; u < XMAX; ++u) {
+                    const int i = i0 + threadIdx.x + u * blockDim.x;
+                    const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
+                    const int gx = gx0 - 1 + tx, gy = gy0 - 1 + ty;
+                    const int zs = (NNB == 26) ? z + tz : z + 1;  // storage slice (halo at 0, nz+1)
+                    inb[u] = i < ntile && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny;
+                    const int cx = min(max(gx, 0), P.nx - 1), cy = min(max(gy, 0), P.ny - 1);
+                    xv[u] = i < ntile ? P.x[(size_t)min(zs, P.nz_local + 1) * plane + (size_t)cy * P.nx + cx] : 0.f;
+                }
+#pragma unroll
+                for (int u = 0; u < XMAX; ++u) {
+                    const int i = i0 + threadIdx.x + u * blockDim.x;
+                    if (i < ntile) xt[i] = inb[u] ? xv[u] : 0.f;
+                }
+            }
+        }
+        __syncthreads();
+
+        // ---- 2. zero-skip predicate at visit start (reading R9): slot v kept iff valid
+        //         and (skip inactive or x_j or an in-volume neighbour is non-zero)
+        int kept = 0;
+        for (int v0 = threadIdx.x; v0 < S2; v0 += blockDim.x) {
+            const int lx = v0 % side, ly = v0 / side;
+            int keep = 0;
+            if (lx < tw && ly < th) {
+                keep = 1;
+                if (P.zero_skip_active) {
+                    keep = xt[(zc * TW + ly + 1) * TW + lx + 1] != 0.f;
+                    for (int r = 0; r < P.pc.nnb && !keep; ++r) {
+                        const int dx = nbt[r], dy = nbt[32 + r], dz = nbt[64 + r];
+                        const int gx = gx0 + lx + dx, gy = gy0 + ly + dy, gz = zg + dz;
+                        if (gx < 0 || gx >= P.nx || gy < 0 || gy >= P.ny || gz < 0 || gz >= P.nz_total) continue;
+                        keep = xt[((zc + dz) * TW + ly + 1 + dy) * TW + lx + 1 + dx] != 0.f;
+                    }
+                }
+            }
+            flags[v0] = keep;
+            kept += keep;
+        }
+        if (!__syncthreads_or(kept)) {  // the whole SV is zero-skipped: account for it, next task
+            if (threadIdx.x == 0) {
+                P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
+                atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
+                atomicAdd(P.counters + 2, 1ull);
+                atomicAdd(P.counters + 3, 1ull);
+                s_task[nslot] = fetch_task();
+            }
+            __syncthreads();
+            if (s_task[nslot] < tend) band_info(P, P.flat[s_task[nslot]], binfo + (tb ^ 1) * VA, threadIdx.x, blockDim.x);
+            continue;  // the next task's x-tile barrier orders these writes before its pack
+        }
+
+        // ---- 3. visiting order (prior warp): one of NPERM host-drawn random permutations of the
+        //         tile, chosen per (seed, iteration, slice, SV) visit (raster order in
+        //         deterministic mode), compacted to the kept voxels with a warp ballot; per-voxel
+        //         scale and theta2 staged in smem; then the first pair's surrogate terms.
+        //         Delta warp: the next task.  View warps: the first R A records, then the pack.
+        const size_t arec = (size_t)sv * S2;  // first A record of this SV
+        constexpr int CB = U8 ? 4 : 16;       // record bytes per view position
+        const int tpm = vw * 32 + lane;
+        const unsigned char* g_code = (const unsigned char*)(U8 ? (const void*)P.A.codes : (const void*)P.A.vals) +
+                                      ((size_t)arec * VA + tpm * VPT) * CB;
+        const unsigned char* g_off = P.A.off + (size_t)arec * VA + tpm * VPT;
+        int nvis = 0;  // kept voxels of this visit (every warp computes it)
+        for (int base = 0; base < S2; base += 32) nvis += __popc(__ballot_sync(kFull, base + lane < S2 && flags[base + lane]));
+        const int nactv = nvis;
+        // view thread: asynchronous copy of its own slice of voxel j's record into ring stage stg,
+        // one commit group per voxel (empty past the visit's end)
+        auto copy_record_to = [&](int j, int stg, int v) {
+            if (j < nactv) {
+                unsigned char* st = astage + stg * L.stage_bytes;
+                const unsigned char* gc = g_code + (size_t)v * (VA * CB);
+                if (U8) {
+                    if (VPT == 4)
+                        cp_async16(st + tpm * 16, gc);
+                    else if (VPT == 2)
+                        cp_async8(st + tpm * 8, gc);
+                    else
+                        cp_async4(st + tpm * 4, gc);
+                } else {
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t) cp_async16(st + (tpm * VPT + t) * 16, gc + t * 16);
+                }
+                if ((tpm & (4 / VPT - 1)) == 0)  // offsets: VPT bytes per thread, as 4-byte words
+                    cp_async4(st + L.off_in_stage + tpm * VPT, g_off + (size_t)v * VA);
+            }
+            cp_async_commit();
+        };
+        const int sbase = (int)(gseq % (uint32_t)R);  // ring stage of this visit's voxel 0
+        const int cslot = (zc * TW + 1) * TW + 1;     // tile index of local (0,0)
+        if (is_prior) {
+            const uint64_t h = mix64(P.seed ^ mix64(((uint64_t)P.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)sv));
+            const uint8_t* perm = P.perm + (size_t)(h % (uint64_t)P.nperm) * S2;
+            int n = 0;
+            for (int base = 0; base < S2; base += 32) {
+                const int i = base + lane;
+                const int v = i < S2 ? (P.deterministic ? i : (int)perm[i]) : 0;
+                const bool k = i < S2 && flags[v];
+                const unsigned m = __ballot_sync(kFull, k);
+                if (k) {
+                    const int p = n + __popc(m & ((1u << lane) - 1));
+                    list[p] = v;
+                    tof[p] = ((v / side) << 8) | (v % side);  // packed (ly, lx): no div in the loop
+                }
+                n += __popc(m);
+            }
+            __syncwarp();
+            for (int i = lane; i < nactv; i += 32) {
+                const int v = list[i];
+                vscale[i] = P.A.scale[arec + v];
+                vth2[i] = P.theta2[((size_t)z * P.nsv + sv) * S2 + v];
+            }
+            prior_pair(tof, 0, nactv, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + (pseq & 1));
+            __syncwarp();
+        } else if (is_delta) {
+            if (lane == 0) s_task[nslot] = fetch_task();
+        }
+        if (PROF && threadIdx.x == 0) tp1 = clock64();
+
+        // ---- 4. view warps: SVB pack (coalesced band-row windows transposed through staging
+        //         tiles); e_init rows go to this CTA's L2-resident scratch tile for the write-back
+        float* scr = P.scratch + (size_t)blockIdx.x * (size_t)VS * 32;
+        const int ntw = tile_warps(VA);
+        if (is_view && vw < ntw) {
+            const float* wz = P.w + (size_t)z * V * M;
+            float* ez = P.e + (size_t)z * V * M;
+            // Each band row is read as the 16-byte-aligned 32-float window that contains it (the
+            // slice base is 16-byte aligned, V*M % 4 == 0): 8 lanes x float4 per row, 4 rows per
+            // LDG.128; the window goes through the warp's staging tile and band column
+            // c = p - s_k lands in sb row c, column k (bank k)
+            const int sub = lane >> 3, ch = lane & 7;  // row-in-quad and float4 chunk of this lane
+            auto issue = [&](int t, bool isw, float4 (&v4)[8]) {
+                const int kk = (vw * kTileW + t) * 32 + lane;
+                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const int rot = (int)(bi >> 5);
+#pragma unroll
+                for (int m = 0; m < 8; ++m) {
+                    const int oi = __shfl_sync(kFull, rot, 4 * m + sub);
+                    // unconditional loads: the whole aligned window is read (padded views read the
+                    // slice start; the sinogram allocations carry 32 floats of tail padding)
+                    const size_t a4 = (size_t)(oi - (oi & 3)) + 4 * ch;
+                    v4[m] = isw ? __ldg((const float4*)(wz + a4)) : __ldcg((const float4*)(ez + a4));
+                }
+            };
+            auto finish = [&](int t, bool isw, const float4 (&v4)[8]) {
+                const int k0 = (vw * kTileW + t) * 32;
+                const int kk = k0 + lane;
+                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const int bwt = (int)(bi & 31u), sk = (int)(bi >> 5) & 3;
+                const uint32_t bmask = ((1u << bwt) - 1u) << sk;  // band's window positions
+                if (!isw) {
+#pragma unroll
+                    for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), v4[m]);
+                }
+                float* d = sb + (isw ? VS : 0) + kk - sk * RS;  // + p RS = band row p - sk of view kk
+#pragma unroll
+                for (int m = 0; m < 8; ++m) *(float4*)(stg_w + (4 * m + sub) * kStg + 4 * ch) = v4[m];
+                __syncwarp();
+#pragma unroll
+                for (int q4 = 0; q4 < 8; ++q4) {
+                    const float4 r = *(const float4*)(stg_w + lane * kStg + 4 * q4);
+                    const float rv[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        if (bmask & (1u << (4 * q4 + j))) d[(4 * q4 + j) * RS] = rv[j];
+                }
+                __syncwarp();
+            };
+            float4 wa4[2][8], ea4[2][8];
+            issue(0, true, wa4[0]);
+            issue(0, false, ea4[0]);
+#pragma unroll
+            for (int t = 0; t < kTileW; ++t) {
+                if (t + 1 < kTileW) {
+                    issue(t + 1, true, wa4[(t + 1) & 1]);
+                    issue(t + 1, false, ea4[(t + 1) & 1]);
+                }
+                finish(t, true, wa4[t & 1]);
+                finish(t, false, ea4[t & 1]);
+            }
+        }
+        __syncthreads();
+        if (PROF && threadIdx.x == 0) tp2 = clock64();
+
+        // ---- 5. the voxel loop, TWO voxels (a, b) per step, exactly sequential ICD
+        float amount = 0.f;
+        const int npair = (nactv + 1) >> 1;
+        if (is_view) {
+            const int tp = tpm;
+            constexpr int CW = U8 ? 1 : 4;  // record words per view
+            // Per-pair state of a view thread for its VPT views: band offsets of a and b (packed
+            // bytes), smem addresses of their first rows, the dequantised A of a, of b, and of a
+            // on b's channels, w*A of both, and this lane's part of H = sum w A_b A_a.
+            struct PairState {
+                uint32_t oa, ob;
+                int pa[VPT], pb[VPT];        // float index of (row offset, view) in sb
+                float2 fa[VPT][2], fb[VPT][2], fab[VPT][2];
+                float2 wa[VPT][2], wb[VPT][2];
+                float hh;
+                int sj;                      // ring stage of the pair's first voxel
+            };
+            auto avals = [&](const uint32_t (&c)[CW], float2 (&f)[2]) {
+                if (U8) {
+                    f[0] = dq2(c[0], 0);
+                    f[1] = dq2(c[0], 2);
+                } else {
+                    f[0] = make_float2(__uint_as_float(c[0]), __uint_as_float(c[CW > 1 ? 1 : 0]));
+                    f[1] = make_float2(__uint_as_float(c[CW > 2 ? 2 : 0]), __uint_as_float(c[CW > 3 ? 3 : 0]));
+                }
+            };
+            auto off_of = [&](uint32_t packed, int t) { return (int)((packed >> (8 * t)) & 255u); };
+            // voxels j, j + 1 of the visiting order -> ps.  A pair without a second voxel (the last
+            // step of an odd visit, hb = false) gets a dummy b with zero A on a's channels: its
+            // theta1 and H vanish, its delta is 0 and its scatter rewrites a's entries with the
+            // same values.
+            auto prep = [&](int j, bool hb, PairState& ps) {
+                cp_async_wait<R - 2>();      // this thread's copies of voxels j, j + 1 have landed
+                if (VPT != 4) __syncwarp();  // offset words copied by another lane of the warp
+                const int s1 = ps.sj + 1 == R ? 0 : ps.sj + 1;
+                uint32_t ca[VPT][CW], cb[VPT][CW];
+                load_words<VPT, CW>(astage + ps.sj * L.stage_bytes, L.off_in_stage, tp, ca, ps.oa);
+                load_words<VPT, CW>(astage + s1 * L.stage_bytes, L.off_in_stage, tp, cb, ps.ob);
+                ps.ob = hb ? ps.ob : ps.oa;
+                float2 h2[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+#pragma unroll
+                for (int t = 0; t < VPT; ++t) {
+#pragma unroll
+                    for (int c = 0; c < CW; ++c) cb[t][c] = hb ? cb[t][c] : 0u;
+                    avals(ca[t], ps.fa[t]);
+                    avals(cb[t], ps.fb[t]);
+                    const int oa = off_of(ps.oa, t), ob = off_of(ps.ob, t);
+                    shifted<U8>(ca[t][0], ps.fa[t], ob - oa, ps.fab[t]);  // A_a on b's channels
+                    ps.pa[t] = oa * RS + kv[t];
+                    ps.pb[t] = ob * RS + kv[t];
+                    const float* pw = sb + VS + ps.pa[t];
+                    const float* qw = sb + VS + ps.pb[t];
+                    ps.wa[t][0] = __fmul2_rn(make_float2(pw[0], pw[RS]), ps.fa[t][0]);
+                    ps.wa[t][1] = __fmul2_rn(make_float2(pw[2 * RS], pw[3 * RS]), ps.fa[t][1]);
+                    ps.wb[t][0] = __fmul2_rn(make_float2(qw[0], qw[RS]), ps.fb[t][0]);
+                    ps.wb[t][1] = __fmul2_rn(make_float2(qw[2 * RS], qw[3 * RS]), ps.fb[t][1]);
+                    h2[t & 1] = __ffma2_rn(ps.wb[t][0], ps.fab[t][0], h2[t & 1]);
+                    h2[t & 1] = __ffma2_rn(ps.wb[t][1], ps.fab[t][1], h2[t & 1]);
+                }
+                const float2 hs = __fadd2_rn(h2[0], h2[1]);
+                ps.hh = hs.x + hs.y;
+            };
+            // refill two ring stages with the records R voxels ahead (one commit group per voxel,
+            // empty past the visit's end, keeps the wait counts fixed)
+            auto refill = [&](int j, int sj) {
+                const int s1 = sj + 1 == R ? 0 : sj + 1;
+                copy_record_to(j + R, sj, j + R < nactv ? list[j + R] : 0);
+                copy_record_to(j + 1 + R, s1, j + 1 + R < nactv ? list[j + 1 + R] : 0);
+            };
+            // one voxel pair: theta1 partials from e -> barrier A -> the next pair's state ->
+            // barrier B (deltas) -> scatter
+            auto pair_step = [&](int idx, PairState& cur, PairState& nxt) {
+                const uint32_t pn = pseq + (uint32_t)(idx >> 1);  // running pair number
+                float2 ea[VPT][2], eb[VPT][2];
+                {
+                    float2 acc[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+                    float2 accb[2] = {acc[0], acc[0]};
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t) {
+                        const float* pe = sb + cur.pa[t];
+                        const float* qe = sb + cur.pb[t];
+                        ea[t][0] = make_float2(pe[0], pe[RS]);
+                        ea[t][1] = make_float2(pe[2 * RS], pe[3 * RS]);
+                        eb[t][0] = make_float2(qe[0], qe[RS]);
+                        eb[t][1] = make_float2(qe[2 * RS], qe[3 * RS]);
+                        acc[t & 1] = __ffma2_rn(cur.wa[t][0], ea[t][0], acc[t & 1]);
+                        acc[t & 1] = __ffma2_rn(cur.wa[t][1], ea[t][1], acc[t & 1]);
+                        accb[t & 1] = __ffma2_rn(cur.wb[t][0], eb[t][0], accb[t & 1]);
+                        accb[t & 1] = __ffma2_rn(cur.wb[t][1], eb[t][1], accb[t & 1]);
+                    }
+                    const float2 ac = __fadd2_rn(acc[0], acc[1]), acb = __fadd2_rn(accb[0], accb[1]);
+                    float2 gab = make_float2(ac.x + ac.y, acb.x + acb.y);
+                    float hh = cur.hh;
+#pragma unroll
+                    for (int o = 16; o > 0; o >>= 1) {
+                        const float2 r = make_float2(__shfl_xor_sync(kFull, gab.x, o), __shfl_xor_sync(kFull, gab.y, o));
+                        hh += __shfl_xor_sync(kFull, hh, o);
+                        gab = __fadd2_rn(gab, r);
+                    }
+                    if (lane == 0) {
+                        float* rs = red + (pn & 1) * 3 * kNSL + vw;
+                        rs[0] = gab.x;
+                        rs[kNSL] = gab.y;
+                        rs[2 * kNSL] = hh;
+                    }
+                }
+                bar_arrive(kBarA, nab);
+                // meanwhile: the next pair's e-independent state, then refill its freed stages
+                nxt.sj = cur.sj + 2 >= R ? cur.sj + 2 - R : cur.sj + 2;
+                if (idx + 2 < nactv) prep(idx + 2, idx + 3 < nactv, nxt);
+                refill(idx + 2, nxt.sj);
+                bar_sync(kBarB, nb2);
+                // Alg1:9-11 for both voxels on this thread's views: a's channels with a's update,
+                // then b's channels with both updates -- b's write carries the full value on the
+                // entries the two voxels share
+                const float sda = dslot[(pn & 1) * 2], sdb = dslot[(pn & 1) * 2 + 1];
+                if (sda != 0.f || sdb != 0.f) {
+                    const float2 nda = make_float2(-sda, -sda), ndb = make_float2(-sdb, -sdb);
+#pragma unroll
+                    for (int t = 0; t < VPT; ++t) {
+                        float* pe = sb + cur.pa[t];
+                        float* qe = sb + cur.pb[t];
+                        const float2 a0 = __ffma2_rn(cur.fa[t][0], nda, ea[t][0]);
+                        const float2 a1 = __ffma2_rn(cur.fa[t][1], nda, ea[t][1]);
+                        const float2 b0 = __ffma2_rn(cur.fb[t][0], ndb, __ffma2_rn(cur.fab[t][0], nda, eb[t][0]));
+                        const float2 b1 = __ffma2_rn(cur.fb[t][1], ndb, __ffma2_rn(cur.fab[t][1], nda, eb[t][1]));
+                        pe[0] = a0.x;
+                        pe[RS] = a0.y;
+                        pe[2 * RS] = a1.x;
+                        pe[3 * RS] = a1.y;
+                        qe[0] = b0.x;
+                        qe[RS] = b0.y;
+                        qe[2 * RS] = b1.x;
+                        qe[3 * RS] = b1.y;
+                    }
+                }
+            };
+            // the first R records (the ring region held the pack's staging tiles until the barrier)
+            for (int i = 0; i < R; ++i) copy_record_to(i, (sbase + i) % R, i < nactv ? list[i] : 0);
+            PairState st0, st1;
+            st0.sj = sbase;
+            prep(0, 1 < nactv, st0);
+            refill(0, sbase);
+            for (int idx = 0; idx < nactv; idx += 4) {
+                pair_step(idx, st0, st1);
+                if (idx + 2 < nactv) pair_step(idx + 2, st1, st0);
+            }
+        } else if (is_delta) {
+            // ---- delta warp: per pair wait for the partial sums and the surrogate terms (A),
+            //      derive both deltas (every lane, identical inputs), publish them (B), write the
+            //      new values into the x tile (X, releases the prior warp)
+            for (int p = 0; p < npair; ++p) {
+                const int idx = 2 * p;
+                const uint32_t pn = pseq + (uint32_t)p;
+                const bool hasb = idx + 1 < nactv;
+                bar_sync(kBarA, nab);
+                const float* rb = red + (pn & 1) * 3 * kNSL;  // nvw <= kNSL partials, rest 0
+                float sa = 0.f, sbs = 0.f, sh = 0.f;
+#pragma unroll
+                for (int i = 0; i < kNSL; ++i) {  // fixed order: every run gets the same bits
+                    sa += rb[i];
+                    sbs += rb[kNSL + i];
+                    sh += rb[2 * kNSL + i];
+                }
+                const PriPair pp = pri[pn & 1];
+                const float scale_a = vscale[idx];
+                float ua = pp.va;
+                const float theta1a = -scale_a * sa;  // Alg1:5
+                const float theta2a = vth2[idx];      // Alg1:6 (precomputed)
+                {
+                    const float num = theta2a * pp.va - theta1a + 2.f * pp.sxa;
+                    const float den = theta2a + 2.f * pp.sa;
+                    if (den > 0.f) ua = __fdividef(num, den);
+                    if (P.pc.positivity) ua = fmaxf(ua, 0.f);
+                }
+                const float da = ua - pp.va;  // Alg1:7-8
+                float ub = pp.vb, db = 0.f, scale_b = 0.f, theta1b = 0.f, theta2b = 0.f;
+                if (hasb) {
+                    scale_b = vscale[idx + 1];
+                    // e after a's update: sum w A_b e' = s_b (S_b - s_a delta_a H)
+                    theta1b = -scale_b * fmaf(-scale_a * da, sh, sbs);
+                    theta2b = vth2[idx + 1];
+                    float psb = pp.sb, psx = pp.sxb;
+                    if (pp.bab != 0.f) {  // a is b's neighbour: its term with a's new value
+                        const float bn = pp.bab * phi_f(P.pc, pp.vb - ua);
+                        psb += bn - pp.btab;
+                        psx += bn * ua - pp.btab * pp.va;
+                    }
+                    const float num = theta2b * pp.vb - theta1b + 2.f * psx;
+                    const float den = theta2b + 2.f * psb;
+                    if (den > 0.f) ub = __fdividef(num, den);
+                    if (P.pc.positivity) ub = fmaxf(ub, 0.f);
+                    db = ub - pp.vb;
+                }
+                if (lane == 0) {
+                    dslot[(pn & 1) * 2] = scale_a * da;
+                    dslot[(pn & 1) * 2 + 1] = scale_b * db;
+                }
+                bar_arrive(kBarB, nb2);
+                if (lane == 0) {
+                    const int ta = tof[idx];
+                    xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
+                    if (hasb) {
+                        const int tbv = tof[idx + 1];
+                        xt[cslot + (tbv >> 8) * TW + (tbv & 255)] = ub;
+                    }
+                }
+                bar_arrive(kBarX, 64);
+                if (lane == 0) {
+                    amount += fabsf(da) + fabsf(db);
+                    if (P.dump) {
+                        // test hook (mbir_set_update_dump): the pair's (voxel, theta1, theta2,
+                        // delta) exactly as the delta chain used them, a then b
+                        const unsigned long long slot = atomicAdd(P.dump_count, hasb ? 2ull : 1ull);
+                        for (int u = 0; u < (hasb ? 2 : 1); ++u) {
+                            const int tv = tof[idx + u];
+                            const uint32_t vox = (uint32_t)(((size_t)z * P.ny + gy0 + (tv >> 8)) * P.nx + gx0 + (tv & 255));
+                            if (slot + u < (unsigned long long)P.dump_cap)
+                                *(float4*)(P.dump + 4 * (slot + u)) = make_float4(
+                                    __uint_as_float(vox), u ? theta1b : theta1a, u ? theta2b : theta2a, u ? db : da);
+                        }
+                    }
+                }
+            }
+        } else if (is_prior) {
+            // ---- prior warp: the surrogate terms of pair p + 1 once pair p's new values are in
+            //      the x tile (X); its own arrival on A completes the pair's inputs
+            bar_arrive(kBarA, nab);  // pair 0's terms were computed in step 3
+            for (int p = 0; p < npair; ++p) {
+                bar_sync(kBarX, 64);
+                if (p + 1 < npair) {
+                    prior_pair(tof, 2 * (p + 1), nactv, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
+                               pri + ((pseq + (uint32_t)p + 1) & 1));
+                    __syncwarp();
+                    bar_arrive(kBarA, nab);
+                }
+            }
+        }
+        gseq += nactv;
+        pseq += (uint32_t)npair;
+        if (PROF && threadIdx.x == 0) tp3 = clock64();
+        __syncthreads();
+
+        // ---- 6. write-back: delta e of the band, atomically, and the SV's voxels
+        if (is_view && vw < ntw) {
+            float* ez = P.e + (size_t)z * V * M;
+            const int sub = lane >> 3, ch = lane & 7;
+            auto ld_init = [&](int t, float4 (&s4)[8]) {
+                const int k0 = (vw * kTileW + t) * 32;
+#pragma unroll
+                for (int m = 0; m < 8; ++m) s4[m] = __ldcg((const float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch));
+            };
+            float4 s4b[2][8];
+            ld_init(0, s4b[0]);
+#pragma unroll
+            for (int t = 0; t < kTileW; ++t) {
+                if (t + 1 < kTileW) ld_init(t + 1, s4b[(t + 1) & 1]);
+                const float4 (&s4)[8] = s4b[t & 1];
+                const int k0 = (vw * kTileW + t) * 32;
+                const int kk = k0 + lane;
+                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const int bw = (int)(bi & 31u), roff = (int)(bi >> 5);
+                const uint32_t bmask = ((1u << bw) - 1u) << (roff & 3);
+                // this view's final band -> its staging row (positions outside the band: 0)
+                const float* se = sb + kk - (roff & 3) * RS;
+#pragma unroll
+                for (int q4 = 0; q4 < 8; ++q4) {
+                    float rv[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int p = 4 * q4 + j;
+                        rv[j] = (bmask & (1u << p)) ? se[p * RS] : 0.f;
+                    }
+                    *(float4*)(stg_w + lane * kStg + 4 * q4) = make_float4(rv[0], rv[1], rv[2], rv[3]);
+                }
+                __syncwarp();
+#pragma unroll
+                for (int m = 0; m < 8; ++m) {
+                    const int i = 4 * m + sub;
+                    const int oi = __shfl_sync(kFull, roff, i);
+                    const uint32_t nib = __shfl_sync(kFull, bmask, i) >> (4 * ch);
+                    const float4 f4 = *(const float4*)(stg_w + i * kStg + 4 * ch);
+                    const float fv[4] = {f4.x, f4.y, f4.z, f4.w};
+                    const float e0[4] = {s4[m].x, s4[m].y, s4[m].z, s4[m].w};
+                    float d[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) d[j] = (nib & (1u << j)) ? fv[j] - e0[j] : 0.f;
+                    if (k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
+                        red_add_v4(ez + (oi - (oi & 3)) + 4 * ch, d[0], d[1], d[2], d[3]);
+                }
+                __syncwarp();
+            }
+        } else if (is_delta) {
+            // the image and the counters
+            for (int i = lane; i < tw * th; i += 32) {
+                const int lx = i % tw, ly = i / tw;
+                P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] = xt[cslot + ly * TW + lx];
+            }
+            if (lane == 0) {
+                P.sv_amount[(size_t)z * P.nsv + sv] = amount;
+                atomicAdd(P.counters + 0, (unsigned long long)nactv);
+                atomicAdd(P.counters + 1, (unsigned long long)(tw * th - nactv));
+                atomicAdd(P.counters + 2, 1ull);
+                atomicAdd(P.sum_delta, (double)amount);
+            }
+        } else if (is_prior) {
+            // the next task's band info, with an L2 warm-up of its band rows (the next pack
+            // then reads L2)
+            const int nq = s_task[nslot];
+            if (nq < tend) {
+                const int nt = P.flat[nq];
+                constexpr int KMAX = 6;  // views per lane and pass: all loads in flight at once
+                const int psv = nt & 16383, pz = nt >> 14;
+                uint32_t* dst = binfo + (tb ^ 1) * VA;
+                const float* wz = P.w + (size_t)pz * V * M;
+                const float* ez = P.e + (size_t)pz * V * M;
+#pragma unroll 1
+                for (int k0 = 0; k0 < V; k0 += 32 * KMAX) {
+                    int bs[KMAX], bwd[KMAX];
+#pragma unroll
+                    for (int i = 0; i < KMAX; ++i) {
+                        const int k = k0 + lane + 32 * i;
+                        if (k < V) {
+                            bs[i] = P.A.band_start[(size_t)psv * V + k];
+                            bwd[i] = P.A.band_width[(size_t)psv * V + k];
+                        }
+                    }
+#pragma unroll
+                    for (int i = 0; i < KMAX; ++i) {
+                        const int k = k0 + lane + 32 * i;
+                        if (k < V) {
+                            const int r = k * M + bs[i], r1 = r + max(bwd[i], 1) - 1;
+                            dst[k] = ((uint32_t)r << 5) | (uint32_t)bwd[i];
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
+                        }
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        if (PROF && threadIdx.x == 0) {
+            const long long tp4 = clock64();
+            atomicAdd(P.tprof + 0, (unsigned long long)(tp1 - tp0));  // x tile, zero-skip, order
+            atomicAdd(P.tprof + 1, (unsigned long long)(tp2 - tp1));  // SVB pack
+            atomicAdd(P.tprof + 2, (unsigned long long)(tp3 - tp2));  // voxel loop
+            atomicAdd(P.tprof + 3, (unsigned long long)(tp4 - tp3));  // write-back
+            atomicAdd(P.tprof + 4, (unsigned long long)nactv);
+            atomicAdd(P.tprof + 5, 1ull);
+        }
+    }
+}
+
+// A-record ring depth (voxels of cp.async lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
+// (the pair loop needs >= 4: the current pair's two stages plus the next pair's two)
+constexpr int ring_depth(bool u8) { return u8 ? 12 : 4; }
+
+template <int VPT, bool U8, int NNB>
+cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
+{
+    constexpr int R = ring_depth(U8);
+    auto kern = p.tprof ? k_svicd<VPT, U8, NNB, R, true> : k_svicd<VPT, U8, NNB, R, false>;
+    IcdParams q = p;
+    q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT);
+    const int smem = q.lay.total;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e != cudaSuccess) return e;
+    kern<<<gx, 32 * (p.nvw + 2), smem, st>>>(q);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
+{
+    return svicd_layout(p.rows, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw, vpt).total;
+}
+
+template <int VPT, bool U8, int NNB>
+int resident_t(const IcdParams& p)
+{
+    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), false>;
+    const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT).total;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
+    cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    int nb = 0, dev = 0, nsm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, 32 * (p.nvw + 2), smem) != cudaSuccess) return -1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    return nb * nsm;
+}
+
+int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize)
+{
+    if (vpt == 2) {
+        if (quantize) return nnb == 26 ? resident_t<2, true, 26>(p) : resident_t<2, true, 8>(p);
+        return nnb == 26 ? resident_t<2, false, 26>(p) : resident_t<2, false, 8>(p);
+    }
+    if (vpt == 1) {
+        if (quantize) return nnb == 26 ? resident_t<1, true, 26>(p) : resident_t<1, true, 8>(p);
+        return nnb == 26 ? resident_t<1, false, 26>(p) : resident_t<1, false, 8>(p);
+    }
+    if (quantize) return nnb == 26 ? resident_t<4, true, 26>(p) : resident_t<4, true, 8>(p);
+    return nnb == 26 ? resident_t<4, false, 26>(p) : resident_t<4, false, 8>(p);
+}
+
+int svicd_scratch_floats(int vpt) { return svb_cols(vpt) * 32; }
+
+cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid, cudaStream_t st)
+{
+    if (vpt == 2) {
+        if (quantize) return nnb == 26 ? launch_t<2, true, 26>(p, grid, st) : launch_t<2, true, 8>(p, grid, st);
+        return nnb == 26 ? launch_t<2, false, 26>(p, grid, st) : launch_t<2, false, 8>(p, grid, st);
+    }
+    if (vpt == 1) {
+        if (quantize) return nnb == 26 ? launch_t<1, true, 26>(p, grid, st) : launch_t<1, true, 8>(p, grid, st);
+        return nnb == 26 ? launch_t<1, false, 26>(p, grid, st) : launch_t<1, false, 8>(p, grid, st);
+    }
+    if (quantize) return nnb == 26 ? launch_t<4, true, 26>(p, grid, st) : launch_t<4, true, 8>(p, grid, st);
+    return nnb == 26 ? launch_t<4, false, 26>(p, grid, st) : launch_t<4, false, 8>(p, grid, st);
+}
+
+}  // namespace mbir

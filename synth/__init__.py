@@ -12,6 +12,8 @@ from .phantom import (  # noqa: F401
     baggage_phantom,
     make_case,
     make_sinogram_torch,
+    noisy_counts,
+    slice_ellipses,
     phantom_image,
     shepp_logan_2d,
     shepp_logan_3d,

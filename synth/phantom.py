@@ -6,7 +6,8 @@ Views theta_k = k*pi/V.  Channel i covers [t0 + i*dc, t0 + (i+1)*dc),
 t0 = -M*dc/2 + center_offset*dc.
 
 Sinogram: p_i = mean over `subrays` equally spaced rays inside channel i of the analytic
-line integral of the phantom; counts lambda_i ~ Poisson(lambda0 * exp(-p_i));
+line integral of the phantom; counts lambda_i ~ Poisson(lambda0 * exp(-p_i)) from a numpy
+generator seeded per slice by (noise seed, z);
 y_i = ln(lambda0 / max(lambda_i, 1)), w_i = max(lambda_i, 1) (inverse variance of y_i).
 """
 from __future__ import annotations
@@ -161,12 +162,31 @@ CONFIGS = {
 }
 
 
+def slice_ellipses(cfg: WorkloadConfig, z: int, phantom_seed: int):
+    """The ellipses of global slice z of a config's phantom (2-D Shepp-Logan, a slab of the 3-D
+    head with slices sampling z in [-0.25, 0.25], or a baggage scene)."""
+    if cfg.phantom == "baggage":
+        return baggage_phantom(phantom_seed * 1000 + z)
+    if cfg.nz == 1:
+        return shepp_logan_2d()
+    return shepp_logan_3d(-0.25 + 0.5 * (z + 0.5) / cfg.nz)
+
+
+def noisy_counts(p: np.ndarray, lambda0: float, noise_seed: int, z: int):
+    """Poisson counts of slice z: lambda ~ Poisson(lambda0 exp(-p)) from a generator seeded by
+    (noise_seed, z), so any slab of a volume is the same whoever computes it; returns (y, w)
+    float32 with y = ln(lambda0 / max(lambda, 1)), w = max(lambda, 1)."""
+    rng = np.random.default_rng([noise_seed, z])
+    lam = np.maximum(rng.poisson(lambda0 * np.exp(-p)), 1).astype(np.float64)
+    return np.log(lambda0 / lam).astype(np.float32), lam.astype(np.float32)
+
+
 def make_sinogram_torch(cfg: WorkloadConfig, case_id: int = 0, device="cuda", z0: int = 0,
                         z1: int | None = None):
-    """Same recipe as make_case (3-D Shepp-Logan slices, 4 sub-rays, Poisson counts) computed
-    with torch on `device` for the large bench configs; returns float32 tensors y, w
-    [z1-z0, V, M] on that device for global slices [z0, z1).  Poisson draws use a torch
-    generator seeded with (2000+case)*1000 + z per slice, so a slab is the same on any rank."""
+    """The make_case recipe for the large bench configs: the analytic projections (double) are
+    computed with torch on `device`, the Poisson counts with the same per-slice numpy generator
+    as make_case (noisy_counts), so the result equals make_case(cfg, case_id) slice by slice.
+    Returns float32 tensors y, w [z1-z0, V, M] on `device` for global slices [z0, z1)."""
     import torch
     V, M, nz = cfg.nviews, cfg.nchannels, cfg.nz
     z1 = nz if z1 is None else z1
@@ -176,17 +196,11 @@ def make_sinogram_torch(cfg: WorkloadConfig, case_id: int = 0, device="cuda", z0
     sub = (torch.arange(4, dtype=torch.float64, device=dev) + 0.5) / 4
     t = t0 + (torch.arange(M, dtype=torch.float64, device=dev)[:, None] + sub[None, :]).reshape(-1) * cfg.dchannel
     c, s = torch.cos(theta)[:, None], torch.sin(theta)[:, None]
-    gen = torch.Generator(device=dev)
     y = torch.empty((z1 - z0, V, M), dtype=torch.float32, device=dev)
     w = torch.empty_like(y)
     for z in range(z0, z1):
-        gen.manual_seed((2000 + case_id) * 1000 + z)
-        if nz == 1:
-            ells = shepp_logan_2d()
-        else:
-            ells = shepp_logan_3d(-0.25 + 0.5 * (z + 0.5) / nz)
         p = torch.zeros((V, t.numel()), dtype=torch.float64, device=dev)
-        for (x0, y0, a, b, phi, mu) in ells:
+        for (x0, y0, a, b, phi, mu) in slice_ellipses(cfg, z, 1000 + case_id):
             ct = torch.cos(theta - phi)[:, None]
             st = torch.sin(theta - phi)[:, None]
             r2 = a * a * ct * ct + b * b * st * st
@@ -194,9 +208,9 @@ def make_sinogram_torch(cfg: WorkloadConfig, case_id: int = 0, device="cuda", z0
             disc = r2 - sp * sp
             p += torch.where(disc > 0, mu * 2.0 * a * b * torch.sqrt(disc.clamp_min(0.0)) / r2, 0.0)
         p = p.reshape(V, M, 4).mean(dim=2)
-        lam = torch.poisson(cfg.lambda0 * torch.exp(-p), generator=gen).clamp_min(1.0)
-        y[z - z0] = torch.log(cfg.lambda0 / lam).float()
-        w[z - z0] = lam.float()
+        yz, wz = noisy_counts(p.cpu().numpy(), cfg.lambda0, 2000 + case_id, z)
+        y[z - z0] = torch.from_numpy(yz).to(dev)
+        w[z - z0] = torch.from_numpy(wz).to(dev)
     return y, w
 
 
@@ -214,24 +228,14 @@ def make_case(cfg: WorkloadConfig, case_id: int = 0, *, phantom_seed=None, noise
     """Seeds: phantom 1000+case, noise 2000+case."""
     ps = 1000 + case_id if phantom_seed is None else phantom_seed
     ns = 2000 + case_id if noise_seed is None else noise_seed
-    rng = np.random.default_rng(ns)
     V, M, nz = cfg.nviews, cfg.nchannels, cfg.nz
     y = np.empty((nz, V, M), np.float32)
     w = np.empty((nz, V, M), np.float32)
     truth = np.empty((nz, cfg.n, cfg.n)) if with_truth else None
     for z in range(nz):
-        if cfg.phantom == "baggage":
-            ells = baggage_phantom(ps * 1000 + z)
-        elif nz == 1:
-            ells = shepp_logan_2d()
-        else:  # slices sample z in [-0.25, 0.25] of the normalised 3-D head
-            zn = -0.25 + 0.5 * (z + 0.5) / nz
-            ells = shepp_logan_3d(zn)
+        ells = slice_ellipses(cfg, z, ps)
         p = sinogram(ells, V, M, cfg.dchannel, cfg.center_offset)
-        lam = rng.poisson(cfg.lambda0 * np.exp(-p))
-        lam = np.maximum(lam, 1).astype(np.float64)
-        y[z] = np.log(cfg.lambda0 / lam)
-        w[z] = lam
+        y[z], w[z] = noisy_counts(p, cfg.lambda0, ns, z)
         if with_truth:
             truth[z] = phantom_image(ells, cfg.n)
     return Case(cfg, y, w, truth, {"phantom_seed": ps, "noise_seed": ns})

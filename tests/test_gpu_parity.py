@@ -384,16 +384,16 @@ def m720():
     return cfg, case, g, og, Aq
 
 
-@pytest.mark.parametrize("cluster", [1, 2])
-def test_bench_shape_deterministic_tracks_oracle(m720, cluster):
-    """The launch configuration bench.py times (uint8 A, 4 views per lane, 6 view warps, one CTA
-    or a 2-CTA cluster per task): deterministic order, 2 equits, against the sequential oracle."""
+def test_bench_shape_deterministic_tracks_oracle(m720):
+    """The launch configuration bench.py times (uint8 A, 4 views per lane, 6 view warps + the
+    delta and prior warps, one CTA per task): deterministic order, 2 equits, against the
+    sequential oracle."""
     cfg, case, g, og, Aq = m720
     pr = O.Prior(sigma=cfg.sigma, nbhd=26)
     order = deterministic_order(cfg.n, cfg.nz, cfg.sv_side, 26)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
-                         M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0, cluster=cluster)) as r:
-        assert r.sizes()["cluster"] == cluster
+                         M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0)) as r:
+        assert r.sizes()["cluster"] == 1
         r.set_sinogram(case.y, case.w)
         x = np.zeros(cfg.nz * cfg.n * cfg.n)
         e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
@@ -408,8 +408,7 @@ def test_bench_shape_deterministic_tracks_oracle(m720, cluster):
     assert np.abs(eg.ravel() - e.ravel()).max() < 1e-4 * np.abs(case.y).max()
 
 
-@pytest.mark.parametrize("cluster", [1, 2])
-def test_bench_shape_converged_matches_oracle(m720, cluster):
+def test_bench_shape_converged_matches_oracle(m720):
     """Asynchronous GPU-ICD in the bench's launch shape (persistent grid, random orders, 25 %
     SV selection, zero-skipping off) reaches the oracle's MAP point: 1 HU / 1e-4."""
     cfg, case, g, og, Aq = m720
@@ -418,7 +417,7 @@ def test_bench_shape_converged_matches_oracle(m720, cluster):
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
     O.icd_run(og, pr, Aq, case.w, x, e, 80, seed=3000, zero_skip=False)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
-                         M.Options(sv_side=cfg.sv_side, zero_skip=0, cluster=cluster)) as r:
+                         M.Options(sv_side=cfg.sv_side, zero_skip=0)) as r:
         r.set_sinogram(case.y, case.w)
         r.reconstruct(200)
         xg = r.image().ravel().astype(np.float64)
@@ -429,14 +428,17 @@ def test_bench_shape_converged_matches_oracle(m720, cluster):
 
 
 def test_cluster_option_validation():
-    """cluster = 2 needs uint8 A and an even number of 128-view warps (include/mbir.h)."""
-    cfg = CONFIGS["cfg1"]  # 90 views: one warp of 1 view per lane
+    """One CTA owns an SV task (include/mbir.h mbir_options.cluster): 0 (auto) and 1 are
+    accepted, anything else is EINVAL."""
+    cfg = CONFIGS["cfg1"]  # 90 views: three warps of 1 view per lane
     g, _ = geoms(cfg)
-    with pytest.raises(M.MbirError) as ei:
-        M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side, cluster=2))
-    assert ei.value.code == -1
+    for bad in (2, -1):
+        with pytest.raises(M.MbirError) as ei:
+            M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side, cluster=bad))
+        assert ei.value.code == -1
     with M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side)) as r:
         assert r.sizes()["cluster"] == 1
+        assert r.sizes()["threads_per_cta"] == 32 * (3 + 2)
 
 
 # ------------------------------------------------------------------ FBP initial image (R23)
