@@ -57,7 +57,7 @@ __host__ __device__ __forceinline__ int apos(int k, int vpt)
 // configuration and passed in the parameter block, so the kernel addresses them from the
 // constant bank instead of recomputing the layout in registers)
 struct SmemLayout {
-    int sb_e, sb_w, xt, list, flags, tof, red, pri, vscale, vth2, misc, astage, stage_bytes,
+    int sb_e, sb_w, xt, list, flags, tof, red, pri, vscale, vth2, misc, astage, stage_bytes, rscale, rth2, rbs, rbw,
         off_in_stage, mbar, staging, binfo, total;
 };
 

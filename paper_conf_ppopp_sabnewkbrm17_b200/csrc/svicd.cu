@@ -87,11 +87,24 @@ __device__ __forceinline__ void cp_async4(void* dst, const void* src)
 {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
+// 4-byte copy that writes zeros instead when !valid (src_size 0)
+__device__ __forceinline__ void cp_async4_zfill(void* dst, const void* src, bool valid)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(valid ? 4 : 0) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait()
 {
     asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+// one 128-bit shared-memory load (kept vector: the staging row reads are conflict-free only as
+// LDS.128; split into scalar loads they would be 4-way bank conflicts)
+__device__ __forceinline__ float4 lds128(const float* p)
+{
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(smem_u32(p)));
+    return v;
 }
 // named barriers: sync (wait for `n` threads incl. this warp) / arrive (count and go on)
 __device__ __forceinline__ void bar_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
@@ -227,10 +240,11 @@ __host__ __device__ constexpr int max_threads(int vpt) { return vpt == 2 ? 448 :
 constexpr int kBarA = 1;  // view warps' partials + the prior warp's terms of a pair are ready
 constexpr int kBarB = 2;  // the delta warp has published the pair's deltas
 constexpr int kBarX = 3;  // the delta warp has written the pair's new values into the x tile
+constexpr int kBarP = 4;  // task preparation steps (delta + prior warps)
 
 // A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
 __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, int nnb, int VA, bool u8,
-                                                   int nstage, int nvw, int vpt)
+                                                   int nstage, int nvw, int vpt, int V)
 {
     SmemLayout L;
     const int TW = side + 2;
@@ -238,14 +252,14 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     int o = 0;
     L.sb_e = o;  o = align16(o + 2 * rows * svb_cols(vpt) * 4);  // e / w rows interleaved
     L.sb_w = L.sb_e + svb_cols(vpt) * 4;
-    L.xt = o;    o = align16(o + nzt * TW * TW * 4);
-    L.list = o;  o = align16(o + S2 * 4);
+    L.xt = o;    o = align16(o + 2 * nzt * TW * TW * 4);  // [2 tasks]: current / next
+    L.list = o;  o = align16(o + 2 * S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
-    L.tof = o;   o = align16(o + S2 * 4);
+    L.tof = o;   o = align16(o + 2 * S2 * 4);
     L.red = o;   o = align16(o + 2 * 3 * kNSL * 4);  // [2 bufs][3 quantities][kNSL view warps]
     L.pri = o;   o = align16(o + 2 * (int)sizeof(PriPair));
-    L.vscale = o; o = align16(o + S2 * 4);
-    L.vth2 = o;  o = align16(o + S2 * 4);
+    L.vscale = o; o = align16(o + 2 * S2 * 4);
+    L.vth2 = o;  o = align16(o + 2 * S2 * 4);
     L.misc = o;  o = align16(o + 16 * 4);
     L.off_in_stage = VA * (u8 ? 4 : 16);
     L.stage_bytes = align16(L.off_in_stage + VA);
@@ -254,7 +268,11 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     L.astage = o;
     L.staging = o;
     o = align16(o + max(nstage * L.stage_bytes, tile_warps(VA) * 32 * kStg * 4));
-    L.mbar = o;  o = align16(o + 4 * 32 * 4);  // neighbour tables [dx | dy | dz | b][32]
+    L.mbar = o;  o = align16(o + 5 * 32 * 4);  // neighbour tables [dx | dy | dz | b | tile offset][32]
+    L.rscale = o; o = align16(o + S2 * 4);      // the next task's inputs as copied (cp.async):
+    L.rth2 = o;  o = align16(o + S2 * 4);       //   per-slot scales and theta2,
+    L.rbs = o;   o = align16(o + V * 4);        //   band start and width per view
+    L.rbw = o;   o = align16(o + V);
     L.binfo = o; o = align16(o + 2 * VA * 4);  // band (row offset << 5 | width), 2 tasks
     L.total = o;
     return L;
@@ -322,21 +340,17 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     constexpr int RS = 2 * VS;             // float stride between consecutive e (or w) rows
     const SmemLayout& L = P.lay;
     float* sb = (float*)(smem + L.sb_e);   // e row r at sb + r RS, w row r at sb + r RS + VS
-    float* xt = (float*)(smem + L.xt);
-    int* list = (int*)(smem + L.list);
     int* flags = (int*)(smem + L.flags);
-    int* tof = (int*)(smem + L.tof);       // visiting order as packed (ly << 8 | lx)
     float* red = (float*)(smem + L.red);
     PriPair* pri = (PriPair*)(smem + L.pri);
-    float* vscale = (float*)(smem + L.vscale);
-    float* vth2 = (float*)(smem + L.vth2);
     unsigned char* astage = smem + L.astage;
     float* stg_w = (float*)(smem + L.staging) + vw * 32 * kStg;
-    int* s_task = (int*)(smem + L.misc);            // [0] first task, [1 + (n & 1)] the task after n
+    int* s_task = (int*)(smem + L.misc);            // [b]: the task prepared in buffer b, [2 + b]: its kept voxels
     float* dslot = (float*)(smem + L.misc) + 4;     // [2 pairs][2]: scale_a delta_a, scale_b delta_b
     uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA]
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
+    const int ntile = (NNB == 26 ? 3 : 1) * TW * TW;  // x tile entries
     const size_t plane = (size_t)P.nx * P.ny;
     const int nab = (nvw + 2) * 32;      // barrier A: view warps + delta warp + prior warp
     const int nb2 = (nvw + 1) * 32;      // barrier B: view warps + the delta warp
@@ -351,6 +365,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         nbt[32 + i] = ok ? P.pc.dy[i] : 0;
         nbt[64 + i] = ok ? P.pc.dz[i] : 0;
         nbt[96 + i] = ok ? __float_as_int(P.pc.b[i]) : 0;
+        nbt[128 + i] = ok ? (P.pc.dz[i] * (side + 2) + P.pc.dy[i]) * (side + 2) + P.pc.dx[i] : 0;
     }
     __syncthreads();
     // SVB rows outside a visit's band are never packed: start them finite (zero)
@@ -392,96 +407,163 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         }
         return q;
     };
-    if (threadIdx.x == 0) s_task[0] = fetch_task();
+    // ---- task preparation.  A task's inputs are stable during a phase (its own voxels are only
+    //      updated by its owner, its ring belongs to other colours, its +-1 slices to the other z
+    //      parity), so they are gathered early: while the current task is packed, the delta warp
+    //      fetches the next task and copies its x tile (+1 halo ring, +-1 slice in 3-D; zeros
+    //      off the image), the slots' scales and theta2 and its band start / width into shared
+    //      memory with cp.async; during the current task's write-back the delta and prior warps
+    //      (64 threads, named barrier kBarP) evaluate its zero-skip predicate (reading R9:
+    //      slot kept iff valid and (skip inactive or x_j or a neighbour is non-zero) -- the tile
+    //      holds zeros outside the volume), build its visiting order (one of NPERM host-drawn
+    //      random permutations of the tile chosen per (seed, iteration, slice, SV) visit, raster
+    //      order in deterministic mode, compacted with a ballot), stage the ordered scales and
+    //      theta2 and its band info (+ an L2 warm-up of its band rows).  A task whose every voxel
+    //      is skipped is accounted and replaced by the next one (synchronously).
+    const int rt = threadIdx.x - nvw * 32;  // thread index among the delta and prior warps
+    float* rscale = (float*)(smem + L.rscale);
+    float* rth2 = (float*)(smem + L.rth2);
+    int* rbs = (int*)(smem + L.rbs);
+    unsigned char* rbw = smem + L.rbw;
+    // delta warp: fetch the next task into s_task[b] and start copying its inputs into buffer b
+    auto fetch_and_copy = [&](int b) {
+        int qn = 0;
+        if (lane == 0) qn = fetch_task();
+        qn = __shfl_sync(kFull, qn, 0);
+        if (lane == 0) s_task[b] = qn;
+        if (qn < tend) {
+            const int tkn = P.flat[qn];
+            const int z = tkn >> 14, sv = tkn & 16383;
+            const int gx0 = (sv % P.nsvx) * side, gy0 = (sv / P.nsvx) * side;
+            float* xb = (float*)(smem + L.xt) + b * ntile;
+            for (int i = lane; i < ntile; i += 32) {
+                const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
+                const int gx = gx0 - 1 + tx, gy = gy0 - 1 + ty;
+                const int zs = (NNB == 26) ? z + tz : z + 1;  // storage slice (halo at 0, nz+1)
+                const bool inb = gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny;
+                const int cx = min(max(gx, 0), P.nx - 1), cy = min(max(gy, 0), P.ny - 1);
+                cp_async4_zfill(xb + i, P.x + (size_t)min(zs, P.nz_local + 1) * plane + (size_t)cy * P.nx + cx, inb);
+            }
+            const size_t arec = (size_t)sv * S2;
+            for (int i = lane; i < S2; i += 32) {
+                cp_async4(rscale + i, P.A.scale + arec + i);
+                cp_async4(rth2 + i, P.theta2 + ((size_t)z * P.nsv + sv) * S2 + i);
+            }
+            for (int k = lane; k < V; k += 32) cp_async4(rbs + k, P.A.band_start + (size_t)sv * V + k);
+            for (int k = 4 * lane; k < V; k += 128) {  // band widths as 4-byte words (V % 4 == 0)
+                if ((V & 3) == 0) cp_async4(rbw + k, P.A.band_width + (size_t)sv * V + k);
+            }
+        }
+        cp_async_commit();
+    };
+    // delta + prior warps: complete the preparation of the task in buffer b (copies issued by
+    // fetch_and_copy); returns with s_task[b] >= tend or s_task[2 + b] > 0 kept voxels
+    auto finish_prepare = [&](int b) {
+        float* xb = (float*)(smem + L.xt) + b * ntile;
+        int* listb = (int*)(smem + L.list) + b * S2;
+        int* tofb = (int*)(smem + L.tof) + b * S2;
+        for (;;) {
+            if (is_delta) cp_async_wait<0>();
+            bar_sync(kBarP, 64);
+            const int qn = s_task[b];
+            if (qn >= tend) return;
+            const int tkn = P.flat[qn];
+            const int z = tkn >> 14, sv = tkn & 16383, zg = P.z_offset + z;
+            const int gx0 = (sv % P.nsvx) * side, gy0 = (sv / P.nsvx) * side;
+            const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
+            for (int v0 = rt; v0 < S2; v0 += 64) {
+                const int lx = v0 % side, ly = v0 / side;
+                int keep = lx < tw && ly < th;
+                if (keep && P.zero_skip_active) {
+                    const float* c = xb + (zc * TW + ly + 1) * TW + lx + 1;
+                    float acc = fabsf(c[0]);
+#pragma unroll
+                    for (int r = 0; r < NNB; ++r) acc += fabsf(c[nbt[128 + r]]);
+                    keep = acc != 0.f;
+                }
+                flags[v0] = keep;
+            }
+            bar_sync(kBarP, 64);
+            if (is_prior) {
+                const uint64_t h = mix64(P.seed ^ mix64(((uint64_t)P.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)sv));
+                const uint8_t* perm = P.perm + (size_t)(h % (uint64_t)P.nperm) * S2;
+                int n = 0;
+                for (int base = 0; base < S2; base += 32) {
+                    const int i = base + lane;
+                    const int v = i < S2 ? (P.deterministic ? i : (int)perm[i]) : 0;
+                    const bool k = i < S2 && flags[v];
+                    const unsigned m = __ballot_sync(kFull, k);
+                    if (k) {
+                        const int p = n + __popc(m & ((1u << lane) - 1));
+                        listb[p] = v;
+                        tofb[p] = ((v / side) << 8) | (v % side);  // packed (ly, lx): no div in the loop
+                    }
+                    n += __popc(m);
+                }
+                if (lane == 0) {
+                    s_task[2 + b] = n;
+                    if (n == 0) {  // the whole SV is zero-skipped: account for it
+                        P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
+                        atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
+                        atomicAdd(P.counters + 2, 1ull);
+                        atomicAdd(P.counters + 3, 1ull);
+                    }
+                }
+                __syncwarp();
+                float* vsb = (float*)(smem + L.vscale) + b * S2;
+                float* vtb = (float*)(smem + L.vth2) + b * S2;
+                for (int i = lane; i < n; i += 32) {
+                    const int v = listb[i];
+                    vsb[i] = rscale[v];
+                    vtb[i] = rth2[v];
+                }
+                if (n > 0) {
+                    // band info (row offset << 5 | width) and an L2 warm-up of the band rows
+                    uint32_t* dst = binfo + b * VA;
+                    const float* wz = P.w + (size_t)z * V * M;
+                    const float* ez = P.e + (size_t)z * V * M;
+                    for (int k = lane; k < V; k += 32) {
+                        const int wd = (V & 3) == 0 ? rbw[k] : P.A.band_width[(size_t)sv * V + k];
+                        const int r = k * M + rbs[k], r1 = r + max(wd, 1) - 1;
+                        dst[k] = ((uint32_t)r << 5) | (uint32_t)wd;
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
+                    }
+                }
+            }
+            bar_sync(kBarP, 64);
+            if (s_task[2 + b] > 0) return;
+            if (is_delta) fetch_and_copy(b);  // fully skipped: the next task, synchronously
+        }
+    };
+    int cb = 0;  // buffer of the current task (binfo, x tile, order, scales)
+    if (is_delta) fetch_and_copy(0);
+    if (!is_view) finish_prepare(0);
     __syncthreads();
     int q = s_task[0];
-    if (q < tend) band_info(P, P.flat[q], binfo, threadIdx.x, blockDim.x);
-    int tb = 0;     // binfo buffer of the current task
-    int nslot = 1;  // s_task slot of the next task
-    for (;; q = s_task[nslot], nslot ^= 3, tb ^= 1) {
-        if (q >= tend) break;
+    for (; q < tend; q = s_task[cb ^ 1], cb ^= 1) {
         const int tk = P.flat[q];
         const int z = tk >> 14, sv = tk & 16383;  // local slice, SV
         const int zg = P.z_offset + z;            // global slice
         const int gx0 = (sv % P.nsvx) * side, gy0 = (sv / P.nsvx) * side;
         const int tw = min(side, P.nx - gx0), th = min(side, P.ny - gy0);
+        const int tb = cb;
+        float* xt = (float*)(smem + L.xt) + cb * ntile;
+        const int* list = (const int*)(smem + L.list) + cb * S2;
+        const int* tof = (const int*)(smem + L.tof) + cb * S2;
+        const float* vscale = (const float*)(smem + L.vscale) + cb * S2;
+        const float* vth2 = (const float*)(smem + L.vth2) + cb * S2;
+        const int nactv = s_task[2 + cb];
         long long tp0 = 0, tp1 = 0, tp2 = 0, tp3 = 0;
         if (PROF && threadIdx.x == 0) tp0 = clock64();
-
-        // ---- 1. x tile (+1 halo ring, +-1 slice in 3-D) into shared memory
-        {
-            constexpr int XMAX = 2;  // tile entries per thread and round: all loads in flight
-            const int ntile = (NNB == 26 ? 3 : 1) * TW * TW;
-            for (int i0 = 0; i0 < ntile; i0 += XMAX * blockDim.x) {
-                float xv[XMAX];
-                bool inb[XMAX];
-#pragma unroll
-                for (int u = 0; u < XMAX; ++u) {
-                    const int i = i0 + threadIdx.x + u * blockDim.x;
-                    const int tz = i / (TW * TW), r = i % (TW * TW), ty = r / TW, tx = r % TW;
-                    const int gx = gx0 - 1 + tx, gy = gy0 - 1 + ty;
-                    const int zs = (NNB == 26) ? z + tz : z + 1;  // storage slice (halo at 0, nz+1)
-                    inb[u] = i < ntile && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny;
-                    const int cx = min(max(gx, 0), P.nx - 1), cy = min(max(gy, 0), P.ny - 1);
-                    xv[u] = i < ntile ? P.x[(size_t)min(zs, P.nz_local + 1) * plane + (size_t)cy * P.nx + cx] : 0.f;
-                }
-#pragma unroll
-                for (int u = 0; u < XMAX; ++u) {
-                    const int i = i0 + threadIdx.x + u * blockDim.x;
-                    if (i < ntile) xt[i] = inb[u] ? xv[u] : 0.f;
-                }
-            }
-        }
-        __syncthreads();
-
-        // ---- 2. zero-skip predicate at visit start (reading R9): slot v kept iff valid
-        //         and (skip inactive or x_j or an in-volume neighbour is non-zero)
-        int kept = 0;
-        for (int v0 = threadIdx.x; v0 < S2; v0 += blockDim.x) {
-            const int lx = v0 % side, ly = v0 / side;
-            int keep = 0;
-            if (lx < tw && ly < th) {
-                keep = 1;
-                if (P.zero_skip_active) {
-                    keep = xt[(zc * TW + ly + 1) * TW + lx + 1] != 0.f;
-                    for (int r = 0; r < P.pc.nnb && !keep; ++r) {
-                        const int dx = nbt[r], dy = nbt[32 + r], dz = nbt[64 + r];
-                        const int gx = gx0 + lx + dx, gy = gy0 + ly + dy, gz = zg + dz;
-                        if (gx < 0 || gx >= P.nx || gy < 0 || gy >= P.ny || gz < 0 || gz >= P.nz_total) continue;
-                        keep = xt[((zc + dz) * TW + ly + 1 + dy) * TW + lx + 1 + dx] != 0.f;
-                    }
-                }
-            }
-            flags[v0] = keep;
-            kept += keep;
-        }
-        if (!__syncthreads_or(kept)) {  // the whole SV is zero-skipped: account for it, next task
-            if (threadIdx.x == 0) {
-                P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
-                atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
-                atomicAdd(P.counters + 2, 1ull);
-                atomicAdd(P.counters + 3, 1ull);
-                s_task[nslot] = fetch_task();
-            }
-            __syncthreads();
-            if (s_task[nslot] < tend) band_info(P, P.flat[s_task[nslot]], binfo + (tb ^ 1) * VA, threadIdx.x, blockDim.x);
-            continue;  // the next task's x-tile barrier orders these writes before its pack
-        }
-
-        // ---- 3. visiting order (prior warp): one of NPERM host-drawn random permutations of the
-        //         tile, chosen per (seed, iteration, slice, SV) visit (raster order in
-        //         deterministic mode), compacted to the kept voxels with a warp ballot; per-voxel
-        //         scale and theta2 staged in smem; then the first pair's surrogate terms.
-        //         Delta warp: the next task.  View warps: the first R A records, then the pack.
         const size_t arec = (size_t)sv * S2;  // first A record of this SV
         constexpr int CB = U8 ? 4 : 16;       // record bytes per view position
         const int tpm = vw * 32 + lane;
         const unsigned char* g_code = (const unsigned char*)(U8 ? (const void*)P.A.codes : (const void*)P.A.vals) +
                                       ((size_t)arec * VA + tpm * VPT) * CB;
         const unsigned char* g_off = P.A.off + (size_t)arec * VA + tpm * VPT;
-        int nvis = 0;  // kept voxels of this visit (every warp computes it)
-        for (int base = 0; base < S2; base += 32) nvis += __popc(__ballot_sync(kFull, base + lane < S2 && flags[base + lane]));
-        const int nactv = nvis;
         // view thread: asynchronous copy of its own slice of voxel j's record into ring stage stg,
         // one commit group per voxel (empty past the visit's end)
         auto copy_record_to = [&](int j, int stg, int v) {
@@ -506,32 +588,13 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         };
         const int sbase = (int)(gseq % (uint32_t)R);  // ring stage of this visit's voxel 0
         const int cslot = (zc * TW + 1) * TW + 1;     // tile index of local (0,0)
+        // the first pair's surrogate terms (prior warp) and the next task's input copies (delta
+        // warp) while the view warps pack
         if (is_prior) {
-            const uint64_t h = mix64(P.seed ^ mix64(((uint64_t)P.iter << 40) ^ ((uint64_t)zg << 20) ^ (uint64_t)sv));
-            const uint8_t* perm = P.perm + (size_t)(h % (uint64_t)P.nperm) * S2;
-            int n = 0;
-            for (int base = 0; base < S2; base += 32) {
-                const int i = base + lane;
-                const int v = i < S2 ? (P.deterministic ? i : (int)perm[i]) : 0;
-                const bool k = i < S2 && flags[v];
-                const unsigned m = __ballot_sync(kFull, k);
-                if (k) {
-                    const int p = n + __popc(m & ((1u << lane) - 1));
-                    list[p] = v;
-                    tof[p] = ((v / side) << 8) | (v % side);  // packed (ly, lx): no div in the loop
-                }
-                n += __popc(m);
-            }
-            __syncwarp();
-            for (int i = lane; i < nactv; i += 32) {
-                const int v = list[i];
-                vscale[i] = P.A.scale[arec + v];
-                vth2[i] = P.theta2[((size_t)z * P.nsv + sv) * S2 + v];
-            }
             prior_pair(tof, 0, nactv, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + (pseq & 1));
             __syncwarp();
         } else if (is_delta) {
-            if (lane == 0) s_task[nslot] = fetch_task();
+            fetch_and_copy(cb ^ 1);
         }
         if (PROF && threadIdx.x == 0) tp1 = clock64();
 
@@ -576,7 +639,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 __syncwarp();
 #pragma unroll
                 for (int q4 = 0; q4 < 8; ++q4) {
-                    const float4 r = *(const float4*)(stg_w + lane * kStg + 4 * q4);
+                    const float4 r = lds128(stg_w + lane * kStg + 4 * q4);
                     const float rv[4] = {r.x, r.y, r.z, r.w};
 #pragma unroll
                     for (int j = 0; j < 4; ++j)
@@ -893,7 +956,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 __syncwarp();
             }
         } else if (is_delta) {
-            // the image and the counters
+            // the image and the counters, then the next task's preparation (with the prior warp)
             for (int i = lane; i < tw * th; i += 32) {
                 const int lx = i % tw, ly = i / tw;
                 P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] = xt[cslot + ly * TW + lx];
@@ -905,42 +968,9 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 atomicAdd(P.counters + 2, 1ull);
                 atomicAdd(P.sum_delta, (double)amount);
             }
+            finish_prepare(cb ^ 1);
         } else if (is_prior) {
-            // the next task's band info, with an L2 warm-up of its band rows (the next pack
-            // then reads L2)
-            const int nq = s_task[nslot];
-            if (nq < tend) {
-                const int nt = P.flat[nq];
-                constexpr int KMAX = 6;  // views per lane and pass: all loads in flight at once
-                const int psv = nt & 16383, pz = nt >> 14;
-                uint32_t* dst = binfo + (tb ^ 1) * VA;
-                const float* wz = P.w + (size_t)pz * V * M;
-                const float* ez = P.e + (size_t)pz * V * M;
-#pragma unroll 1
-                for (int k0 = 0; k0 < V; k0 += 32 * KMAX) {
-                    int bs[KMAX], bwd[KMAX];
-#pragma unroll
-                    for (int i = 0; i < KMAX; ++i) {
-                        const int k = k0 + lane + 32 * i;
-                        if (k < V) {
-                            bs[i] = P.A.band_start[(size_t)psv * V + k];
-                            bwd[i] = P.A.band_width[(size_t)psv * V + k];
-                        }
-                    }
-#pragma unroll
-                    for (int i = 0; i < KMAX; ++i) {
-                        const int k = k0 + lane + 32 * i;
-                        if (k < V) {
-                            const int r = k * M + bs[i], r1 = r + max(bwd[i], 1) - 1;
-                            dst[k] = ((uint32_t)r << 5) | (uint32_t)bwd[i];
-                            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
-                            asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
-                            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
-                            asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r1));
-                        }
-                    }
-                }
-            }
+            finish_prepare(cb ^ 1);
         }
         __syncthreads();
         if (PROF && threadIdx.x == 0) {
@@ -965,7 +995,7 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
     constexpr int R = ring_depth(U8);
     auto kern = p.tprof ? k_svicd<VPT, U8, NNB, R, true> : k_svicd<VPT, U8, NNB, R, false>;
     IcdParams q = p;
-    q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT);
+    q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT, p.V);
     const int smem = q.lay.total;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
@@ -979,14 +1009,14 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
 
 int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
 {
-    return svicd_layout(p.rows, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw, vpt).total;
+    return svicd_layout(p.rows, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw, vpt, p.V).total;
 }
 
 template <int VPT, bool U8, int NNB>
 int resident_t(const IcdParams& p)
 {
     auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), false>;
-    const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT).total;
+    const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT, p.V).total;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
     cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     int nb = 0, dev = 0, nsm = 0;

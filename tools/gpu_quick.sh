@@ -1,9 +1,9 @@
 #!/bin/bash
-# Quick GPU check of the update kernel (outputs under gpurun_out/): hook tests, then timings.
+# Quick GPU check of the update kernel (outputs under gpurun_out/): hook tests, A/B timing vs the
+# round-1 kernel, phase profile, then the whole GPU suite.
 timeout 300 python -m pytest tests/test_gpu_hooks.py -x -q -s > gpurun_out/q_hooks.log 2>&1
 echo "hooks rc=$?" >> gpurun_out/q_hooks.log
+rm -f gpurun_out/ab_libmbir_r1.so.log; bash tools/gpu_ab.sh libmbir_r1.so 6
 MBIR_PHASE_PROFILE=1 timeout 200 python tools/iter_profile.py --iters 6 > gpurun_out/q_iter_cfg4_prof.log 2>&1
-timeout 200 python tools/iter_profile.py --iters 12 > gpurun_out/q_iter_cfg4.log 2>&1
-timeout 200 python tools/iter_profile.py --config cfg3 --iters 8 > gpurun_out/q_iter_cfg3.log 2>&1
 timeout 900 python -m pytest tests -q -m gpu -x -p no:cacheprovider > gpurun_out/q_pytest_gpu.log 2>&1
 echo "gpu rc=$?" >> gpurun_out/q_pytest_gpu.log
