@@ -224,6 +224,16 @@ int mbir_get_sysmatrix_columns(mbir_handle* h, const int64_t* voxels, int n, int
 int mbir_probe_update(mbir_handle* h, const int64_t* voxels, int n, float* theta1,
                       float* theta2, float* delta);
 
+/* Test hook (the z-slab partition of DESIGN.md section 9 without several GPUs): link n handles
+ * created on ONE device with nranks = n, rank = i, no NCCL id, owning consecutive slabs of one
+ * volume (rank order), so that their halo exchanges (mbir_halo_plan) become device-to-device
+ * copies between the handles behind a host barrier.  The caller must then drive all of them
+ * concurrently (one host thread per handle) with the same sequence of collective calls
+ * (set_image, init_fbp, iterate, reconstruct).  Counters and RMSE are NOT reduced across linked
+ * handles (each reports its own slab).  Errors: EINVAL (wrong ranks/order/device, already
+ * linked), ENOMEM. */
+int mbir_link_slabs(mbir_handle** handles, int n);
+
 /* Test hook: record every voxel update the fused update kernel executes from now on -- the
  * (theta1, theta2, delta) of Alg. 1 steps 3-8 exactly as the kernel's delta chain
  * used them (theta1 of the second voxel of a pair includes the first one's update of e, so it

@@ -16,6 +16,10 @@ from .api import (  # noqa: F401
     mbir_get_sysmatrix,
     mbir_get_sysmatrix_columns,
     mbir_iterate,
+    mbir_link_slabs,
+    mbir_get_update_dump,
+    mbir_set_update_dump,
+    mbir_get_schedule,
     mbir_nccl_unique_id,
     mbir_probe_update,
     mbir_query_sizes,

@@ -27,6 +27,7 @@ EXPORTS = (
     "mbir_get_error_sinogram", "mbir_rmse_hu", "mbir_query_sizes", "mbir_get_sysmatrix",
     "mbir_get_sysmatrix_columns",
     "mbir_probe_update", "mbir_set_update_dump", "mbir_get_update_dump", "mbir_get_schedule",
+    "mbir_link_slabs",
     "mbir_nccl_unique_id", "mbir_halo_plan", "mbir_destroy",
     "mbir_strerror", "mbir_last_error",
 )
@@ -132,6 +133,8 @@ def load(path: str = LIB_PATH):
     L.mbir_get_sysmatrix_columns.argtypes = [H, vp, C.c_int, vp, vp, vp, vp, vp]
     L.mbir_probe_update.restype = C.c_int
     L.mbir_probe_update.argtypes = [H, vp, C.c_int, vp, vp, vp]
+    L.mbir_link_slabs.restype = C.c_int
+    L.mbir_link_slabs.argtypes = [C.POINTER(C.c_void_p), C.c_int]
     L.mbir_set_update_dump.restype = C.c_int
     L.mbir_set_update_dump.argtypes = [H, C.c_int64]
     L.mbir_get_update_dump.restype = C.c_int

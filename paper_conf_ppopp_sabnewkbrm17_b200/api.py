@@ -18,7 +18,7 @@ __all__ = [
     "mbir_reconstruct", "mbir_iterate", "mbir_get_image", "mbir_get_error_sinogram",
     "mbir_rmse_hu", "mbir_query_sizes", "mbir_get_sysmatrix", "mbir_get_sysmatrix_columns",
     "mbir_probe_update", "mbir_set_update_dump", "mbir_get_update_dump", "mbir_get_schedule",
-    "mbir_nccl_unique_id", "mbir_destroy", "Reconstructor",
+    "mbir_link_slabs", "mbir_nccl_unique_id", "mbir_destroy", "Reconstructor",
 ]
 
 
@@ -246,6 +246,12 @@ def mbir_probe_update(h, voxels):
     L.check(L.load().mbir_probe_update(h, vox.ctypes.data, n, t1.ctypes.data, t2.ctypes.data,
                                        dl.ctypes.data), h, "mbir_probe_update")
     return t1, t2, dl
+
+
+def mbir_link_slabs(handles):
+    """Test hook: link handles of consecutive slabs on one device (include/mbir.h)."""
+    arr = (C.c_void_p * len(handles))(*[h.value if isinstance(h, C.c_void_p) else h for h in handles])
+    L.check(L.load().mbir_link_slabs(arr, len(handles)), None, "mbir_link_slabs")
 
 
 def mbir_set_update_dump(h, capacity: int):

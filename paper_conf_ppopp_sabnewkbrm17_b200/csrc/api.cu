@@ -13,6 +13,8 @@
 #include <string.h>
 
 #include <algorithm>
+#include <condition_variable>
+#include <mutex>
 #include <new>
 #include <string>
 #include <vector>
@@ -72,6 +74,30 @@ NcclApi& nccl()
 
 }  // namespace
 
+struct mbir_handle;
+
+// Test hook (mbir_link_slabs): handles owning consecutive slabs of one volume on ONE device,
+// exchanging halo slices by device-to-device copies behind a host barrier instead of NCCL.
+struct LocalGroup {
+    std::mutex mu;
+    std::condition_variable cv;
+    int n = 0, arrived = 0;
+    unsigned long long generation = 0;
+    std::vector<mbir_handle*> members;  // by rank
+    void barrier()
+    {
+        std::unique_lock<std::mutex> lk(mu);
+        const unsigned long long gen = generation;
+        if (++arrived == n) {
+            arrived = 0;
+            ++generation;
+            cv.notify_all();
+        } else {
+            cv.wait(lk, [&] { return generation != gen; });
+        }
+    }
+};
+
 struct mbir_handle {
     mbir_geometry g{};
     std::vector<double> angles;
@@ -82,6 +108,7 @@ struct mbir_handle {
     bool own_stream = false;
     int rank = 0, nranks = 1;
     ncclComm_t comm = nullptr;
+    LocalGroup* lg = nullptr;  // mbir_link_slabs group (shared by its members; rank 0 frees it)
     int side = 0, nsvx = 0, nsvy = 0, nsv = 0, S2 = 0, nsv_pad = 0;
     int rows = 0, band_max = 0;
     int vpt = 1, nvw = 0, Vs = 0, threads = 0, smem = 0, blocks_per_sm = 1, nsm = 148;
@@ -198,6 +225,27 @@ int exchange_halo(mbir_handle* h, int parity)
     int32_t ops[4][3];
     const int n = mbir_halo_plan(h->g.z_offset, h->g.nz_local, h->rank, h->nranks, parity, &ops[0][0]);
     if (n < 0) return fail(h, MBIR_EINVAL, "bad halo plan");
+    if (!h->comm) {
+        // linked slabs on one device (test hook): every member has finished the half (stream
+        // synchronised) when the barrier opens; each then copies the peers' boundary slices it
+        // receives into its halo.  The next half only writes slices of the other parity, and the
+        // member cannot reach the next exchange before this copy completed, so one barrier per
+        // exchange orders everything.
+        if (!h->lg) return fail(h, MBIR_ESTATE, "nranks > 1 without NCCL: call mbir_link_slabs first");
+        CK(cudaStreamSynchronize(h->st));
+        h->lg->barrier();
+        for (int i = 0; i < n; ++i) {
+            if (ops[i][1]) continue;  // sends are the peer's receives
+            const mbir_handle* p = h->lg->members[ops[i][0]];
+            // my lower halo (0) <- the peer's last slice; my upper halo (nz + 1) <- its first
+            const int src = ops[i][2] == 0 ? p->g.nz_local : 1;
+            CK(cudaMemcpyAsync(h->d_x + (size_t)ops[i][2] * pl, p->d_x + (size_t)src * pl, pl * 4,
+                               cudaMemcpyDeviceToDevice, h->st));
+        }
+        CK(cudaStreamSynchronize(h->st));
+        h->lg->barrier();
+        return MBIR_OK;
+    }
     NcclApi& N = nccl();
     CKN(N.GroupStart());
     for (int i = 0; i < n; ++i) {
@@ -350,7 +398,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
                 if (r) return r;
             }
         }
-        if (h->nranks > 1) {
+        if (h->nranks > 1 && h->comm) {
             CKN(nccl().AllReduce(h->d_counters, h->d_counters, 4, ncclUint64, ncclSum, h->comm, h->st));
             CKN(nccl().AllReduce(h->d_sum_delta, h->d_sum_delta, 1, ncclFloat64, ncclSum, h->comm, h->st));
         }
@@ -526,6 +574,16 @@ void mbir_destroy(mbir_handle* h)
     if (h->ev1) cudaEventDestroy(h->ev1);
     for (cudaEvent_t e : h->kev) cudaEventDestroy(e);
     if (h->comm && nccl().CommDestroy) nccl().CommDestroy(h->comm);
+    if (h->lg) {
+        LocalGroup* g = h->lg;
+        bool last = false;
+        {
+            std::lock_guard<std::mutex> lk(g->mu);
+            g->members[h->rank] = nullptr;
+            last = std::all_of(g->members.begin(), g->members.end(), [](mbir_handle* m) { return m == nullptr; });
+        }
+        if (last) delete g;
+    }
     if (h->own_stream && h->st) cudaStreamDestroy(h->st);
     delete h;
 }
@@ -580,7 +638,8 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
             return (fail(h, MBIR_EINVAL, "nz_local too large: at most " + std::to_string(kMaxPhaseSlices) +
                                              " slices per z-parity phase per rank"), bail(MBIR_EINVAL));
     }
-    if (h->nranks > 1 && (!d || !d->nccl_unique_id || h->rank < 0 || h->rank >= h->nranks))
+    // nranks > 1 needs an NCCL id -- or none, for slabs linked on one device by mbir_link_slabs
+    if (h->nranks > 1 && (!d || h->rank < 0 || h->rank >= h->nranks))
         return bail(MBIR_EINVAL);
     if (G.angles) h->angles.assign(G.angles, G.angles + G.nviews);
     h->g.angles = nullptr;
@@ -700,6 +759,11 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_y, ns + 32))) return bail(r);
     if ((r = dalloc(h, &h->d_w, ns + 32))) return bail(r);
     if ((r = dalloc(h, &h->d_e, ns + 32))) return bail(r);
+    // the pack reads whole 16-byte-aligned 32-float windows around band rows, up to 32 floats past
+    // the last row: the padding is zero, never uninitialised
+    cudaMemsetAsync(h->d_y, 0, (ns + 32) * 4, h->st);
+    cudaMemsetAsync(h->d_w, 0, (ns + 32) * 4, h->st);
+    cudaMemsetAsync(h->d_e, 0, (ns + 32) * 4, h->st);
     if ((r = dalloc(h, &h->d_x, pl * (G.nz_local + 2)))) return bail(r);
     if ((r = dalloc(h, &h->d_theta2, (size_t)G.nz_local * h->nsv * h->S2))) return bail(r);
     if ((r = dalloc(h, &h->d_amount, (size_t)G.nz_local * h->nsv))) return bail(r);
@@ -771,7 +835,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     }
 
     // ---- multi-GPU communicator (z-slab partition)
-    if (h->nranks > 1) {
+    if (h->nranks > 1 && d->nccl_unique_id) {
         NcclApi& N = nccl();
         if (!N.ok) return (fail(h, MBIR_ENOTSUP, "libnccl.so.2 not found"), bail(MBIR_ENOTSUP));
         ncclUniqueId id;
@@ -835,7 +899,7 @@ int mbir_set_image(mbir_handle* h, const float* x0, int where)
         CK(cudaMemcpyAsync(tmp, x0, n * 4, kind_in(where), h->st));
         CK(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->st));
         CK(launch_check_finite(tmp, (int64_t)n, h->pr.positivity, h->d_flag, h->st));
-        if (h->nranks > 1) CKN(nccl().AllReduce(h->d_flag, h->d_flag, 1, ncclInt32, ncclMax, h->comm, h->st));
+        if (h->comm) CKN(nccl().AllReduce(h->d_flag, h->d_flag, 1, ncclInt32, ncclMax, h->comm, h->st));
         int flag = 0;
         CK(cudaMemcpyAsync(&flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost, h->st));
         CK(cudaStreamSynchronize(h->st));
@@ -886,6 +950,9 @@ int mbir_init_fbp(mbir_handle* h)
 int mbir_reconstruct(mbir_handle* h, double equits, mbir_stats* st)
 {
     if (!h || !(equits >= 0)) return MBIR_EINVAL;
+    // linked slabs do not reduce their counters, so an equit target could stop them after
+    // different iteration counts: they run fixed iteration counts (mbir_iterate)
+    if (h->lg) return fail(h, MBIR_ENOTSUP, "linked slabs (mbir_link_slabs) run mbir_iterate only");
     return run_iterations(h, -1, equits, st);
 }
 
@@ -925,7 +992,7 @@ int mbir_rmse_hu(mbir_handle* h, const float* golden, int where, double mu_water
     }
     CK(cudaMemsetAsync(h->d_acc, 0, sizeof(double), h->st));
     CK(launch_rmse_partial(h->d_x + pl, g, (int64_t)n, h->d_acc, h->st));
-    if (h->nranks > 1) CKN(nccl().AllReduce(h->d_acc, h->d_acc, 1, ncclFloat64, ncclSum, h->comm, h->st));
+    if (h->comm) CKN(nccl().AllReduce(h->d_acc, h->d_acc, 1, ncclFloat64, ncclSum, h->comm, h->st));
     double s = 0.0;
     CK(cudaMemcpyAsync(&s, h->d_acc, sizeof(double), cudaMemcpyDeviceToHost, h->st));
     if (tmp) CK(cudaFreeAsync(tmp, h->st));
@@ -1007,6 +1074,24 @@ int mbir_get_sysmatrix_columns(mbir_handle* h, const int64_t* voxels, int n, int
     for (int i = 0; i < n; ++i)
         if (voxels[i] < 0 || voxels[i] >= (int64_t)plane_elems(h)) return fail(h, MBIR_EINVAL, "voxel index out of range");
     return export_sysmatrix(h, voxels, n, first, count, values, codes, scales);
+}
+
+int mbir_link_slabs(mbir_handle** hs, int n)
+{
+    if (!hs || n < 2) return MBIR_EINVAL;
+    for (int i = 0; i < n; ++i) {
+        mbir_handle* h = hs[i];
+        if (!h || h->nranks != n || h->rank != i || h->comm || h->lg) return MBIR_EINVAL;
+        if (h->device != hs[0]->device) return fail(h, MBIR_EINVAL, "linked slabs must share one device");
+        if (i > 0 && h->g.z_offset != hs[i - 1]->g.z_offset + hs[i - 1]->g.nz_local)
+            return fail(h, MBIR_EINVAL, "linked slabs must be consecutive in rank order");
+    }
+    LocalGroup* g = new (std::nothrow) LocalGroup();
+    if (!g) return MBIR_ENOMEM;
+    g->n = n;
+    g->members.assign(hs, hs + n);
+    for (int i = 0; i < n; ++i) hs[i]->lg = g;
+    return MBIR_OK;
 }
 
 int mbir_set_update_dump(mbir_handle* h, int64_t capacity)

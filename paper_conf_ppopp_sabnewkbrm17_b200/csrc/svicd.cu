@@ -106,9 +106,11 @@ __device__ __forceinline__ float4 lds128(const float* p)
     asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(smem_u32(p)));
     return v;
 }
-// named barriers: sync (wait for `n` threads incl. this warp) / arrive (count and go on)
-__device__ __forceinline__ void bar_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
-__device__ __forceinline__ void bar_arrive(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+// named barriers: sync (wait for `n` threads incl. this one) / arrive (count and go on).  The
+// non-.aligned forms: the role warps reach them right after lane-0-only work, and the aligned
+// bar.sync / bar.arrive would require the warp to be converged there (compute-sanitizer synccheck)
+__device__ __forceinline__ void bar_sync(int id, int n) { asm volatile("barrier.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+__device__ __forceinline__ void bar_arrive(int id, int n) { asm volatile("barrier.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
 // A values of a voxel re-indexed to another voxel's channels: r[i] = A[i + d] (0 outside), as
 // channel pairs
@@ -728,6 +730,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             // refill two ring stages with the records R voxels ahead (one commit group per voxel,
             // empty past the visit's end, keeps the wait counts fixed)
             auto refill = [&](int j, int sj) {
+                if (VPT != 4) __syncwarp();  // lanes read offset words another lane refills
                 const int s1 = sj + 1 == R ? 0 : sj + 1;
                 copy_record_to(j + R, sj, j + R < nactv ? list[j + R] : 0);
                 copy_record_to(j + 1 + R, s1, j + 1 + R < nactv ? list[j + 1 + R] : 0);
