@@ -235,8 +235,9 @@ constexpr int kNSL = 16;  // partial-sum slots per quantity in the pair exchange
 constexpr int kTileW = 4;
 __host__ __device__ constexpr int tile_warps(int va) { return va / (32 * kTileW); }
 
-// threads per CTA: VPT 4 -> <= 6 view warps, VPT 2 -> <= 12, VPT 1 -> <= 4; + delta + prior warps
-__host__ __device__ constexpr int max_threads(int vpt) { return vpt == 2 ? 448 : 256; }
+// threads per CTA: VPT 4 -> <= 6 view warps, VPT 3 -> <= 8, VPT 2 -> <= 12, VPT 1 -> <= 4;
+// + the delta and prior warps
+__host__ __device__ constexpr int max_threads(int vpt) { return vpt == 2 ? 448 : vpt == 3 ? 320 : 256; }
 
 // named barriers of the pair protocol (0 is __syncthreads)
 constexpr int kBarA = 1;  // view warps' partials + the prior warp's terms of a pair are ready
@@ -322,6 +323,10 @@ __device__ __forceinline__ void load_words(const unsigned char* stg, int off_in_
         }
     }
     if (VPT == 4) ob = ((const uint32_t*)(stg + off_in_stage))[tp];
+    if (VPT == 3) {
+        const unsigned char* o3 = stg + off_in_stage + 3 * tp;
+        ob = (uint32_t)o3[0] | ((uint32_t)o3[1] << 8) | ((uint32_t)o3[2] << 16);
+    }
     if (VPT == 2) ob = ((const uint16_t*)(stg + off_in_stage))[tp];
     if (VPT == 1) ob = stg[off_in_stage + tp];
 }
@@ -578,13 +583,19 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                     else if (VPT == 2)
                         cp_async8(st + tpm * 8, gc);
                     else
-                        cp_async4(st + tpm * 4, gc);
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t) cp_async4(st + (tpm * VPT + t) * 4, gc + t * 4);
                 } else {
 #pragma unroll
                     for (int t = 0; t < VPT; ++t) cp_async16(st + (tpm * VPT + t) * 16, gc + t * 16);
                 }
-                if ((tpm & (4 / VPT - 1)) == 0)  // offsets: VPT bytes per thread, as 4-byte words
+                if (VPT == 3) {  // offsets: 3 bytes per thread, 4 threads' 12 bytes as 3 words
+                    if ((tpm & 3) == 0)
+#pragma unroll
+                        for (int t = 0; t < 3; ++t) cp_async4(st + L.off_in_stage + tpm * 3 + 4 * t, g_off + (size_t)v * VA + 4 * t);
+                } else if ((tpm & (4 / VPT - 1)) == 0) {  // offsets: VPT bytes per thread, as 4-byte words
                     cp_async4(st + L.off_in_stage + tpm * VPT, g_off + (size_t)v * VA);
+                }
             }
             cp_async_commit();
         };
@@ -1031,6 +1042,10 @@ int resident_t(const IcdParams& p)
 
 int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize)
 {
+    if (vpt == 3) {
+        if (quantize) return nnb == 26 ? resident_t<3, true, 26>(p) : resident_t<3, true, 8>(p);
+        return nnb == 26 ? resident_t<3, false, 26>(p) : resident_t<3, false, 8>(p);
+    }
     if (vpt == 2) {
         if (quantize) return nnb == 26 ? resident_t<2, true, 26>(p) : resident_t<2, true, 8>(p);
         return nnb == 26 ? resident_t<2, false, 26>(p) : resident_t<2, false, 8>(p);
@@ -1047,6 +1062,10 @@ int svicd_scratch_floats(int vpt) { return svb_cols(vpt) * 32; }
 
 cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid, cudaStream_t st)
 {
+    if (vpt == 3) {
+        if (quantize) return nnb == 26 ? launch_t<3, true, 26>(p, grid, st) : launch_t<3, true, 8>(p, grid, st);
+        return nnb == 26 ? launch_t<3, false, 26>(p, grid, st) : launch_t<3, false, 8>(p, grid, st);
+    }
     if (vpt == 2) {
         if (quantize) return nnb == 26 ? launch_t<2, true, 26>(p, grid, st) : launch_t<2, true, 8>(p, grid, st);
         return nnb == 26 ? launch_t<2, false, 26>(p, grid, st) : launch_t<2, false, 8>(p, grid, st);
