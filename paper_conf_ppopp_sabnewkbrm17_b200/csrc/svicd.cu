@@ -112,106 +112,49 @@ __device__ __forceinline__ float4 lds128(const float* p)
 __device__ __forceinline__ void bar_sync(int id, int n) { asm volatile("barrier.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 __device__ __forceinline__ void bar_arrive(int id, int n) { asm volatile("barrier.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
-// A values of a voxel re-indexed to another voxel's channels: r[i] = A[i + d] (0 outside), as
-// channel pairs
-template <bool U8>
-__device__ __forceinline__ void shifted(uint32_t cw, const float2 (&a)[2], int d, float2 (&r)[2])
-{
-    if (U8) {
-        // one PRMT: byte i of s = byte i + d of cw, or 0 (selector nibble 4 = byte 0 of the zero
-        // operand); the selector nibbles are read out of 0x444432104444 at nibble 4 + d
-        const int dc = max(-4, min(4, d));
-        const uint32_t sel = (uint32_t)(0x444432104444ull >> (16 + 4 * dc));
-        const uint32_t s = __byte_perm(cw, 0u, sel);
-        r[0] = dq2(s, 0);
-        r[1] = dq2(s, 2);
-        return;
-    }
-    const float v[4] = {a[0].x, a[0].y, a[1].x, a[1].y};
-    float q[4];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-        const int j = i + d;
-        q[i] = j == 0 ? v[0] : j == 1 ? v[1] : j == 2 ? v[2] : j == 3 ? v[3] : 0.f;
-    }
-    r[0] = make_float2(q[0], q[1]);
-    r[1] = make_float2(q[2], q[3]);
-}
-
-// Neighbour slots of a prior-warp lane: half-warp h = lane >> 4 works on voxel a (h = 0) or b
-// (h = 1) of a pair; its lane i owns neighbours i and i + 16 of the neighbourhood (reading R2):
-// offset (dx, dy, dz), tile-index offset dt and weight w (0: no neighbour)
-struct NbrLane {
-    int dx[2], dy[2], dz[2], dt[2];
-    float w[2];
+// The prior warp's lane r owns neighbour r of the neighbourhood (reading R2): offset (dx, dy, dz),
+// tile-index offset dt and weight w (0: no neighbour / lane r >= 26)
+struct NbrOne {
+    int dx, dy, dz, dt;
+    float w;
 };
 
-// surrogate terms of a pair of consecutive voxels (a, b): a's sums, b's sums computed with a's
-// OLD value, and -- if a is b's neighbour -- that neighbour's term (btab) and weight (bab)
-struct PriPair {
-    float sa, sxa, va, sb, sxb, vb, btab, bab;
+// surrogate terms of voxel i of the visiting order, computed from the x tile in which every update
+// before voxel i - 1 is applied and voxel i - 1 still has its OLD value: the sums
+// s = sum_r b_r phi(v - x_r), sx = sum_r b_r phi(v - x_r) x_r (Alg1:7, reading R1; free boundary),
+// v = x_i, and -- if voxel i - 1 is a neighbour of i -- that neighbour's term (btu) and weight
+// (bwu), which the delta warp replaces by the term at i - 1's new value: exact sequential ICD
+struct PriTerm {
+    float s, sx, v, btu, bwu;
 };
 
-// prior warp: PriPair for voxels (i0, i0+1) of the visiting order from the current x tile.
-// Alg1:7's q-GGMRF surrogate sums sb = sum_r b_r phi(v - x_r), sx = sum_r b_r phi(v - x_r) x_r
-// over the neighbourhood (free boundary: off-volume neighbours contribute nothing), voxel a on
-// lanes 0-15 and voxel b (with a's OLD value) on lanes 16-31, two neighbours per lane.
-__device__ __forceinline__ void prior_pair(const int* tof, int i0, int nact, const float* xt, int cslot,
-                                           int TW, int gx0, int gy0, int zg, const IcdParams& P,
-                                           const NbrLane& nb, int lane, PriPair* out)
+__device__ __forceinline__ void prior_one(const int* tof, int i, const float* xt, int cslot, int TW, int gx0,
+                                          int gy0, int zg, const IcdParams& P, const NbrOne& nb, int lane,
+                                          PriTerm* out)
 {
-    const bool hasb = i0 + 1 < nact;
-    const int ta = tof[i0], tb = hasb ? tof[i0 + 1] : ta;
-    const int tv = lane < 16 ? ta : tb;
+    const int tv = tof[i];
     const int lx = tv & 255, ly = tv >> 8;
     const int c0 = cslot + ly * TW + lx;
     const float v = xt[c0];
-    float sb = 0.f, sx = 0.f, btn = 0.f, bwn = 0.f;  // btn, bwn: this lane's term / weight whose
-    bool mine = false;                               // neighbour is voxel a
-    const int dxa = (ta & 255) - lx, dya = (ta >> 8) - ly;  // a relative to this half's voxel
-    float xr[2];
-    bool ok[2];
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-        const int gx = gx0 + lx + nb.dx[k], gy = gy0 + ly + nb.dy[k], gz = zg + nb.dz[k];
-        ok[k] = nb.w[k] != 0.f && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total;
-        xr[k] = xt[c0 + nb.dt[k]];  // always inside the tile (its ring covers the neighbourhood)
+    const int gx = gx0 + lx + nb.dx, gy = gy0 + ly + nb.dy, gz = zg + nb.dz;
+    const bool ok = nb.w != 0.f && gx >= 0 && gx < P.nx && gy >= 0 && gy < P.ny && gz >= 0 && gz < P.nz_total;
+    const float xr = xt[c0 + nb.dt];  // always inside the tile (its ring covers the neighbourhood)
+    const float bt = ok ? nb.w * phi_f(P.pc, v - xr) : 0.f;
+    float s = bt, sx = bt * xr;
+    bool mine = false;
+    if (i > 0) {
+        const int tu = tof[i - 1];
+        mine = ok && nb.dz == 0 && nb.dx == (tu & 255) - lx && nb.dy == (tu >> 8) - ly;
     }
 #pragma unroll
-    for (int k = 0; k < 2; ++k) {
-        const float bt = ok[k] ? nb.w[k] * phi_f(P.pc, v - xr[k]) : 0.f;
-        sb += bt;
-        sx += bt * xr[k];
-        if (ok[k] && nb.dz[k] == 0 && nb.dx[k] == dxa && nb.dy[k] == dya) {
-            btn = bt;
-            bwn = nb.w[k];
-            mine = true;
-        }
-    }
-#pragma unroll
-    for (int o = 8; o > 0; o >>= 1) {
-        sb += __shfl_xor_sync(kFull, sb, o);
+    for (int o = 16; o > 0; o >>= 1) {
+        s += __shfl_xor_sync(kFull, s, o);
         sx += __shfl_xor_sync(kFull, sx, o);
     }
-    // a's neighbour term in b's sums (a and b are distinct voxels, so only lanes >= 16 can own it)
-    const unsigned who = __ballot_sync(kFull, mine && lane >= 16 && hasb);
+    const unsigned who = __ballot_sync(kFull, mine);
     const int src = who ? __ffs(who) - 1 : 0;
-    const float btab = __shfl_sync(kFull, btn, src);
-    const float bab = __shfl_sync(kFull, bwn, src);
-    const float sbb = __shfl_sync(kFull, sb, 16), sxb = __shfl_sync(kFull, sx, 16), vb = __shfl_sync(kFull, v, 16);
-    if (lane == 0) {
-        PriPair pp{sb, sx, v, 0.f, 0.f, 0.f, 0.f, 0.f};
-        if (hasb) {
-            pp.sb = sbb;
-            pp.sxb = sxb;
-            pp.vb = vb;
-            if (who) {
-                pp.btab = btab;
-                pp.bab = bab;
-            }
-        }
-        *out = pp;
-    }
+    const float btu = __shfl_sync(kFull, bt, src), bwu = __shfl_sync(kFull, nb.w, src);
+    if (lane == 0) *out = PriTerm{s, sx, v, who ? btu : 0.f, who ? bwu : 0.f};
 }
 
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
@@ -259,8 +202,8 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     L.list = o;  o = align16(o + 2 * S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
     L.tof = o;   o = align16(o + 2 * S2 * 4);
-    L.red = o;   o = align16(o + 2 * 3 * kNSL * 4);  // [2 bufs][3 quantities][kNSL view warps]
-    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriPair));
+    L.red = o;   o = align16(o + 2 * kNSL * 4);  // [2 steps][kNSL view warps] theta1 partials
+    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriTerm));
     L.vscale = o; o = align16(o + 2 * S2 * 4);
     L.vth2 = o;  o = align16(o + 2 * S2 * 4);
     L.misc = o;  o = align16(o + 16 * 4);
@@ -349,11 +292,11 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     float* sb = (float*)(smem + L.sb_e);   // e row r at sb + r RS, w row r at sb + r RS + VS
     int* flags = (int*)(smem + L.flags);
     float* red = (float*)(smem + L.red);
-    PriPair* pri = (PriPair*)(smem + L.pri);
+    PriTerm* pri = (PriTerm*)(smem + L.pri);
     unsigned char* astage = smem + L.astage;
     float* stg_w = (float*)(smem + L.staging) + vw * 32 * kStg;
     int* s_task = (int*)(smem + L.misc);            // [b]: the task prepared in buffer b, [2 + b]: its kept voxels
-    float* dslot = (float*)(smem + L.misc) + 4;     // [2 pairs][2]: scale_a delta_a, scale_b delta_b
+    float* dslot = (float*)(smem + L.misc) + 4;     // [2 steps]: scale * delta of the step's voxel
     uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA]
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
@@ -362,7 +305,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     const int nab = (nvw + 2) * 32;      // barrier A: view warps + delta warp + prior warp
     const int nb2 = (nvw + 1) * 32;      // barrier B: view warps + the delta warp
 
-    for (int i = threadIdx.x; i < 2 * 3 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
+    for (int i = threadIdx.x; i < 2 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
     // the neighbourhood (reading R2) as shared-memory tables [dx | dy | dz | weight bits][32]: a
     // by-value kernel parameter indexed by a run-time value would be copied to local memory
     int* nbt = (int*)(smem + L.mbar);
@@ -383,18 +326,13 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
 #pragma unroll
     for (int t = 0; t < VPT; ++t) kv[t] = (vw * VPT + t) * 32 + lane;
     uint32_t gseq = 0;  // running voxel sequence number of this CTA: A stage = gseq % R
-    uint32_t pseq = 0;  // running voxel-pair number: exchange buffers pseq & 1
-    // prior-warp lane r owns neighbour r (and r + 16): offsets and weights in registers
-    NbrLane nb;
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-        const int r = (lane & 15) + 16 * k;
-        nb.dx[k] = nbt[r];
-        nb.dy[k] = nbt[32 + r];
-        nb.dz[k] = nbt[64 + r];
-        nb.w[k] = __int_as_float(nbt[96 + r]);
-        nb.dt[k] = (nb.dz[k] * (side + 2) + nb.dy[k]) * (side + 2) + nb.dx[k];
-    }
+    // prior-warp lane r owns neighbour r: offsets and weights in registers
+    NbrOne nb;
+    nb.dx = nbt[lane];
+    nb.dy = nbt[32 + lane];
+    nb.dz = nbt[64 + lane];
+    nb.w = __int_as_float(nbt[96 + lane]);
+    nb.dt = nbt[128 + lane];
 
     // this launch's batch: flat tasks [start, end) of the phase list (sched.cu k_flatten), pulled
     // one at a time by the persistent CTAs (dynamic distribution, Alg3:4 / T3); with the zero-skip
@@ -601,10 +539,10 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         };
         const int sbase = (int)(gseq % (uint32_t)R);  // ring stage of this visit's voxel 0
         const int cslot = (zc * TW + 1) * TW + 1;     // tile index of local (0,0)
-        // the first pair's surrogate terms (prior warp) and the next task's input copies (delta
+        // the first voxel's surrogate terms (prior warp) and the next task's input copies (delta
         // warp) while the view warps pack
         if (is_prior) {
-            prior_pair(tof, 0, nactv, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + (pseq & 1));
+            prior_one(tof, 0, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + (gseq & 1));
             __syncwarp();
         } else if (is_delta) {
             fetch_and_copy(cb ^ 1);
@@ -676,22 +614,24 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         __syncthreads();
         if (PROF && threadIdx.x == 0) tp2 = clock64();
 
-        // ---- 5. the voxel loop, TWO voxels (a, b) per step, exactly sequential ICD
+        // ---- 5. the voxel loop, exactly sequential ICD one voxel per step: the view warps gather
+        //         theta1's partials of voxel i from e (after voxel i - 1's scatter) and arrive on A;
+        //         the delta warp (A also waits for the prior warp's terms of i) writes voxel i - 1's
+        //         new value into the x tile (releasing the prior warp, X, to compute voxel i + 1's
+        //         terms), corrects i's terms if i - 1 is its neighbour, derives delta_i and
+        //         publishes it (B); meanwhile the view warps prepare voxel i + 1 (A record, w A);
+        //         after B they scatter voxel i into their own views.
         float amount = 0.f;
-        const int npair = (nactv + 1) >> 1;
+        const uint32_t g0 = gseq;  // step buffers alternate with the running voxel number
         if (is_view) {
             const int tp = tpm;
             constexpr int CW = U8 ? 1 : 4;  // record words per view
-            // Per-pair state of a view thread for its VPT views: band offsets of a and b (packed
-            // bytes), smem addresses of their first rows, the dequantised A of a, of b, and of a
-            // on b's channels, w*A of both, and this lane's part of H = sum w A_b A_a.
-            struct PairState {
-                uint32_t oa, ob;
-                int pa[VPT], pb[VPT];        // float index of (row offset, view) in sb
-                float2 fa[VPT][2], fb[VPT][2], fab[VPT][2];
-                float2 wa[VPT][2], wb[VPT][2];
-                float hh;
-                int sj;                      // ring stage of the pair's first voxel
+            // per-voxel state of a view thread for its VPT views: the band offsets (packed bytes),
+            // the float index of each view's first row in sb, the dequantised A and w*A
+            struct VoxState {
+                int p[VPT];
+                float2 f[VPT][2], wf[VPT][2];
+                int sj;  // ring stage of the voxel's record
             };
             auto avals = [&](const uint32_t (&c)[CW], float2 (&f)[2]) {
                 if (U8) {
@@ -702,221 +642,147 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                     f[1] = make_float2(__uint_as_float(c[CW > 2 ? 2 : 0]), __uint_as_float(c[CW > 3 ? 3 : 0]));
                 }
             };
-            auto off_of = [&](uint32_t packed, int t) { return (int)((packed >> (8 * t)) & 255u); };
-            // voxels j, j + 1 of the visiting order -> ps.  A pair without a second voxel (the last
-            // step of an odd visit, hb = false) gets a dummy b with zero A on a's channels: its
-            // theta1 and H vanish, its delta is 0 and its scatter rewrites a's entries with the
-            // same values.
-            auto prep = [&](int j, bool hb, PairState& ps) {
-                cp_async_wait<R - 2>();      // this thread's copies of voxels j, j + 1 have landed
+            // voxel j of the visiting order -> vs (e-independent: record, offsets, w A)
+            auto prep = [&](VoxState& vs) {
+                cp_async_wait<R - 1>();      // this thread's copy of the voxel's record has landed
                 if (VPT != 4) __syncwarp();  // offset words copied by another lane of the warp
-                const int s1 = ps.sj + 1 == R ? 0 : ps.sj + 1;
-                uint32_t ca[VPT][CW], cb[VPT][CW];
-                load_words<VPT, CW>(astage + ps.sj * L.stage_bytes, L.off_in_stage, tp, ca, ps.oa);
-                load_words<VPT, CW>(astage + s1 * L.stage_bytes, L.off_in_stage, tp, cb, ps.ob);
-                ps.ob = hb ? ps.ob : ps.oa;
-                float2 h2[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+                uint32_t c[VPT][CW], ow;
+                load_words<VPT, CW>(astage + vs.sj * L.stage_bytes, L.off_in_stage, tp, c, ow);
 #pragma unroll
                 for (int t = 0; t < VPT; ++t) {
-#pragma unroll
-                    for (int c = 0; c < CW; ++c) cb[t][c] = hb ? cb[t][c] : 0u;
-                    avals(ca[t], ps.fa[t]);
-                    avals(cb[t], ps.fb[t]);
-                    const int oa = off_of(ps.oa, t), ob = off_of(ps.ob, t);
-                    shifted<U8>(ca[t][0], ps.fa[t], ob - oa, ps.fab[t]);  // A_a on b's channels
-                    ps.pa[t] = oa * RS + kv[t];
-                    ps.pb[t] = ob * RS + kv[t];
-                    const float* pw = sb + VS + ps.pa[t];
-                    const float* qw = sb + VS + ps.pb[t];
-                    ps.wa[t][0] = __fmul2_rn(make_float2(pw[0], pw[RS]), ps.fa[t][0]);
-                    ps.wa[t][1] = __fmul2_rn(make_float2(pw[2 * RS], pw[3 * RS]), ps.fa[t][1]);
-                    ps.wb[t][0] = __fmul2_rn(make_float2(qw[0], qw[RS]), ps.fb[t][0]);
-                    ps.wb[t][1] = __fmul2_rn(make_float2(qw[2 * RS], qw[3 * RS]), ps.fb[t][1]);
-                    h2[t & 1] = __ffma2_rn(ps.wb[t][0], ps.fab[t][0], h2[t & 1]);
-                    h2[t & 1] = __ffma2_rn(ps.wb[t][1], ps.fab[t][1], h2[t & 1]);
+                    avals(c[t], vs.f[t]);
+                    vs.p[t] = (int)((ow >> (8 * t)) & 255u) * RS + kv[t];
+                    const float* pw = sb + VS + vs.p[t];
+                    vs.wf[t][0] = __fmul2_rn(make_float2(pw[0], pw[RS]), vs.f[t][0]);
+                    vs.wf[t][1] = __fmul2_rn(make_float2(pw[2 * RS], pw[3 * RS]), vs.f[t][1]);
                 }
-                const float2 hs = __fadd2_rn(h2[0], h2[1]);
-                ps.hh = hs.x + hs.y;
             };
-            // refill two ring stages with the records R voxels ahead (one commit group per voxel,
-            // empty past the visit's end, keeps the wait counts fixed)
+            // refill the stage voxel j's record used with the record R voxels ahead (one commit
+            // group per voxel, empty past the visit's end, keeps the wait counts fixed)
             auto refill = [&](int j, int sj) {
                 if (VPT != 4) __syncwarp();  // lanes read offset words another lane refills
-                const int s1 = sj + 1 == R ? 0 : sj + 1;
                 copy_record_to(j + R, sj, j + R < nactv ? list[j + R] : 0);
-                copy_record_to(j + 1 + R, s1, j + 1 + R < nactv ? list[j + 1 + R] : 0);
             };
-            // one voxel pair: theta1 partials from e -> barrier A -> the next pair's state ->
-            // barrier B (deltas) -> scatter
-            auto pair_step = [&](int idx, PairState& cur, PairState& nxt) {
-                const uint32_t pn = pseq + (uint32_t)(idx >> 1);  // running pair number
-                float2 ea[VPT][2], eb[VPT][2];
+            auto step = [&](int idx, VoxState& cur, VoxState& nxt) {
+                const uint32_t sn = (g0 + (uint32_t)idx) & 1u;
+                float2 ev[VPT][2];
                 {
                     float2 acc[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-                    float2 accb[2] = {acc[0], acc[0]};
 #pragma unroll
                     for (int t = 0; t < VPT; ++t) {
-                        const float* pe = sb + cur.pa[t];
-                        const float* qe = sb + cur.pb[t];
-                        ea[t][0] = make_float2(pe[0], pe[RS]);
-                        ea[t][1] = make_float2(pe[2 * RS], pe[3 * RS]);
-                        eb[t][0] = make_float2(qe[0], qe[RS]);
-                        eb[t][1] = make_float2(qe[2 * RS], qe[3 * RS]);
-                        acc[t & 1] = __ffma2_rn(cur.wa[t][0], ea[t][0], acc[t & 1]);
-                        acc[t & 1] = __ffma2_rn(cur.wa[t][1], ea[t][1], acc[t & 1]);
-                        accb[t & 1] = __ffma2_rn(cur.wb[t][0], eb[t][0], accb[t & 1]);
-                        accb[t & 1] = __ffma2_rn(cur.wb[t][1], eb[t][1], accb[t & 1]);
+                        const float* pe = sb + cur.p[t];
+                        ev[t][0] = make_float2(pe[0], pe[RS]);
+                        ev[t][1] = make_float2(pe[2 * RS], pe[3 * RS]);
+                        acc[t & 1] = __ffma2_rn(cur.wf[t][0], ev[t][0], acc[t & 1]);
+                        acc[t & 1] = __ffma2_rn(cur.wf[t][1], ev[t][1], acc[t & 1]);
                     }
-                    const float2 ac = __fadd2_rn(acc[0], acc[1]), acb = __fadd2_rn(accb[0], accb[1]);
-                    float2 gab = make_float2(ac.x + ac.y, acb.x + acb.y);
-                    float hh = cur.hh;
+                    const float2 ac = __fadd2_rn(acc[0], acc[1]);
+                    float g = ac.x + ac.y;
 #pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) {
-                        const float2 r = make_float2(__shfl_xor_sync(kFull, gab.x, o), __shfl_xor_sync(kFull, gab.y, o));
-                        hh += __shfl_xor_sync(kFull, hh, o);
-                        gab = __fadd2_rn(gab, r);
-                    }
-                    if (lane == 0) {
-                        float* rs = red + (pn & 1) * 3 * kNSL + vw;
-                        rs[0] = gab.x;
-                        rs[kNSL] = gab.y;
-                        rs[2 * kNSL] = hh;
-                    }
+                    for (int o = 16; o > 0; o >>= 1) g += __shfl_xor_sync(kFull, g, o);
+                    if (lane == 0) red[sn * kNSL + vw] = g;
                 }
                 bar_arrive(kBarA, nab);
-                // meanwhile: the next pair's e-independent state, then refill its freed stages
-                nxt.sj = cur.sj + 2 >= R ? cur.sj + 2 - R : cur.sj + 2;
-                if (idx + 2 < nactv) prep(idx + 2, idx + 3 < nactv, nxt);
-                refill(idx + 2, nxt.sj);
+                // meanwhile: the next voxel's e-independent state, then refill its stage
+                nxt.sj = cur.sj + 1 == R ? 0 : cur.sj + 1;
+                if (idx + 1 < nactv) prep(nxt);
+                refill(idx + 1, nxt.sj);
                 bar_sync(kBarB, nb2);
-                // Alg1:9-11 for both voxels on this thread's views: a's channels with a's update,
-                // then b's channels with both updates -- b's write carries the full value on the
-                // entries the two voxels share
-                const float sda = dslot[(pn & 1) * 2], sdb = dslot[(pn & 1) * 2 + 1];
-                if (sda != 0.f || sdb != 0.f) {
-                    const float2 nda = make_float2(-sda, -sda), ndb = make_float2(-sdb, -sdb);
+                // Alg1:9-11 on this thread's views
+                const float sd = dslot[sn];
+                if (sd != 0.f) {
+                    const float2 nd = make_float2(-sd, -sd);
 #pragma unroll
                     for (int t = 0; t < VPT; ++t) {
-                        float* pe = sb + cur.pa[t];
-                        float* qe = sb + cur.pb[t];
-                        const float2 a0 = __ffma2_rn(cur.fa[t][0], nda, ea[t][0]);
-                        const float2 a1 = __ffma2_rn(cur.fa[t][1], nda, ea[t][1]);
-                        const float2 b0 = __ffma2_rn(cur.fb[t][0], ndb, __ffma2_rn(cur.fab[t][0], nda, eb[t][0]));
-                        const float2 b1 = __ffma2_rn(cur.fb[t][1], ndb, __ffma2_rn(cur.fab[t][1], nda, eb[t][1]));
+                        float* pe = sb + cur.p[t];
+                        const float2 a0 = __ffma2_rn(cur.f[t][0], nd, ev[t][0]);
+                        const float2 a1 = __ffma2_rn(cur.f[t][1], nd, ev[t][1]);
                         pe[0] = a0.x;
                         pe[RS] = a0.y;
                         pe[2 * RS] = a1.x;
                         pe[3 * RS] = a1.y;
-                        qe[0] = b0.x;
-                        qe[RS] = b0.y;
-                        qe[2 * RS] = b1.x;
-                        qe[3 * RS] = b1.y;
                     }
                 }
             };
             // the first R records (the ring region held the pack's staging tiles until the barrier)
             for (int i = 0; i < R; ++i) copy_record_to(i, (sbase + i) % R, i < nactv ? list[i] : 0);
-            PairState st0, st1;
+            VoxState st0, st1;
             st0.sj = sbase;
-            prep(0, 1 < nactv, st0);
+            prep(st0);
             refill(0, sbase);
-            for (int idx = 0; idx < nactv; idx += 4) {
-                pair_step(idx, st0, st1);
-                if (idx + 2 < nactv) pair_step(idx + 2, st1, st0);
+            for (int idx = 0; idx < nactv; idx += 2) {
+                step(idx, st0, st1);
+                if (idx + 1 < nactv) step(idx + 1, st1, st0);
             }
         } else if (is_delta) {
-            // ---- delta warp: per pair wait for the partial sums and the surrogate terms (A),
-            //      derive both deltas (every lane, identical inputs), publish them (B), write the
-            //      new values into the x tile (X, releases the prior warp)
-            for (int p = 0; p < npair; ++p) {
-                const int idx = 2 * p;
-                const uint32_t pn = pseq + (uint32_t)p;
-                const bool hasb = idx + 1 < nactv;
+            // ---- delta warp (every lane computes the same values; lane 0 publishes)
+            float u_prev = 0.f, v_prev = 0.f;
+            for (int idx = 0; idx < nactv; ++idx) {
+                const uint32_t sn = (g0 + (uint32_t)idx) & 1u;
                 bar_sync(kBarA, nab);
-                const float* rb = red + (pn & 1) * 3 * kNSL;  // nvw <= kNSL partials, rest 0
-                float sa = 0.f, sbs = 0.f, sh = 0.f;
-#pragma unroll
-                for (int i = 0; i < kNSL; ++i) {  // fixed order: every run gets the same bits
-                    sa += rb[i];
-                    sbs += rb[kNSL + i];
-                    sh += rb[2 * kNSL + i];
-                }
-                const PriPair pp = pri[pn & 1];
-                const float scale_a = vscale[idx];
-                float ua = pp.va;
-                const float theta1a = -scale_a * sa;  // Alg1:5
-                const float theta2a = vth2[idx];      // Alg1:6 (precomputed)
-                {
-                    const float num = theta2a * pp.va - theta1a + 2.f * pp.sxa;
-                    const float den = theta2a + 2.f * pp.sa;
-                    if (den > 0.f) ua = __fdividef(num, den);
-                    if (P.pc.positivity) ua = fmaxf(ua, 0.f);
-                }
-                const float da = ua - pp.va;  // Alg1:7-8
-                float ub = pp.vb, db = 0.f, scale_b = 0.f, theta1b = 0.f, theta2b = 0.f;
-                if (hasb) {
-                    scale_b = vscale[idx + 1];
-                    // e after a's update: sum w A_b e' = s_b (S_b - s_a delta_a H)
-                    theta1b = -scale_b * fmaf(-scale_a * da, sh, sbs);
-                    theta2b = vth2[idx + 1];
-                    float psb = pp.sb, psx = pp.sxb;
-                    if (pp.bab != 0.f) {  // a is b's neighbour: its term with a's new value
-                        const float bn = pp.bab * phi_f(P.pc, pp.vb - ua);
-                        psb += bn - pp.btab;
-                        psx += bn * ua - pp.btab * pp.va;
-                    }
-                    const float num = theta2b * pp.vb - theta1b + 2.f * psx;
-                    const float den = theta2b + 2.f * psb;
-                    if (den > 0.f) ub = __fdividef(num, den);
-                    if (P.pc.positivity) ub = fmaxf(ub, 0.f);
-                    db = ub - pp.vb;
-                }
-                if (lane == 0) {
-                    dslot[(pn & 1) * 2] = scale_a * da;
-                    dslot[(pn & 1) * 2 + 1] = scale_b * db;
-                }
-                bar_arrive(kBarB, nb2);
-                if (lane == 0) {
-                    const int ta = tof[idx];
-                    xt[cslot + (ta >> 8) * TW + (ta & 255)] = ua;
-                    if (hasb) {
-                        const int tbv = tof[idx + 1];
-                        xt[cslot + (tbv >> 8) * TW + (tbv & 255)] = ub;
-                    }
+                if (idx > 0 && lane == 0) {  // voxel i - 1's new value, deferred until the prior
+                    const int tu = tof[idx - 1];  // warp has computed voxel i's terms with the old one
+                    xt[cslot + (tu >> 8) * TW + (tu & 255)] = u_prev;
                 }
                 bar_arrive(kBarX, 64);
+                const float* rb = red + sn * kNSL;  // nvw <= kNSL partials, rest 0
+                float S = 0.f;
+#pragma unroll
+                for (int i = 0; i < kNSL; ++i) S += rb[i];  // fixed order: every run gets the same bits
+                const PriTerm pp = pri[sn];
+                float ps = pp.s, psx = pp.sx;
+                if (pp.bwu != 0.f) {  // voxel i - 1 is a neighbour: its term at its new value
+                    const float bn = pp.bwu * phi_f(P.pc, pp.v - u_prev);
+                    ps += bn - pp.btu;
+                    psx += bn * u_prev - pp.btu * v_prev;
+                }
+                const float scale = vscale[idx];
+                const float theta1 = -scale * S;  // Alg1:5
+                const float theta2 = vth2[idx];   // Alg1:6 (precomputed)
+                float u = pp.v;
+                {
+                    const float num = theta2 * pp.v - theta1 + 2.f * psx;
+                    const float den = theta2 + 2.f * ps;
+                    if (den > 0.f) u = __fdividef(num, den);
+                    if (P.pc.positivity) u = fmaxf(u, 0.f);
+                }
+                const float d = u - pp.v;  // Alg1:7-8
+                if (lane == 0) dslot[sn] = scale * d;
+                bar_arrive(kBarB, nb2);
+                u_prev = u;
+                v_prev = pp.v;
                 if (lane == 0) {
-                    amount += fabsf(da) + fabsf(db);
+                    amount += fabsf(d);
                     if (P.dump) {
-                        // test hook (mbir_set_update_dump): the pair's (voxel, theta1, theta2,
-                        // delta) exactly as the delta chain used them, a then b
-                        const unsigned long long slot = atomicAdd(P.dump_count, hasb ? 2ull : 1ull);
-                        for (int u = 0; u < (hasb ? 2 : 1); ++u) {
-                            const int tv = tof[idx + u];
-                            const uint32_t vox = (uint32_t)(((size_t)z * P.ny + gy0 + (tv >> 8)) * P.nx + gx0 + (tv & 255));
-                            if (slot + u < (unsigned long long)P.dump_cap)
-                                *(float4*)(P.dump + 4 * (slot + u)) = make_float4(
-                                    __uint_as_float(vox), u ? theta1b : theta1a, u ? theta2b : theta2a, u ? db : da);
-                        }
+                        // test hook (mbir_set_update_dump): the update's (voxel, theta1, theta2,
+                        // delta) exactly as the delta chain used them
+                        const unsigned long long slot = atomicAdd(P.dump_count, 1ull);
+                        const int tv = tof[idx];
+                        const uint32_t vox = (uint32_t)(((size_t)z * P.ny + gy0 + (tv >> 8)) * P.nx + gx0 + (tv & 255));
+                        if (slot < (unsigned long long)P.dump_cap)
+                            *(float4*)(P.dump + 4 * slot) = make_float4(__uint_as_float(vox), theta1, theta2, d);
                     }
                 }
             }
+            if (lane == 0) {  // the last voxel's new value
+                const int tu = tof[nactv - 1];
+                xt[cslot + (tu >> 8) * TW + (tu & 255)] = u_prev;
+            }
+            __syncwarp();
         } else if (is_prior) {
-            // ---- prior warp: the surrogate terms of pair p + 1 once pair p's new values are in
-            //      the x tile (X); its own arrival on A completes the pair's inputs
-            bar_arrive(kBarA, nab);  // pair 0's terms were computed in step 3
-            for (int p = 0; p < npair; ++p) {
+            // ---- prior warp: voxel i + 1's terms once voxel i - 1's new value is in the tile (X);
+            //      its arrival on A completes voxel i + 1's inputs
+            bar_arrive(kBarA, nab);  // voxel 0's terms were computed during the pack
+            for (int idx = 0; idx < nactv; ++idx) {
                 bar_sync(kBarX, 64);
-                if (p + 1 < npair) {
-                    prior_pair(tof, 2 * (p + 1), nactv, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
-                               pri + ((pseq + (uint32_t)p + 1) & 1));
+                if (idx + 1 < nactv) {
+                    prior_one(tof, idx + 1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + ((g0 + (uint32_t)idx + 1) & 1));
                     __syncwarp();
                     bar_arrive(kBarA, nab);
                 }
             }
         }
         gseq += nactv;
-        pseq += (uint32_t)npair;
         if (PROF && threadIdx.x == 0) tp3 = clock64();
         __syncthreads();
 
