@@ -183,10 +183,11 @@ __host__ __device__ constexpr int tile_warps(int va) { return va / (32 * kTileW)
 __host__ __device__ constexpr int max_threads(int vpt) { return vpt == 2 ? 448 : vpt == 3 ? 320 : 256; }
 
 // named barriers of the pair protocol (0 is __syncthreads)
-constexpr int kBarA = 1;  // view warps' partials + the prior warp's terms of a pair are ready
+constexpr int kBarA = 1;  // the view warps' theta1 partials of a voxel are ready
 constexpr int kBarB = 2;  // the delta warp has published the pair's deltas
 constexpr int kBarX = 3;  // the delta warp has written the pair's new values into the x tile
 constexpr int kBarP = 4;  // task preparation steps (delta + prior warps)
+constexpr int kBarT = 5;  // the prior warp's surrogate terms of a voxel are ready
 
 // A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
 __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, int nnb, int VA, bool u8,
@@ -288,6 +289,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     const int VA = P.A.VA;                 // record positions / SVB columns in use
     constexpr int VS = svb_cols(VPT);      // SVB row length (compile-time: row offsets are immediates)
     constexpr int RS = 2 * VS;             // float stride between consecutive e (or w) rows
+    constexpr bool kNSL8 = VPT != 2;       // at most 8 view warps: only the first 8 slots are used
     const SmemLayout& L = P.lay;
     float* sb = (float*)(smem + L.sb_e);   // e row r at sb + r RS, w row r at sb + r RS + VS
     int* flags = (int*)(smem + L.flags);
@@ -302,7 +304,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
     const int ntile = (NNB == 26 ? 3 : 1) * TW * TW;  // x tile entries
     const size_t plane = (size_t)P.nx * P.ny;
-    const int nab = (nvw + 2) * 32;      // barrier A: view warps + delta warp + prior warp
+    const int nab = (nvw + 1) * 32;      // barrier A: view warps + the delta warp
     const int nb2 = (nvw + 1) * 32;      // barrier B: view warps + the delta warp
 
     for (int i = threadIdx.x; i < 2 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
@@ -715,20 +717,20 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 if (idx + 1 < nactv) step(idx + 1, st1, st0);
             }
         } else if (is_delta) {
-            // ---- delta warp (every lane computes the same values; lane 0 publishes)
+            // ---- delta warp (every lane computes the same values; lane 0 publishes).  The prior
+            //      side of the update (voxel i - 1's neighbour correction, the numerator's and the
+            //      denominator's prior terms, the reciprocal) is done as soon as the prior warp's
+            //      terms are in (T), before the view warps' partial sums (A): after A only
+            //      theta1, one FMA and the clip remain on the chain
             float u_prev = 0.f, v_prev = 0.f;
             for (int idx = 0; idx < nactv; ++idx) {
                 const uint32_t sn = (g0 + (uint32_t)idx) & 1u;
-                bar_sync(kBarA, nab);
+                bar_sync(kBarT, 64);
                 if (idx > 0 && lane == 0) {  // voxel i - 1's new value, deferred until the prior
                     const int tu = tof[idx - 1];  // warp has computed voxel i's terms with the old one
                     xt[cslot + (tu >> 8) * TW + (tu & 255)] = u_prev;
                 }
                 bar_arrive(kBarX, 64);
-                const float* rb = red + sn * kNSL;  // nvw <= kNSL partials, rest 0
-                float S = 0.f;
-#pragma unroll
-                for (int i = 0; i < kNSL; ++i) S += rb[i];  // fixed order: every run gets the same bits
                 const PriTerm pp = pri[sn];
                 float ps = pp.s, psx = pp.sx;
                 if (pp.bwu != 0.f) {  // voxel i - 1 is a neighbour: its term at its new value
@@ -737,15 +739,30 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                     psx += bn * u_prev - pp.btu * v_prev;
                 }
                 const float scale = vscale[idx];
-                const float theta1 = -scale * S;  // Alg1:5
-                const float theta2 = vth2[idx];   // Alg1:6 (precomputed)
-                float u = pp.v;
-                {
-                    const float num = theta2 * pp.v - theta1 + 2.f * psx;
-                    const float den = theta2 + 2.f * ps;
-                    if (den > 0.f) u = __fdividef(num, den);
-                    if (P.pc.positivity) u = fmaxf(u, 0.f);
+                const float theta2 = vth2[idx];  // Alg1:6 (precomputed)
+                const float den = theta2 + 2.f * ps;
+                const float c1 = theta2 * pp.v + 2.f * psx;  // numerator without -theta1
+                const float rden = den > 0.f ? __fdividef(1.f, den) : 0.f;
+                bar_sync(kBarA, nab);
+                const float4 r0 = *(const float4*)(red + sn * kNSL), r1 = *(const float4*)(red + sn * kNSL + 4);
+                float S;
+                if (kNSL8) {  // <= 8 view warps: slots 8.. are zero; fixed tree order
+                    const float2 q = __fadd2_rn(__fadd2_rn(make_float2(r0.x, r0.y), make_float2(r0.z, r0.w)),
+                                                __fadd2_rn(make_float2(r1.x, r1.y), make_float2(r1.z, r1.w)));
+                    S = q.x + q.y;
+                } else {
+                    const float4 r2 = *(const float4*)(red + sn * kNSL + 8), r3 = *(const float4*)(red + sn * kNSL + 12);
+                    const float2 q = __fadd2_rn(
+                        __fadd2_rn(__fadd2_rn(make_float2(r0.x, r0.y), make_float2(r0.z, r0.w)),
+                                   __fadd2_rn(make_float2(r1.x, r1.y), make_float2(r1.z, r1.w))),
+                        __fadd2_rn(__fadd2_rn(make_float2(r2.x, r2.y), make_float2(r2.z, r2.w)),
+                                   __fadd2_rn(make_float2(r3.x, r3.y), make_float2(r3.z, r3.w))));
+                    S = q.x + q.y;
                 }
+                const float theta1 = -scale * S;  // Alg1:5
+                float u = pp.v;
+                if (den > 0.f) u = (c1 - theta1) * rden;
+                if (P.pc.positivity) u = fmaxf(u, 0.f);
                 const float d = u - pp.v;  // Alg1:7-8
                 if (lane == 0) dslot[sn] = scale * d;
                 bar_arrive(kBarB, nb2);
@@ -772,13 +789,13 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         } else if (is_prior) {
             // ---- prior warp: voxel i + 1's terms once voxel i - 1's new value is in the tile (X);
             //      its arrival on A completes voxel i + 1's inputs
-            bar_arrive(kBarA, nab);  // voxel 0's terms were computed during the pack
+            bar_arrive(kBarT, 64);  // voxel 0's terms were computed during the pack
             for (int idx = 0; idx < nactv; ++idx) {
                 bar_sync(kBarX, 64);
                 if (idx + 1 < nactv) {
                     prior_one(tof, idx + 1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + ((g0 + (uint32_t)idx + 1) & 1));
                     __syncwarp();
-                    bar_arrive(kBarA, nab);
+                    bar_arrive(kBarT, 64);
                 }
             }
         }
