@@ -82,9 +82,9 @@ typedef struct mbir_options {
     double sv_fraction;    /* fraction of SVs per iteration >= 2, default 0.25  */
     int batch_svs;         /* BATCH_SIZE: SVs per slice per launch (Alg3:25); 0 = auto: a whole
                               checkerboard colour group per launch when the phase spans enough
-                              slices that at most cap = max(8, 2.5 sqrt(#SVs / 4)) SVs of one
-                              slice run at once, else batches of cap SVs per slice (no threshold);
-                              default 0 (reading R22)                                    */
+                              slices that at most cap = max(4, N / 12) SVs of one slice (N =
+                              max(nx, ny)) run at once, else batches of cap SVs per slice (no
+                              threshold); default 0 (reading R22)                       */
     int batch_threshold;   /* Alg3:26-27: drop a group's remainder smaller than this; -1 =
                               batch_svs/4; ignored when batch_svs == 0                   */
     int zero_skip;         /* P:115, default 1 (never in iteration 1; reading R9)               */

@@ -346,15 +346,14 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         // ---- flat task lists + batch ranges per (z-parity, colour) phase (Alg3:24-27)
         const bool det = h->o.deterministic != 0;
         // batch_svs = 0 (auto): a whole colour group per launch, unless the phase has so few slices
-        // that more than kAutoBatch SVs of one slice would run at once -- then batches of
-        // kAutoBatch SVs per slice, each launch seeing the previous one's write-backs.  Same-colour
-        // SVs updated concurrently fit the same residual along shared rays; with ~148 of them in
-        // one 2-D slice the first sweeps from x0 = 0 overshoot, clip whole SVs to 0 and zero-skip
-        // then freezes them (reading R22).
-        // A ray crosses ~sqrt(G) SVs of a colour group of G, so with C of them in flight per slice
-        // it meets ~C / sqrt(G) concurrently updated SVs; the cap keeps that near kAutoRayLoad.
+        // that more than `cap` SVs of one slice would run at once -- then batches of `cap` SVs per
+        // slice, each launch seeing the previous one's write-backs.  Same-colour SVs updated
+        // concurrently fit the same residual along shared rays, and too many of them make
+        // asynchronous SV-ICD oscillate or diverge (reading R22: on the paper's 512^2
+        // geometry 42 per slice converge, 84 diverge; on 256^2 side-5 cases 39 oscillate, 20
+        // converge).  cap = N / 12 SVs per slice of width N pixels, whatever the SV side.
         const int slices_in_phase = std::max(1, h->g.nz_local / parities);
-        const int ray_cap = std::max(8, (int)(kAutoRayLoad * std::sqrt(0.25 * h->nsv)));
+        const int ray_cap = std::max(kAutoCapMin, (std::max(h->g.nx, h->g.ny) + kAutoCapDiv / 2) / kAutoCapDiv);
         const bool auto_batch = !det && h->o.batch_svs == 0 && target_ctas > ray_cap * slices_in_phase;
         const int B = auto_batch ? ray_cap : (det || h->o.batch_svs <= 0) ? h->max_group : h->o.batch_svs;
         const int thr = (det || h->o.batch_svs <= 0) ? 0 : (h->o.batch_threshold >= 0 ? h->o.batch_threshold : B / 4);

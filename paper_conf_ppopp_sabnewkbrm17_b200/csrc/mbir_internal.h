@@ -16,7 +16,8 @@ constexpr int kK = 4;             // max channels per (voxel, view) (reading R5;
 constexpr int kMaxNbr = 26;       // 3-D neighbourhood (reading R2)
 constexpr int kMaxSvbRows = 32;   // SV-buffer rows held by one 32-lane transpose tile
 constexpr int kMaxPhaseSlices = 1024;  // slices of one (z-parity, colour) phase (sched.cu k_flatten)
-constexpr double kAutoRayLoad = 1.5;  // batch_svs = 0: concurrently updated SVs one ray meets (R22)
+constexpr int kAutoCapDiv = 12;  // batch_svs = 0: at most N / 12 concurrently updated SVs per slice (R22)
+constexpr int kAutoCapMin = 4;
 
 // ---- prior constants, per handle: passed by value in the kernels' parameter blocks ----
 struct PriorConst {

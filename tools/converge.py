@@ -30,12 +30,20 @@ def main():
     ap.add_argument("--target", type=float, default=10.0)
     ap.add_argument("--sv-side", type=int, default=0)
     ap.add_argument("--det", type=int, default=0)
+    ap.add_argument("--sweep", type=int, default=-1, help="a config-5 case index (golden from goldens/sweep/)")
     a = ap.parse_args()
-    cfg = CONFIGS[a.config]
-    gpath = a.golden or os.path.join(ROOT, "tests", "golden", f"golden_{a.config}.npz")
+    cid = 0
+    if a.sweep >= 0:
+        from synth import sweep_configs
+        cfg, cid = sweep_configs()[a.sweep]
+        a.config = cfg.name
+        gpath = os.path.join(ROOT, "goldens", "sweep", f"{cfg.name}.npz")
+    else:
+        cfg = CONFIGS[a.config]
+        gpath = a.golden or os.path.join(ROOT, "tests", "golden", f"golden_{a.config}.npz")
     gz = np.load(gpath)
     meta = json.loads(str(gz["meta"]))
-    y, w = make_sinogram_torch(cfg, 0, "cuda")
+    y, w = make_sinogram_torch(cfg, cid, "cuda")
     if sino_hash(y.cpu().numpy(), w.cpu().numpy()) != meta["sino_sha"]:
         raise SystemExit("golden was computed for a different sinogram")
     golden = torch.from_numpy(gz["x"]).cuda()
@@ -66,7 +74,7 @@ def main():
                     hit = {"time_s": t, "equits": eq, "iterations": it + 1}
         print(json.dumps({"config": a.config, "init": a.init, "batch_svs": a.batch_svs, "det": a.det,
                           "zero_skip": a.zero_skip, "period": a.period, "to_target": hit,
-                          "target_hu": a.target, "golden": {k: meta[k] for k in ("equits", "selfconv_hu_last20", "init")},
+                          "target_hu": a.target, "golden": {k: meta.get(k) for k in ("equits", "golden_equits", "selfconv_hu_last20", "init")},
                           "final_hu": hist[-1][2], "curve": hist}))
 
 
