@@ -516,3 +516,17 @@ def test_sweep_configs_grid():
         assert c.nchannels == 2 * c.n and abs(c.dchannel - c.dxy / 2) < 1e-12
         assert c.sv_side in (5, 7, 9) and c.nviews in (90, 180, 360, 720) and c.lambda0 in (1e3, 1e4, 1e5)
     assert {c.phantom for c, _ in a} == {"shepp_logan", "baggage"}
+
+
+def test_synthetic_generators_agree():
+    """The bench's generator (device projections, synth.make_sinogram_torch) and the oracle-side
+    one (numpy, synth.make_case) produce the same y and w bit for bit, for any slab of a volume:
+    the oracle goldens (tools/make_golden.py) are computed for exactly the bench's inputs."""
+    torch = pytest.importorskip("torch")
+    from synth import WorkloadConfig, make_case, make_sinogram_torch
+    for cfg, cid in ((WorkloadConfig("t3d", 32, 4, 30, 48, 7, 26, 0.003), 0),
+                     (WorkloadConfig("tbag", 32, 3, 24, 64, 5, 8, 0.003, phantom="baggage", lambda0=1e3), 101)):
+        c = make_case(cfg, cid, with_truth=False)
+        y, w = make_sinogram_torch(cfg, cid, "cpu", 1, cfg.nz)
+        np.testing.assert_array_equal(y.numpy(), c.y[1:])
+        np.testing.assert_array_equal(w.numpy(), c.w[1:])
