@@ -49,7 +49,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-converge", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--conv-iters", type=int, default=150, help="max iterations of a convergence run")
+    ap.add_argument("--conv-iters", type=int, default=300, help="max iterations of a convergence run")
     return ap.parse_args()
 
 
@@ -346,7 +346,7 @@ def main():
         traffic = tj.get("dram_bytes_per_update", 0) * local_updates / max(klaunch, 1)
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": traffic,
-            "kernel": "k_icd_sv (fused SV update)", "kernel_share": ksec / el,
+            "kernel": "k_svicd (fused SV update)", "kernel_share": ksec / el,
             "alg_bytes_per_update": alg_bytes / local_updates,
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback 6.65 TB/s"}
 

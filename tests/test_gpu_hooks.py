@@ -1,7 +1,7 @@
 """GPU parity of the hot kernel's own arithmetic and of the device-side bookkeeping, through the
 C-ABI test hooks (VERDICT r1 "What's weak" 1-2):
 
-  - every update k_icd_sv executes (theta1, theta2, delta of Alg. 1, as its delta chain
+  - every update k_svicd executes (theta1, theta2, delta of Alg. 1, as its delta chain
     used them) against the oracle's orc_voxel_update at the same state (reading R20's 1e-5),
     in deterministic mode, replayed update by update;
   - the device RMSE-HU reduction against oracle.rmse_hu;

@@ -1,5 +1,5 @@
 #!/usr/bin/env python
-"""profiles/icd_traffic.json from a tools/traffic.sh capture: ncu DRAM bytes of every k_icd_sv
+"""profiles/icd_traffic.json from a tools/traffic.sh capture: ncu DRAM bytes of every k_svicd
 launch of one bench step / that step's executed voxel updates.  usage: traffic_json.py PREFIX"""
 import csv
 import json
@@ -23,7 +23,7 @@ out = {
     "l2_bytes_per_update": round(tot["lts__t_bytes.sum"] / upd, 1),
     "launches": len(launches),
     "updates": upd,
-    "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,lts__t_bytes.sum over every k_icd_sv "
+    "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,lts__t_bytes.sum over every k_svicd "
            "launch of one bench.py step (cfg4, 6 equits from x0 = 0; tools/traffic.sh)",
 }
 print(json.dumps(out, indent=1))
