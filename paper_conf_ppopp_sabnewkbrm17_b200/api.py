@@ -72,7 +72,7 @@ class Options:
     quantize_A: int = 1
     seed: int = 3000
     deterministic: int = 0
-    cluster: int = 0  # update-kernel CTAs per SV task: 0 (auto) or 1
+    cluster: int = 0  # update-kernel CTAs per SV task: 0 (auto) = 1, or 2 (a cluster splits the views)
     zero_skip_period: int = 4  # every n-th iteration without zero-skip (reading R9); 0 = never
 
     def c(self) -> L.mbir_options:

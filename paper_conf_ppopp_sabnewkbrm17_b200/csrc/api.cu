@@ -271,7 +271,7 @@ int timed_icd(mbir_handle* h, const IcdParams& p, int nnb, bool q, int gx, int g
     }
     CK(cudaEventRecord(h->kev[2 * h->kev_used], h->st));
     (void)gy;
-    CK(launch_svicd(p, h->vpt, nnb, q, gx, h->st));
+    CK(launch_svicd(p, h->vpt, nnb, q, h->cl, gx, h->st));
     CK(cudaEventRecord(h->kev[2 * h->kev_used + 1], h->st));
     h->kev_used++;
     return MBIR_OK;
@@ -297,7 +297,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
     const bool q = h->o.quantize_A != 0;
     const int nnb = h->pr.neighborhood;
     const int parities = (nnb == 26 && h->g.nz_total > 1) ? 2 : 1;
-    const int target_ctas = h->nsm * h->blocks_per_sm;
+    const int target_ctas = h->resident;  // persistent grid: every resident CTA (cluster)
     int64_t updates = 0, skipped = 0, visits = 0, empty = 0, iters = 0, launches = 0, klaunches = 0;
     int zero_iters = 0;  // consecutive iterations without an executed update
     double ksec = 0.0;
@@ -354,7 +354,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         // converge).  cap = N / 12 SVs per slice of width N pixels, whatever the SV side.
         const int slices_in_phase = std::max(1, h->g.nz_local / parities);
         const int ray_cap = std::max(kAutoCapMin, (std::max(h->g.nx, h->g.ny) + kAutoCapDiv / 2) / kAutoCapDiv);
-        const bool auto_batch = !det && h->o.batch_svs == 0 && target_ctas > ray_cap * slices_in_phase;
+        const bool auto_batch = !det && h->o.batch_svs == 0 && target_ctas / h->cl > ray_cap * slices_in_phase;
         const int B = auto_batch ? ray_cap : (det || h->o.batch_svs <= 0) ? h->max_group : h->o.batch_svs;
         const int thr = (det || h->o.batch_svs <= 0) ? 0 : (h->o.batch_threshold >= 0 ? h->o.batch_threshold : B / 4);
         const int nb = (h->max_group + B - 1) / B;
@@ -368,7 +368,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         const size_t cap = (size_t)h->g.nz_local * h->max_group;
         // deterministic: one CTA (or one cluster) walks the phase list in order (sequential ICD,
         // known order)
-        const int grid = det ? 1 : target_ctas;
+        const int grid = det ? h->cl : target_ctas;
         // iterations >= 2 without batching: the tasks whose whole tile is zero are flagged per
         // phase (sched.cu k_zero_flags) and skipped at task fetch by the update kernel
         const bool prefilter = p.zero_skip_active && nb == 1 && !det;
@@ -736,20 +736,23 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
     {
-        // the fused update kernel: nvw view warps + the delta warp + the prior warp, one CTA per SM
+        // the fused update kernel: nvw view warps + the delta warp + the prior warp per task; the
+        // task's CTA owns all views (cluster 1) or a 2-CTA cluster splits them (cluster 2: each
+        // CTA holds half the views' SV buffer and exchanges one partial sum per voxel through
+        // distributed shared memory -- two SMs per SV for few-SV (2-D) workloads)
         IcdParams p = make_params(h);
-        if (h->o.cluster < 0 || h->o.cluster > 1)
-            return (fail(h, MBIR_EINVAL, "cluster must be 0 (auto) or 1: one CTA per SV task"), bail(MBIR_EINVAL));
-        h->cl = 1;
-        h->threads = 32 * (h->nvw + 2);
-        h->smem = svicd_smem_bytes(p, h->vpt, P.neighborhood, quant);
+        if (h->o.cluster < 0 || h->o.cluster > 2)
+            return (fail(h, MBIR_EINVAL, "cluster must be 0 (auto), 1 or 2"), bail(MBIR_EINVAL));
+        h->cl = h->o.cluster == 2 ? 2 : 1;
+        if (h->cl == 2 && !(h->vpt == 4 && h->nvw % 2 == 0))
+            return (fail(h, MBIR_EINVAL, "cluster = 2 needs > 128 views in an even number of 128-view warps"), bail(MBIR_EINVAL));
+        h->threads = 32 * (h->nvw / h->cl + 2);
+        h->smem = svicd_smem_bytes(p, h->vpt, P.neighborhood, quant, h->cl);
         if (h->smem > (int)prop.sharedMemPerBlockOptin)
             return (fail(h, MBIR_EINVAL, "SV buffer (" + std::to_string(h->smem) + " B) exceeds shared memory: reduce sv_side"), bail(MBIR_EINVAL));
-        h->blocks_per_sm = std::max(1, std::min((int)(prop.sharedMemPerMultiprocessor / (h->smem + 1024)),
-                                                (int)(2048 / h->threads)));
-        h->resident = svicd_resident_ctas(p, h->vpt, P.neighborhood, quant);
+        h->resident = svicd_resident_ctas(p, h->vpt, P.neighborhood, quant, h->cl);
         if (h->resident <= 0) return (fail(h, MBIR_ECUDA, "update kernel does not fit on the device"), bail(MBIR_ECUDA));
-        h->blocks_per_sm = std::max(1, h->resident / h->nsm);
+        h->blocks_per_sm = std::max(1, (h->resident + h->nsm - 1) / h->nsm);
     }
 
     // ---- state buffers

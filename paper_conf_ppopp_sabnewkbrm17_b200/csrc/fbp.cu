@@ -52,11 +52,13 @@ __global__ void k_backproject(const float* __restrict__ q, const double2* __rest
     const int z = blockIdx.z;
     if (ix >= nx || iy >= ny) return;
     const double xc = (ix - 0.5 * (nx - 1)) * dxy, yc = (iy - 0.5 * (ny - 1)) * dxy;
+    const double inv_dc = 1.0 / dc;
     const float* qz = q + (size_t)z * V * M;
     float acc = 0.f;
     for (int k = 0; k < V; ++k) {
         const double2 c = cs[k];
-        const float u = (float)((xc * c.x + yc * c.y - t0) / dc) - 0.5f;  // channel-centre coordinate
+        // channel-centre coordinate (double FMAs, no per-sample division)
+        const float u = (float)(fma(xc, c.x, fma(yc, c.y, -t0)) * inv_dc) - 0.5f;
         const float fl = floorf(u);
         const int m = (int)fl;
         const float f = u - fl;

@@ -58,7 +58,7 @@ __host__ __device__ __forceinline__ int apos(int k, int vpt)
 // configuration and passed in the parameter block, so the kernel addresses them from the
 // constant bank instead of recomputing the layout in registers)
 struct SmemLayout {
-    int sb_e, sb_w, xt, list, flags, tof, red, pri, vscale, vth2, misc, astage, stage_bytes, rscale, rth2, rbs, rbw,
+    int sb_e, sb_w, xt, list, flags, tof, red, pri, vscale, vth2, misc, astage, stage_bytes, rscale, rth2, rbs, rbw, cx,
         off_in_stage, mbar, staging, binfo, total;
 };
 
@@ -114,12 +114,12 @@ struct SchedParams {
 cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, int side, int nsvx,
                             int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxoff,
                             cudaStream_t st);
-// the fused update kernel (svicd.cu): nvw view warps + the delta warp + the prior warp per CTA,
-// vpt = 4 (or 1 for <= 128 views) views per lane
-int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize);
-int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize);
+// the fused update kernel (svicd.cu): per CTA nvw / cl view warps + the delta warp + the prior
+// warp, vpt = 4 (or 1 for <= 128 views) views per lane; cl = 2: a 2-CTA cluster splits a task's views
+int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
+int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
 int svicd_scratch_floats(int vpt);  // per-CTA e_init scratch tile
-cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid, cudaStream_t st);
+cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int cl, int grid, cudaStream_t st);
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st);
 cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cudaStream_t st);
 cudaError_t launch_probe(const IcdParams& p, bool quantize, int nnb, const int64_t* vox, int n,

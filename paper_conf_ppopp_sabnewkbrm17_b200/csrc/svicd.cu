@@ -98,6 +98,55 @@ __device__ __forceinline__ void cp_async_wait()
 {
     asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
+// ---- thread-block cluster (CL = 2: the two CTAs of a cluster split a task's views) ----
+__device__ __forceinline__ uint32_t cluster_rank()
+{
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+// shared::cluster address of the same shared-memory location in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t peer_addr(const void* p, uint32_t rank)
+{
+    uint32_t a;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(smem_u32(p)), "r"(rank));
+    return a;
+}
+__device__ __forceinline__ void st_peer_f32(uint32_t a, float v)
+{
+    asm volatile("st.shared::cluster.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
+}
+__device__ __forceinline__ void st_peer_u32(uint32_t a, uint32_t v)
+{
+    asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+// arrive on the peer CTA's mbarrier; release at cluster scope orders this thread's earlier
+// st.shared::cluster writes before the arrival
+__device__ __forceinline__ void mbar_arrive_peer(uint32_t a)
+{
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(a) : "memory");
+}
+// wait for phase `parity` of a local mbarrier with acquire at cluster scope (sees the peer's
+// released writes)
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity)
+{
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAITC_%=:\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAITC_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all()
+{
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 // one 128-bit shared-memory load (kept vector: the staging row reads are conflict-free only as
 // LDS.128; split into scalar loads they would be 4-way bank conflicts)
 __device__ __forceinline__ float4 lds128(const float* p)
@@ -168,7 +217,7 @@ constexpr int kStg = 36;
 // rows of e and w interleaved, so e row r sits at float offset 2 r VS and w row r at (2 r + 1) VS:
 // a thread reaches all four channels of a voxel's record in both arrays with immediate offsets
 // from one address
-__host__ __device__ constexpr int svb_cols(int vpt) { return vpt == 1 ? 128 : 768; }
+__host__ __device__ constexpr int svb_cols(int vpt, int cl = 1) { return (vpt == 1 ? 128 : 768) / cl; }
 
 constexpr int kNSL = 16;  // partial-sum slots per quantity in the pair exchange (>= view warps)
 
@@ -191,14 +240,15 @@ constexpr int kBarT = 5;  // the prior warp's surrogate terms of a voxel are rea
 
 // A-record stage: U8: codes u32[VA] then offsets u8[VA]; fp32: float4[VA] then offsets u8[VA]
 __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, int nnb, int VA, bool u8,
-                                                   int nstage, int nvw, int vpt, int V)
+                                                   int nstage, int nvw, int vpt, int V, int cl = 1)
 {
+    VA /= cl;  // this CTA's record positions (and views)
     SmemLayout L;
     const int TW = side + 2;
     const int nzt = nnb == 26 ? 3 : 1;
     int o = 0;
-    L.sb_e = o;  o = align16(o + 2 * rows * svb_cols(vpt) * 4);  // e / w rows interleaved
-    L.sb_w = L.sb_e + svb_cols(vpt) * 4;
+    L.sb_e = o;  o = align16(o + 2 * rows * svb_cols(vpt, cl) * 4);  // e / w rows interleaved
+    L.sb_w = L.sb_e + svb_cols(vpt, cl) * 4;
     L.xt = o;    o = align16(o + 2 * nzt * TW * TW * 4);  // [2 tasks]: current / next
     L.list = o;  o = align16(o + 2 * S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
@@ -220,7 +270,8 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     L.rth2 = o;  o = align16(o + S2 * 4);       //   per-slot scales and theta2,
     L.rbs = o;   o = align16(o + V * 4);        //   band start and width per view
     L.rbw = o;   o = align16(o + V);
-    L.binfo = o; o = align16(o + 2 * VA * 4);  // band (row offset << 5 | width), 2 tasks
+    L.binfo = o; o = align16(o + 2 * VA * cl * 4);  // band (row offset << 5 | width) per view, 2 tasks
+    L.cx = o;    o = align16(o + 2 * 2 * 4 + 4 * 8);  // CL = 2: partial theta1 sums [2 steps][2 CTAs], mbarriers
     L.total = o;
     return L;
 }
@@ -277,17 +328,20 @@ __device__ __forceinline__ void load_words(const unsigned char* stg, int off_in_
 
 // The update kernel.  VPT views per lane (4, or 1 for <= 128 views), uint8 or fp32 A, 8 or 26
 // neighbours, R-voxel A-record ring; PROF adds per-phase cycle counters.
-template <int VPT, bool U8, int NNB, int R, bool PROF>
+template <int VPT, bool U8, int NNB, int R, int CL, bool PROF>
 __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int nvw = P.nvw;                 // view warps
+    const int nvw = P.nvw / CL;            // view warps of this CTA (CL = 2: half of the task's)
+    const uint32_t crank = CL == 1 ? 0u : cluster_rank();  // this CTA's rank in its cluster
     const bool is_view = warp < nvw, is_delta = warp == nvw, is_prior = warp == nvw + 1;
     const int vw = is_view ? warp : 0;
     const int V = P.V, M = P.M, S2 = P.S2, side = P.side;
-    const int VA = P.A.VA;                 // record positions / SVB columns in use
-    constexpr int VS = svb_cols(VPT);      // SVB row length (compile-time: row offsets are immediates)
+    const int VA = P.A.VA;                 // record positions per voxel (all views)
+    const int VAL = VA / CL;               // this CTA's record positions / SVB columns
+    const int vbase = (int)crank * VAL;    // this CTA's first view
+    constexpr int VS = svb_cols(VPT, CL);  // SVB row length (compile-time: row offsets are immediates)
     constexpr int RS = 2 * VS;             // float stride between consecutive e (or w) rows
     constexpr bool kNSL8 = VPT != 2;       // at most 8 view warps: only the first 8 slots are used
     const SmemLayout& L = P.lay;
@@ -299,7 +353,10 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     float* stg_w = (float*)(smem + L.staging) + vw * 32 * kStg;
     int* s_task = (int*)(smem + L.misc);            // [b]: the task prepared in buffer b, [2 + b]: its kept voxels
     float* dslot = (float*)(smem + L.misc) + 4;     // [2 steps]: scale * delta of the step's voxel
-    uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA]
+    uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA], indexed by (global) view
+    float* xs = (float*)(smem + L.cx);               // CL = 2: [2 steps][2 ranks] theta1 partial sums
+    uint64_t* xbar = (uint64_t*)(smem + L.cx + 16);  // CL = 2: [2 steps] the peer's partial arrived
+    uint64_t* tbar = xbar + 2;                       // CL = 2: [2 buffers] rank 0's task id arrived
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
     const int ntile = (NNB == 26 ? 3 : 1) * TW * TW;  // x tile entries
@@ -319,14 +376,20 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         nbt[96 + i] = ok ? __float_as_int(P.pc.b[i]) : 0;
         nbt[128 + i] = ok ? (P.pc.dz[i] * (side + 2) + P.pc.dy[i]) * (side + 2) + P.pc.dx[i] : 0;
     }
+    if (CL == 2 && threadIdx.x == 0) {
+        for (int i = 0; i < 4; ++i) mbar_init(xbar + i, 1);  // one arrival: the peer's
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
     __syncthreads();
+    if (CL == 2) cluster_sync_all();  // peer mbarriers initialised before any remote arrival
+    uint32_t nfetch[2] = {0u, 0u};    // CL = 2: task ids received per buffer (tbar phases)
     // SVB rows outside a visit's band are never packed: start them finite (zero)
     for (int i = threadIdx.x; i < (L.xt - L.sb_e) / 16; i += blockDim.x)
         ((float4*)(smem + L.sb_e))[i] = make_float4(0.f, 0.f, 0.f, 0.f);
     // per-thread view ownership: view warp w, lane l owns views (w*VPT + t)*32 + l
     int kv[VPT];
 #pragma unroll
-    for (int t = 0; t < VPT; ++t) kv[t] = (vw * VPT + t) * 32 + lane;
+    for (int t = 0; t < VPT; ++t) kv[t] = (vw * VPT + t) * 32 + lane;  // local SVB column
     uint32_t gseq = 0;  // running voxel sequence number of this CTA: A stage = gseq % R
     // prior-warp lane r owns neighbour r: offsets and weights in registers
     NbrOne nb;
@@ -375,9 +438,22 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     // delta warp: fetch the next task into s_task[b] and start copying its inputs into buffer b
     auto fetch_and_copy = [&](int b) {
         int qn = 0;
-        if (lane == 0) qn = fetch_task();
+        if (crank == 0) {
+            if (lane == 0) {
+                qn = fetch_task();
+                s_task[b] = qn;
+                if (CL == 2) {  // rank 1 takes the same task
+                    st_peer_u32(peer_addr(s_task + b, 1), (uint32_t)qn);
+                    mbar_arrive_peer(peer_addr(tbar + b, 1));
+                }
+            }
+        } else {
+            if (lane == 0) mbar_wait_cluster(tbar + b, nfetch[b] & 1u);
+            __syncwarp();
+            qn = s_task[b];
+        }
+        ++nfetch[b];
         qn = __shfl_sync(kFull, qn, 0);
-        if (lane == 0) s_task[b] = qn;
         if (qn < tend) {
             const int tkn = P.flat[qn];
             const int z = tkn >> 14, sv = tkn & 16383;
@@ -449,7 +525,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 }
                 if (lane == 0) {
                     s_task[2 + b] = n;
-                    if (n == 0) {  // the whole SV is zero-skipped: account for it
+                    if (n == 0 && crank == 0) {  // the whole SV is zero-skipped: account for it
                         P.sv_amount[(size_t)z * P.nsv + sv] = 0.f;
                         atomicAdd(P.counters + 1, (unsigned long long)(tw * th));
                         atomicAdd(P.counters + 2, 1ull);
@@ -509,8 +585,8 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         constexpr int CB = U8 ? 4 : 16;       // record bytes per view position
         const int tpm = vw * 32 + lane;
         const unsigned char* g_code = (const unsigned char*)(U8 ? (const void*)P.A.codes : (const void*)P.A.vals) +
-                                      ((size_t)arec * VA + tpm * VPT) * CB;
-        const unsigned char* g_off = P.A.off + (size_t)arec * VA + tpm * VPT;
+                                      ((size_t)arec * VA + vbase + tpm * VPT) * CB;
+        const unsigned char* g_off = P.A.off + (size_t)arec * VA + vbase + tpm * VPT;
         // view thread: asynchronous copy of its own slice of voxel j's record into ring stage stg,
         // one commit group per voxel (empty past the visit's end)
         auto copy_record_to = [&](int j, int stg, int v) {
@@ -554,7 +630,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         // ---- 4. view warps: SVB pack (coalesced band-row windows transposed through staging
         //         tiles); e_init rows go to this CTA's L2-resident scratch tile for the write-back
         float* scr = P.scratch + (size_t)blockIdx.x * (size_t)VS * 32;
-        const int ntw = tile_warps(VA);
+        const int ntw = tile_warps(VAL);
         if (is_view && vw < ntw) {
             const float* wz = P.w + (size_t)z * V * M;
             float* ez = P.e + (size_t)z * V * M;
@@ -564,7 +640,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             // c = p - s_k lands in sb row c, column k (bank k)
             const int sub = lane >> 3, ch = lane & 7;  // row-in-quad and float4 chunk of this lane
             auto issue = [&](int t, bool isw, float4 (&v4)[8]) {
-                const int kk = (vw * kTileW + t) * 32 + lane;
+                const int kk = vbase + (vw * kTileW + t) * 32 + lane;  // global view
                 const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
                 const int rot = (int)(bi >> 5);
 #pragma unroll
@@ -577,9 +653,9 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 }
             };
             auto finish = [&](int t, bool isw, const float4 (&v4)[8]) {
-                const int k0 = (vw * kTileW + t) * 32;
+                const int k0 = (vw * kTileW + t) * 32;  // local column of the tile
+                const uint32_t bi = vbase + k0 + lane < V ? binfo[tb * VA + vbase + k0 + lane] : 0u;
                 const int kk = k0 + lane;
-                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
                 const int bwt = (int)(bi & 31u), sk = (int)(bi >> 5) & 3;
                 const uint32_t bmask = ((1u << bwt) - 1u) << sk;  // band's window positions
                 if (!isw) {
@@ -759,6 +835,18 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                                    __fadd2_rn(make_float2(r3.x, r3.y), make_float2(r3.z, r3.w))));
                     S = q.x + q.y;
                 }
+                if (CL == 2) {
+                    // this CTA's partial sum to both CTAs; the peer's arrives on xbar[sn] (its
+                    // phase flips every second step); both add in rank order: identical bits
+                    if (lane == 0) {
+                        xs[sn * 2 + crank] = S;
+                        st_peer_f32(peer_addr(xs + sn * 2 + crank, crank ^ 1u), S);
+                        mbar_arrive_peer(peer_addr(xbar + sn, crank ^ 1u));
+                        mbar_wait_cluster(xbar + sn, ((g0 + (uint32_t)idx) >> 1) & 1u);
+                    }
+                    __syncwarp();
+                    S = xs[sn * 2] + xs[sn * 2 + 1];
+                }
                 const float theta1 = -scale * S;  // Alg1:5
                 float u = pp.v;
                 if (den > 0.f) u = (c1 - theta1) * rden;
@@ -770,7 +858,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 v_prev = pp.v;
                 if (lane == 0) {
                     amount += fabsf(d);
-                    if (P.dump) {
+                    if (P.dump && crank == 0) {
                         // test hook (mbir_set_update_dump): the update's (voxel, theta1, theta2,
                         // delta) exactly as the delta chain used them
                         const unsigned long long slot = atomicAdd(P.dump_count, 1ull);
@@ -818,9 +906,9 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             for (int t = 0; t < kTileW; ++t) {
                 if (t + 1 < kTileW) ld_init(t + 1, s4b[(t + 1) & 1]);
                 const float4 (&s4)[8] = s4b[t & 1];
-                const int k0 = (vw * kTileW + t) * 32;
+                const int k0 = (vw * kTileW + t) * 32;  // local column of the tile
                 const int kk = k0 + lane;
-                const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
+                const uint32_t bi = vbase + kk < V ? binfo[tb * VA + vbase + kk] : 0u;
                 const int bw = (int)(bi & 31u), roff = (int)(bi >> 5);
                 const uint32_t bmask = ((1u << bw) - 1u) << (roff & 3);
                 // this view's final band -> its staging row (positions outside the band: 0)
@@ -847,18 +935,18 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                     float d[4];
 #pragma unroll
                     for (int j = 0; j < 4; ++j) d[j] = (nib & (1u << j)) ? fv[j] - e0[j] : 0.f;
-                    if (k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
+                    if (vbase + k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
                         red_add_v4(ez + (oi - (oi & 3)) + 4 * ch, d[0], d[1], d[2], d[3]);
                 }
                 __syncwarp();
             }
         } else if (is_delta) {
             // the image and the counters, then the next task's preparation (with the prior warp)
-            for (int i = lane; i < tw * th; i += 32) {
+            for (int i = lane; i < tw * th && crank == 0; i += 32) {
                 const int lx = i % tw, ly = i / tw;
                 P.x[(size_t)(z + 1) * plane + (size_t)(gy0 + ly) * P.nx + gx0 + lx] = xt[cslot + ly * TW + lx];
             }
-            if (lane == 0) {
+            if (lane == 0 && crank == 0) {
                 P.sv_amount[(size_t)z * P.nsv + sv] = amount;
                 atomicAdd(P.counters + 0, (unsigned long long)nactv);
                 atomicAdd(P.counters + 1, (unsigned long long)(tw * th - nactv));
@@ -870,7 +958,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             finish_prepare(cb ^ 1);
         }
         __syncthreads();
-        if (PROF && threadIdx.x == 0) {
+        if (PROF && threadIdx.x == 0 && crank == 0) {
             const long long tp4 = clock64();
             atomicAdd(P.tprof + 0, (unsigned long long)(tp1 - tp0));  // x tile, zero-skip, order
             atomicAdd(P.tprof + 1, (unsigned long long)(tp2 - tp1));  // SVB pack
@@ -880,85 +968,113 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             atomicAdd(P.tprof + 5, 1ull);
         }
     }
+    if (CL == 2) cluster_sync_all();  // no CTA leaves while its peer may still write into it
 }
 
 // A-record ring depth (voxels of cp.async lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
 // (the pair loop needs >= 4: the current pair's two stages plus the next pair's two)
 constexpr int ring_depth(bool u8) { return u8 ? 12 : 4; }
 
-template <int VPT, bool U8, int NNB>
+template <int VPT, bool U8, int NNB, int CL>
 cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
 {
     constexpr int R = ring_depth(U8);
-    auto kern = p.tprof ? k_svicd<VPT, U8, NNB, R, true> : k_svicd<VPT, U8, NNB, R, false>;
+    auto kern = p.tprof ? k_svicd<VPT, U8, NNB, R, CL, true> : k_svicd<VPT, U8, NNB, R, CL, false>;
     IcdParams q = p;
-    q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT, p.V);
+    q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT, p.V, CL);
     const int smem = q.lay.total;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     if (e != cudaSuccess) return e;
-    kern<<<gx, 32 * (p.nvw + 2), smem, st>>>(q);
-    return cudaGetLastError();
+    const int threads = 32 * (p.nvw / CL + 2);
+    if (CL == 1) {
+        kern<<<gx, threads, smem, st>>>(q);
+        return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(gx);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, q);
 }
+
+template <int VPT, bool U8, int NNB, int CL>
+int resident_t(const IcdParams& p)
+{
+    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), CL, false>;
+    const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT, p.V, CL).total;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
+    cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    const int threads = 32 * (p.nvw / CL + 2);
+    if (CL == 1) {
+        int nb = 0, dev = 0, nsm = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, threads, smem) != cudaSuccess) return -1;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        return nb * nsm;
+    }
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(4 * 148);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int ncl = 0;
+    if (cudaOccupancyMaxActiveClusters(&ncl, kern, &cfg) != cudaSuccess) return -1;
+    return ncl * CL;
+}
+
+#define SVICD_DISPATCH(FN, ...)                                                                      \
+    if (cl == 2) {                                                                                   \
+        if (quantize) return nnb == 26 ? FN<4, true, 26, 2>(__VA_ARGS__) : FN<4, true, 8, 2>(__VA_ARGS__); \
+        return nnb == 26 ? FN<4, false, 26, 2>(__VA_ARGS__) : FN<4, false, 8, 2>(__VA_ARGS__);       \
+    }                                                                                                \
+    if (vpt == 3) {                                                                                  \
+        if (quantize) return nnb == 26 ? FN<3, true, 26, 1>(__VA_ARGS__) : FN<3, true, 8, 1>(__VA_ARGS__); \
+        return nnb == 26 ? FN<3, false, 26, 1>(__VA_ARGS__) : FN<3, false, 8, 1>(__VA_ARGS__);       \
+    }                                                                                                \
+    if (vpt == 2) {                                                                                  \
+        if (quantize) return nnb == 26 ? FN<2, true, 26, 1>(__VA_ARGS__) : FN<2, true, 8, 1>(__VA_ARGS__); \
+        return nnb == 26 ? FN<2, false, 26, 1>(__VA_ARGS__) : FN<2, false, 8, 1>(__VA_ARGS__);       \
+    }                                                                                                \
+    if (vpt == 1) {                                                                                  \
+        if (quantize) return nnb == 26 ? FN<1, true, 26, 1>(__VA_ARGS__) : FN<1, true, 8, 1>(__VA_ARGS__); \
+        return nnb == 26 ? FN<1, false, 26, 1>(__VA_ARGS__) : FN<1, false, 8, 1>(__VA_ARGS__);       \
+    }                                                                                                \
+    if (quantize) return nnb == 26 ? FN<4, true, 26, 1>(__VA_ARGS__) : FN<4, true, 8, 1>(__VA_ARGS__); \
+    return nnb == 26 ? FN<4, false, 26, 1>(__VA_ARGS__) : FN<4, false, 8, 1>(__VA_ARGS__);
 
 }  // namespace
 
-int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize)
+int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl)
 {
-    return svicd_layout(p.rows, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw, vpt, p.V).total;
+    return svicd_layout(p.rows, p.side, p.S2, nnb, p.A.VA, quantize, ring_depth(quantize), p.nvw, vpt, p.V, cl).total;
 }
 
-template <int VPT, bool U8, int NNB>
-int resident_t(const IcdParams& p)
+int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int cl)
 {
-    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), false>;
-    const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT, p.V).total;
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
-    cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    int nb = 0, dev = 0, nsm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, 32 * (p.nvw + 2), smem) != cudaSuccess) return -1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    return nb * nsm;
-}
-
-int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize)
-{
-    if (vpt == 3) {
-        if (quantize) return nnb == 26 ? resident_t<3, true, 26>(p) : resident_t<3, true, 8>(p);
-        return nnb == 26 ? resident_t<3, false, 26>(p) : resident_t<3, false, 8>(p);
-    }
-    if (vpt == 2) {
-        if (quantize) return nnb == 26 ? resident_t<2, true, 26>(p) : resident_t<2, true, 8>(p);
-        return nnb == 26 ? resident_t<2, false, 26>(p) : resident_t<2, false, 8>(p);
-    }
-    if (vpt == 1) {
-        if (quantize) return nnb == 26 ? resident_t<1, true, 26>(p) : resident_t<1, true, 8>(p);
-        return nnb == 26 ? resident_t<1, false, 26>(p) : resident_t<1, false, 8>(p);
-    }
-    if (quantize) return nnb == 26 ? resident_t<4, true, 26>(p) : resident_t<4, true, 8>(p);
-    return nnb == 26 ? resident_t<4, false, 26>(p) : resident_t<4, false, 8>(p);
+    SVICD_DISPATCH(resident_t, p)
 }
 
 int svicd_scratch_floats(int vpt) { return svb_cols(vpt) * 32; }
 
-cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int grid, cudaStream_t st)
+cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int cl, int grid, cudaStream_t st)
 {
-    if (vpt == 3) {
-        if (quantize) return nnb == 26 ? launch_t<3, true, 26>(p, grid, st) : launch_t<3, true, 8>(p, grid, st);
-        return nnb == 26 ? launch_t<3, false, 26>(p, grid, st) : launch_t<3, false, 8>(p, grid, st);
-    }
-    if (vpt == 2) {
-        if (quantize) return nnb == 26 ? launch_t<2, true, 26>(p, grid, st) : launch_t<2, true, 8>(p, grid, st);
-        return nnb == 26 ? launch_t<2, false, 26>(p, grid, st) : launch_t<2, false, 8>(p, grid, st);
-    }
-    if (vpt == 1) {
-        if (quantize) return nnb == 26 ? launch_t<1, true, 26>(p, grid, st) : launch_t<1, true, 8>(p, grid, st);
-        return nnb == 26 ? launch_t<1, false, 26>(p, grid, st) : launch_t<1, false, 8>(p, grid, st);
-    }
-    if (quantize) return nnb == 26 ? launch_t<4, true, 26>(p, grid, st) : launch_t<4, true, 8>(p, grid, st);
-    return nnb == 26 ? launch_t<4, false, 26>(p, grid, st) : launch_t<4, false, 8>(p, grid, st);
+    SVICD_DISPATCH(launch_t, p, grid, st)
 }
 
 }  // namespace mbir

@@ -67,11 +67,12 @@ def _replay(og, pr, Aq, case, x32, vox, t1g, t2g, dg):
 
 
 CASES = {
-    # (config, nbhd, quantize_A, sweeps of the oracle to reach the fixed state)
-    "cfg1-u8": (CONFIGS["cfg1"], 8, 1, 3),
-    "cfg1-f32": (CONFIGS["cfg1"], 8, 0, 3),
-    "mini720-u8": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2),
-    "mini3d-f32": (WorkloadConfig("mini3d", 40, 4, 60, 64, 7, 26, 0.002), 26, 0, 2),
+    # (config, nbhd, quantize_A, sweeps of the oracle to reach the fixed state, CTAs per task)
+    "cfg1-u8": (CONFIGS["cfg1"], 8, 1, 3, 1),
+    "cfg1-f32": (CONFIGS["cfg1"], 8, 0, 3, 1),
+    "mini720-u8": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 1),
+    "mini720-u8-cluster2": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 2),
+    "mini3d-f32": (WorkloadConfig("mini3d", 40, 4, 60, 64, 7, 26, 0.002), 26, 0, 2, 1),
 }
 
 
@@ -81,8 +82,9 @@ def test_hot_kernel_every_update_matches_oracle(name):
     of each pair), theta2 (precomputed per sinogram) and delta (neighbour-corrected prior) for every
     update of one deterministic sweep from a non-trivial state, against Alg. 1 in the oracle at the
     identical state: reading R20's 1e-5.  mini720 is the bench's launch shape (720 views, 4 views
-    per lane, six view warps, uint8 A, 26-neighbourhood)."""
-    cfg, nbhd, quant, sweeps = CASES[name]
+    per lane, six view warps, uint8 A, 26-neighbourhood); cluster2 splits every task's views over a
+    2-CTA cluster that exchanges the partial sums through distributed shared memory."""
+    cfg, nbhd, quant, sweeps, cl = CASES[name]
     case = make_case(cfg)
     g, og = geoms(cfg)
     A = O.sysmatrix(og)
@@ -90,7 +92,9 @@ def test_hot_kernel_every_update_matches_oracle(name):
     pr, x32 = _state(cfg, case, og, Ause, nbhd, sweeps)
     nvox = x32.size
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=nbhd),
-                         M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0, quantize_A=quant)) as r:
+                         M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0, quantize_A=quant,
+                                   cluster=cl)) as r:
+        assert r.sizes()["cluster"] == cl
         r.set_sinogram(case.y, case.w)
         r.set_image(x32.reshape(cfg.nz, cfg.n, cfg.n))
         r.set_update_dump(nvox + 16)

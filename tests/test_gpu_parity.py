@@ -384,7 +384,8 @@ def m720():
     return cfg, case, g, og, Aq
 
 
-def test_bench_shape_deterministic_tracks_oracle(m720):
+@pytest.mark.parametrize("cluster", [1, 2])
+def test_bench_shape_deterministic_tracks_oracle(m720, cluster):
     """The launch configuration bench.py times (uint8 A, 4 views per lane, 6 view warps + the
     delta and prior warps, one CTA per task): deterministic order, 2 equits, against the
     sequential oracle."""
@@ -392,8 +393,8 @@ def test_bench_shape_deterministic_tracks_oracle(m720):
     pr = O.Prior(sigma=cfg.sigma, nbhd=26)
     order = deterministic_order(cfg.n, cfg.nz, cfg.sv_side, 26)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
-                         M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0)) as r:
-        assert r.sizes()["cluster"] == 1
+                         M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0, cluster=cluster)) as r:
+        assert r.sizes()["cluster"] == cluster
         r.set_sinogram(case.y, case.w)
         x = np.zeros(cfg.nz * cfg.n * cfg.n)
         e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
@@ -408,7 +409,8 @@ def test_bench_shape_deterministic_tracks_oracle(m720):
     assert np.abs(eg.ravel() - e.ravel()).max() < 1e-4 * np.abs(case.y).max()
 
 
-def test_bench_shape_converged_matches_oracle(m720):
+@pytest.mark.parametrize("cluster", [1, 2])
+def test_bench_shape_converged_matches_oracle(m720, cluster):
     """Asynchronous GPU-ICD in the bench's launch shape (persistent grid, random orders, 25 %
     SV selection, zero-skipping off) reaches the oracle's MAP point: 1 HU / 1e-4."""
     cfg, case, g, og, Aq = m720
@@ -417,7 +419,7 @@ def test_bench_shape_converged_matches_oracle(m720):
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
     O.icd_run(og, pr, Aq, case.w, x, e, 80, seed=3000, zero_skip=False)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
-                         M.Options(sv_side=cfg.sv_side, zero_skip=0)) as r:
+                         M.Options(sv_side=cfg.sv_side, zero_skip=0, cluster=cluster)) as r:
         r.set_sinogram(case.y, case.w)
         r.reconstruct(200)
         xg = r.image().ravel().astype(np.float64)
@@ -428,17 +430,22 @@ def test_bench_shape_converged_matches_oracle(m720):
 
 
 def test_cluster_option_validation():
-    """One CTA owns an SV task (include/mbir.h mbir_options.cluster): 0 (auto) and 1 are
-    accepted, anything else is EINVAL."""
+    """CTAs per SV task (include/mbir.h mbir_options.cluster): 0 (auto) and 1 = one CTA; 2 = a
+    2-CTA cluster splitting the views, which needs > 128 views in an even number of 128-view warps;
+    anything else is EINVAL."""
     cfg = CONFIGS["cfg1"]  # 90 views: three warps of 1 view per lane
     g, _ = geoms(cfg)
-    for bad in (2, -1):
+    for bad in (2, 3, -1):
         with pytest.raises(M.MbirError) as ei:
             M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side, cluster=bad))
         assert ei.value.code == -1
     with M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=cfg.sv_side)) as r:
         assert r.sizes()["cluster"] == 1
         assert r.sizes()["threads_per_cta"] == 32 * (3 + 2)
+    cfg = mini720()
+    g, _ = geoms(cfg)
+    with M.Reconstructor(g, M.Prior(neighborhood=26), M.Options(sv_side=cfg.sv_side, cluster=2)) as r:
+        assert r.sizes()["cluster"] == 2 and r.sizes()["threads_per_cta"] == 32 * (3 + 2)
 
 
 # ------------------------------------------------------------------ FBP initial image (R23)

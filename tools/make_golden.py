@@ -41,6 +41,7 @@ def main():
     ap.add_argument("--equits", type=int, default=100)
     ap.add_argument("--threads", type=int, default=0)
     ap.add_argument("--out", default="")
+    ap.add_argument("--resume", default="", help="continue from this golden file's image (sweeps numbered on)")
     a = ap.parse_args()
     cfg = CONFIGS[a.config]
     t0 = time.time()
@@ -49,19 +50,27 @@ def main():
     A = O.sysmatrix(og)
     _, _, Aq = O.quantize(A)  # the uint8 A the GPU path runs with
     pr = O.Prior(sigma=cfg.sigma, nbhd=cfg.nbhd)
-    x = O.fbp(og, case.y).ravel().copy()
+    first = 1
+    if a.resume:
+        z0 = np.load(a.resume)
+        m0 = json.loads(str(z0["meta"]))
+        assert m0["sino_sha"] == sino_hash(case.y, case.w)
+        x = z0["x"].ravel().astype(np.float64).copy()
+        first = m0["equits"] + 1
+    else:
+        x = O.fbp(og, case.y).ravel().copy()
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
     print(f"setup {time.time() - t0:.0f} s", flush=True)
     hist, prev = [], None
     for s in range(1, a.equits + 1):
-        O.icd_run_zpar(og, pr, Aq, case.w, x, e, 1, first_sweep=s, seed=7000, zero_skip=False,
+        O.icd_run_zpar(og, pr, Aq, case.w, x, e, 1, first_sweep=first + s - 1, seed=7000, zero_skip=False,
                        threads=a.threads or None)
         if s == a.equits - 20:
             prev = x.copy()
         if s % 10 == 0:
             print(f"equit {s}  {time.time() - t0:.0f} s", flush=True)
     selfconv = O.rmse_hu(prev, x) if prev is not None else None
-    meta = {"config": a.config, "case_id": 0, "init": "oracle FBP (clipped at 0)", "equits": a.equits,
+    meta = {"config": a.config, "case_id": 0, "init": "oracle FBP (clipped at 0)", "equits": first - 1 + a.equits,
             "order": "random per sweep and slice, slice-parity halves (oracle.icd_run_zpar), seed 7000",
             "zero_skip": False, "A": "uint8 codes (oracle.quantize)", "sigma": cfg.sigma, "nbhd": cfg.nbhd,
             "selfconv_hu_last20": selfconv, "sino_sha": sino_hash(case.y, case.w),
