@@ -175,7 +175,10 @@ def run_reference(args, rank, world):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot_t / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "impl": "reference",
-            "config": workload_config(cfg_full, args.sv_side or cfg_full.sv_side, args, world),
+            "config": dict(workload_config(cfg_full, args.sv_side or cfg_full.sv_side, args, world),
+                           sample="the oracle times a bounded sample with the workload's per-update work "
+                                  "(a 128x128 slice at config-4 pitch, 720 views x 256 channels, 2396 "
+                                  "nnz/voxel), not the whole cfg4 volume"),
             "cpu_baseline": {"value": v, "unit": "voxel updates/s", "cores": 1, "kind": "oracle",
                              "sample": "each step: >= 3 s of sequential-oracle equits on a bounded "
                                        "sample of the workload's per-update work: a 128x128 slice "

@@ -596,3 +596,27 @@ def test_paper_scale_error_sinogram_consistent_on_sampled_rays(name):
         busy += acc > 0.1 * abs(float(ys[z, k, m]))
         assert abs(float(eg[z, k, m]) - ref) <= 2e-4 * max(1.0, abs(float(ys[z, k, m]))), (z, k, m, eg[z, k, m], ref)
     assert busy >= 3  # the sampled rays cross the reconstructed object
+
+
+def test_bench_template_mid_size_3d_converges_to_oracle_map():
+    """The bench's kernel template at a size the oracle can converge: 96^2 x 8
+    slices, 720 views x 192 channels (dc = dxy/2, paper pitch ratio), SV side 9, uint8 A,
+    26-neighbourhood, zero-skip with re-admission, whole colour groups per launch (unbatched, as
+    cfg4 runs), from x0 = 0 -- against the oracle's no-skip MAP (slice-parity threads): 1 HU / 1e-4."""
+    cfg = WorkloadConfig("mid3d", 96, 8, 720, 192, 9, 26, 0.005)
+    case = make_case(cfg)
+    g, og = geoms(cfg)
+    _, _, Aq = O.quantize(O.sysmatrix(og))
+    pr = O.Prior(sigma=cfg.sigma, nbhd=26)
+    x = O.fbp(og, case.y).ravel().copy()
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+    O.icd_run_zpar(og, pr, Aq, case.w, x, e, 60, seed=3000, zero_skip=False)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
+                         M.Options(sv_side=cfg.sv_side, batch_svs=100000, batch_threshold=0)) as r:
+        r.set_sinogram(case.y, case.w)
+        r.reconstruct(120)
+        xg = r.image().ravel().astype(np.float64)
+    assert O.rmse_hu(xg, x) < 1.0, O.rmse_hu(xg, x)
+    cg = O.cost(og, pr, Aq, case.y, case.w, xg)
+    co = O.cost(og, pr, Aq, case.y, case.w, x)
+    assert abs(cg - co) <= 1e-4 * abs(co), (cg, co)
