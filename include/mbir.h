@@ -170,8 +170,10 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* p, const mbir_options*
 
 /* Load the measured sinogram y and its weights w (inverse noise variance), both
  * [nz_local][nviews][nchannels].  Resets the error sinogram e = y - A x for the current image
- * (Alg. 1 input) and the scheduler state.  Errors: EINVAL (NULL, NaN/Inf or negative w),
- * ECUDA. */
+ * (Alg. 1 input) and the scheduler state.  theta2 = A^T W A (Alg1:6), which depends only on w,
+ * is computed by the next iteration's update kernel (the first iteration visits every voxel),
+ * or by a separate pass first when a batch threshold could drop tasks.  Errors: EINVAL (NULL,
+ * NaN/Inf or negative w), ECUDA. */
 int mbir_set_sinogram(mbir_handle* h, const float* y, const float* w, int where);
 
 /* Set the image (warm start / resume; default 0).  x0 == NULL sets 0.  Recomputes e = y - A x

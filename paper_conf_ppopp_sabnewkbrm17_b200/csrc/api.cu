@@ -25,9 +25,6 @@ using namespace mbir;
 
 // views per lane of the update kernel for > 128 views (build-time choice: 4 = six view warps,
 // 2 = twelve)
-#ifndef MBIR_WIDE_VPT
-#define MBIR_WIDE_VPT 4
-#endif
 
 namespace {
 
@@ -130,6 +127,7 @@ struct mbir_handle {
     double* d_acc = nullptr;
     unsigned long long* h_counters = nullptr;  // pinned [5] (4 counters + sum_delta bits)
     bool have_sino = false;
+    bool theta2_ok = false;  // d_theta2 holds sum w A^2 for the current weights
     bool x_zero = true;  // the image is known to be all zero (then e = y needs no projection)
     int iter = 0;
     int64_t nnz = 0, a_bytes = 0, band_entries = 0;
@@ -277,8 +275,8 @@ int timed_icd(mbir_handle* h, const IcdParams& p, int nnb, bool q, int gx, int g
     return MBIR_OK;
 }
 
-// e = y - A x (and theta2 when the weights changed)
-int refresh_error(mbir_handle* h, bool theta2)
+// e = y - A x
+int refresh_error(mbir_handle* h)
 {
     IcdParams p = make_params(h);
     const bool q = h->o.quantize_A != 0;
@@ -286,7 +284,6 @@ int refresh_error(mbir_handle* h, bool theta2)
         CK(cudaMemcpyAsync(h->d_e, h->d_y, sino_elems(h) * 4, cudaMemcpyDeviceToDevice, h->st));
     else
         CK(launch_forward(p, q, h->d_y, h->st));
-    if (theta2) CK(launch_theta2(p, q, h->st));
     return MBIR_OK;
 }
 
@@ -363,6 +360,19 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
         ++launches;
         CK(cudaMemsetAsync(h->d_fetch, 0, sizeof(int) * 8 * nb, h->st));
         IcdParams p = make_params(h);
+        // theta2 = sum w A^2 (Alg1:6) after new weights: reduced inside the update kernel during an
+        // iteration that visits every voxel (the first one, unless a batch threshold drops tasks);
+        // otherwise by the separate k_theta2 pass first
+        p.theta2_pass = 0;
+        if (!h->theta2_ok) {
+            if (h->iter == 1 && thr == 0) {
+                p.theta2_pass = 1;
+            } else {
+                CK(launch_theta2(p, q, h->st));
+                ++launches;
+                h->theta2_ok = true;
+            }
+        }
         // zero-skip from iteration 2 on, except in re-admission iterations
         p.zero_skip_active = (h->o.zero_skip && h->iter > 1 && !readmit) ? 1 : 0;
         const size_t cap = (size_t)h->g.nz_local * h->max_group;
@@ -397,6 +407,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
                 if (r) return r;
             }
         }
+        if (p.theta2_pass) h->theta2_ok = true;
         if (h->nranks > 1 && h->comm) {
             CKN(nccl().AllReduce(h->d_counters, h->d_counters, 4, ncclUint64, ncclSum, h->comm, h->st));
             CKN(nccl().AllReduce(h->d_sum_delta, h->d_sum_delta, 1, ncclFloat64, ncclSum, h->comm, h->st));
@@ -768,6 +779,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     cudaMemsetAsync(h->d_e, 0, (ns + 32) * 4, h->st);
     if ((r = dalloc(h, &h->d_x, pl * (G.nz_local + 2)))) return bail(r);
     if ((r = dalloc(h, &h->d_theta2, (size_t)G.nz_local * h->nsv * h->S2))) return bail(r);
+    cudaMemset(h->d_theta2, 0, (size_t)G.nz_local * h->nsv * h->S2 * sizeof(float));
     if ((r = dalloc(h, &h->d_amount, (size_t)G.nz_local * h->nsv))) return bail(r);
     // e_init tiles of the concurrently running SV visits: one per CTA of the largest grid
     if ((r = dalloc(h, &h->d_scratch, (size_t)h->nsm * h->blocks_per_sm * svicd_scratch_floats(h->vpt)))) return bail(r);
@@ -877,8 +889,9 @@ int mbir_set_sinogram(mbir_handle* h, const float* y, const float* w, int where)
         h->have_sino = false;
         return fail(h, MBIR_EINVAL, "y must be finite and w finite and >= 0");
     }
-    int r = refresh_error(h, true);
+    int r = refresh_error(h);  // theta2 follows in the first iteration (run_iterations)
     if (r) return r;
+    h->theta2_ok = false;
     CK(cudaMemsetAsync(h->d_amount, 0, sizeof(float) * h->g.nz_local * h->nsv, h->st));
     CK(cudaStreamSynchronize(h->st));
     h->have_sino = true;
@@ -918,7 +931,7 @@ int mbir_set_image(mbir_handle* h, const float* x0, int where)
     int r = exchange_halo(h, -1);
     if (r) return r;
     if (h->have_sino) {
-        r = refresh_error(h, false);
+        r = refresh_error(h);
         if (r) return r;
     }
     CK(cudaMemsetAsync(h->d_amount, 0, sizeof(float) * h->g.nz_local * h->nsv, h->st));
@@ -941,7 +954,7 @@ int mbir_init_fbp(mbir_handle* h)
     h->x_zero = false;
     int r = exchange_halo(h, -1);
     if (r) return r;
-    r = refresh_error(h, false);
+    r = refresh_error(h);
     if (r) return r;
     CK(cudaMemsetAsync(h->d_amount, 0, sizeof(float) * h->g.nz_local * h->nsv, h->st));
     CK(cudaStreamSynchronize(h->st));

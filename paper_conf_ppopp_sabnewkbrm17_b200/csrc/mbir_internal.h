@@ -10,6 +10,12 @@
 
 #include "../../include/mbir.h"
 
+// views per thread of the update kernel when nviews > 128 (VPT = 1 below).  4 is the measured
+// best (VPT 2 and 3 were 35-43 % slower); other values are a rebuild
+#ifndef MBIR_WIDE_VPT
+#define MBIR_WIDE_VPT 4
+#endif
+
 namespace mbir {
 
 constexpr int kK = 4;             // max channels per (voxel, view) (reading R5; K=4 for dc > 0.4714 dxy)
@@ -88,6 +94,7 @@ struct IcdParams {
     uint64_t seed;
     int iter;
     int zero_skip_active;
+    int theta2_pass;  // this launch reduces theta2 (Alg1:6) with theta1 and stores it (iteration 1)
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)
     PriorConst pc;           // q-GGMRF constants and neighbourhood of this handle (reading R1-R2)

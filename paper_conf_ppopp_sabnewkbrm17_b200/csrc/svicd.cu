@@ -253,7 +253,7 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     L.list = o;  o = align16(o + 2 * S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
     L.tof = o;   o = align16(o + 2 * S2 * 4);
-    L.red = o;   o = align16(o + 2 * kNSL * 4);  // [2 steps][kNSL view warps] theta1 partials
+    L.red = o;   o = align16(o + 2 * 2 * kNSL * 4);  // [2 steps][theta1, theta2][kNSL view warps] partials
     L.pri = o;   o = align16(o + 2 * (int)sizeof(PriTerm));
     L.vscale = o; o = align16(o + 2 * S2 * 4);
     L.vth2 = o;  o = align16(o + 2 * S2 * 4);
@@ -271,7 +271,7 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     L.rbs = o;   o = align16(o + V * 4);        //   band start and width per view
     L.rbw = o;   o = align16(o + V);
     L.binfo = o; o = align16(o + 2 * VA * cl * 4);  // band (row offset << 5 | width) per view, 2 tasks
-    L.cx = o;    o = align16(o + 2 * 2 * 4 + 4 * 8);  // CL = 2: partial theta1 sums [2 steps][2 CTAs], mbarriers
+    L.cx = o;    o = align16(o + 2 * 2 * 2 * 4 + 4 * 8);  // CL = 2: partial sums [2 steps][2 quantities][2 CTAs], mbarriers
     L.total = o;
     return L;
 }
@@ -328,7 +328,9 @@ __device__ __forceinline__ void load_words(const unsigned char* stg, int off_in_
 
 // The update kernel.  VPT views per lane (4, or 1 for <= 128 views), uint8 or fp32 A, 8 or 26
 // neighbours, R-voxel A-record ring; PROF adds per-phase cycle counters.
-template <int VPT, bool U8, int NNB, int R, int CL, bool PROF>
+// T2: the theta2 pass -- theta2 = sum w A^2 (Alg1:6) is not precomputed yet: the view warps reduce
+// it with theta1 in this iteration (which visits every voxel) and the delta warp stores it
+template <int VPT, bool U8, int NNB, int R, int CL, bool T2, bool PROF>
 __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
@@ -354,8 +356,8 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     int* s_task = (int*)(smem + L.misc);            // [b]: the task prepared in buffer b, [2 + b]: its kept voxels
     float* dslot = (float*)(smem + L.misc) + 4;     // [2 steps]: scale * delta of the step's voxel
     uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA], indexed by (global) view
-    float* xs = (float*)(smem + L.cx);               // CL = 2: [2 steps][2 ranks] theta1 partial sums
-    uint64_t* xbar = (uint64_t*)(smem + L.cx + 16);  // CL = 2: [2 steps] the peer's partial arrived
+    float* xs = (float*)(smem + L.cx);               // CL = 2: [2 steps][2 quantities][2 ranks] partial sums
+    uint64_t* xbar = (uint64_t*)(smem + L.cx + 32);  // CL = 2: [2 steps] the peer's partials arrived
     uint64_t* tbar = xbar + 2;                       // CL = 2: [2 buffers] rank 0's task id arrived
     const int TW = side + 2;
     const int zc = (NNB == 26) ? 1 : 0;  // centre slice of the x tile
@@ -364,7 +366,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     const int nab = (nvw + 1) * 32;      // barrier A: view warps + the delta warp
     const int nb2 = (nvw + 1) * 32;      // barrier B: view warps + the delta warp
 
-    for (int i = threadIdx.x; i < 2 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
+    for (int i = threadIdx.x; i < 2 * 2 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
     // the neighbourhood (reading R2) as shared-memory tables [dx | dy | dz | weight bits][32]: a
     // by-value kernel parameter indexed by a run-time value would be copied to local memory
     int* nbt = (int*)(smem + L.mbar);
@@ -746,6 +748,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 float2 ev[VPT][2];
                 {
                     float2 acc[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+                    float2 acc2 = make_float2(0.f, 0.f);  // T2: w A^2 (unscaled codes)
 #pragma unroll
                     for (int t = 0; t < VPT; ++t) {
                         const float* pe = sb + cur.p[t];
@@ -753,12 +756,22 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                         ev[t][1] = make_float2(pe[2 * RS], pe[3 * RS]);
                         acc[t & 1] = __ffma2_rn(cur.wf[t][0], ev[t][0], acc[t & 1]);
                         acc[t & 1] = __ffma2_rn(cur.wf[t][1], ev[t][1], acc[t & 1]);
+                        if (T2) {
+                            acc2 = __ffma2_rn(cur.wf[t][0], cur.f[t][0], acc2);
+                            acc2 = __ffma2_rn(cur.wf[t][1], cur.f[t][1], acc2);
+                        }
                     }
                     const float2 ac = __fadd2_rn(acc[0], acc[1]);
-                    float g = ac.x + ac.y;
+                    float g = ac.x + ac.y, g2 = acc2.x + acc2.y;
 #pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) g += __shfl_xor_sync(kFull, g, o);
-                    if (lane == 0) red[sn * kNSL + vw] = g;
+                    for (int o = 16; o > 0; o >>= 1) {
+                        g += __shfl_xor_sync(kFull, g, o);
+                        if (T2) g2 += __shfl_xor_sync(kFull, g2, o);
+                    }
+                    if (lane == 0) {
+                        red[sn * 2 * kNSL + vw] = g;
+                        if (T2) red[sn * 2 * kNSL + kNSL + vw] = g2;
+                    }
                 }
                 bar_arrive(kBarA, nab);
                 // meanwhile: the next voxel's e-independent state, then refill its stage
@@ -815,37 +828,49 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                     psx += bn * u_prev - pp.btu * v_prev;
                 }
                 const float scale = vscale[idx];
-                const float theta2 = vth2[idx];  // Alg1:6 (precomputed)
-                const float den = theta2 + 2.f * ps;
-                const float c1 = theta2 * pp.v + 2.f * psx;  // numerator without -theta1
-                const float rden = den > 0.f ? __fdividef(1.f, den) : 0.f;
+                float theta2 = T2 ? 0.f : vth2[idx];  // Alg1:6 (precomputed, or reduced below)
+                float den = theta2 + 2.f * ps;
+                float c1 = theta2 * pp.v + 2.f * psx;  // numerator without -theta1
+                float rden = den > 0.f ? __fdividef(1.f, den) : 0.f;
                 bar_sync(kBarA, nab);
-                const float4 r0 = *(const float4*)(red + sn * kNSL), r1 = *(const float4*)(red + sn * kNSL + 4);
-                float S;
-                if (kNSL8) {  // <= 8 view warps: slots 8.. are zero; fixed tree order
-                    const float2 q = __fadd2_rn(__fadd2_rn(make_float2(r0.x, r0.y), make_float2(r0.z, r0.w)),
-                                                __fadd2_rn(make_float2(r1.x, r1.y), make_float2(r1.z, r1.w)));
-                    S = q.x + q.y;
-                } else {
-                    const float4 r2 = *(const float4*)(red + sn * kNSL + 8), r3 = *(const float4*)(red + sn * kNSL + 12);
-                    const float2 q = __fadd2_rn(
-                        __fadd2_rn(__fadd2_rn(make_float2(r0.x, r0.y), make_float2(r0.z, r0.w)),
-                                   __fadd2_rn(make_float2(r1.x, r1.y), make_float2(r1.z, r1.w))),
-                        __fadd2_rn(__fadd2_rn(make_float2(r2.x, r2.y), make_float2(r2.z, r2.w)),
-                                   __fadd2_rn(make_float2(r3.x, r3.y), make_float2(r3.z, r3.w))));
-                    S = q.x + q.y;
-                }
+                // sum of the view warps' partials in a fixed tree order (<= 8 or 16 slots)
+                auto slot_sum = [&](const float* rq) {
+                    const float4 r0 = *(const float4*)rq, r1 = *(const float4*)(rq + 4);
+                    float2 q = __fadd2_rn(__fadd2_rn(make_float2(r0.x, r0.y), make_float2(r0.z, r0.w)),
+                                          __fadd2_rn(make_float2(r1.x, r1.y), make_float2(r1.z, r1.w)));
+                    if (!kNSL8) {
+                        const float4 r2 = *(const float4*)(rq + 8), r3 = *(const float4*)(rq + 12);
+                        q = __fadd2_rn(q, __fadd2_rn(__fadd2_rn(make_float2(r2.x, r2.y), make_float2(r2.z, r2.w)),
+                                                     __fadd2_rn(make_float2(r3.x, r3.y), make_float2(r3.z, r3.w))));
+                    }
+                    return q.x + q.y;
+                };
+                float S = slot_sum(red + sn * 2 * kNSL);
+                float Sw = T2 ? slot_sum(red + sn * 2 * kNSL + kNSL) : 0.f;
                 if (CL == 2) {
-                    // this CTA's partial sum to both CTAs; the peer's arrives on xbar[sn] (its
+                    // this CTA's partial sums to both CTAs; the peer's arrive on xbar[sn] (its
                     // phase flips every second step); both add in rank order: identical bits
+                    float* xq = xs + sn * 4;  // [theta1, theta2][rank]
                     if (lane == 0) {
-                        xs[sn * 2 + crank] = S;
-                        st_peer_f32(peer_addr(xs + sn * 2 + crank, crank ^ 1u), S);
+                        xq[crank] = S;
+                        st_peer_f32(peer_addr(xq + crank, crank ^ 1u), S);
+                        if (T2) {
+                            xq[2 + crank] = Sw;
+                            st_peer_f32(peer_addr(xq + 2 + crank, crank ^ 1u), Sw);
+                        }
                         mbar_arrive_peer(peer_addr(xbar + sn, crank ^ 1u));
                         mbar_wait_cluster(xbar + sn, ((g0 + (uint32_t)idx) >> 1) & 1u);
                     }
                     __syncwarp();
-                    S = xs[sn * 2] + xs[sn * 2 + 1];
+                    S = xq[0] + xq[1];
+                    if (T2) Sw = xq[2] + xq[3];
+                }
+                if (T2) {  // theta2 of this voxel, stored for the later iterations
+                    theta2 = U8 ? scale * scale * Sw : Sw;
+                    den = theta2 + 2.f * ps;
+                    c1 = theta2 * pp.v + 2.f * psx;
+                    rden = den > 0.f ? __fdividef(1.f, den) : 0.f;
+                    if (lane == 0 && crank == 0) P.theta2[((size_t)z * P.nsv + sv) * S2 + list[idx]] = theta2;
                 }
                 const float theta1 = -scale * S;  // Alg1:5
                 float u = pp.v;
@@ -979,7 +1004,11 @@ template <int VPT, bool U8, int NNB, int CL>
 cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
 {
     constexpr int R = ring_depth(U8);
-    auto kern = p.tprof ? k_svicd<VPT, U8, NNB, R, CL, true> : k_svicd<VPT, U8, NNB, R, CL, false>;
+    // the phase profile (development aid) is built for the production variant only
+    constexpr bool kProf = VPT == MBIR_WIDE_VPT && U8 && CL == 1;
+    auto kern = p.theta2_pass ? k_svicd<VPT, U8, NNB, R, CL, true, false>
+                : (kProf && p.tprof) ? k_svicd<VPT, U8, NNB, R, CL, false, kProf>
+                                     : k_svicd<VPT, U8, NNB, R, CL, false, false>;
     IcdParams q = p;
     q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT, p.V, CL);
     const int smem = q.lay.total;
@@ -1010,7 +1039,7 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
 template <int VPT, bool U8, int NNB, int CL>
 int resident_t(const IcdParams& p)
 {
-    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), CL, false>;
+    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), CL, false, false>;
     const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT, p.V, CL).total;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
     cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
@@ -1038,25 +1067,19 @@ int resident_t(const IcdParams& p)
     return ncl * CL;
 }
 
+// vpt: 1 (nviews <= 128) or MBIR_WIDE_VPT; cl: 1, or 2 (wide VPT only)
 #define SVICD_DISPATCH(FN, ...)                                                                      \
+    constexpr int W = MBIR_WIDE_VPT;                                                                 \
     if (cl == 2) {                                                                                   \
-        if (quantize) return nnb == 26 ? FN<4, true, 26, 2>(__VA_ARGS__) : FN<4, true, 8, 2>(__VA_ARGS__); \
-        return nnb == 26 ? FN<4, false, 26, 2>(__VA_ARGS__) : FN<4, false, 8, 2>(__VA_ARGS__);       \
-    }                                                                                                \
-    if (vpt == 3) {                                                                                  \
-        if (quantize) return nnb == 26 ? FN<3, true, 26, 1>(__VA_ARGS__) : FN<3, true, 8, 1>(__VA_ARGS__); \
-        return nnb == 26 ? FN<3, false, 26, 1>(__VA_ARGS__) : FN<3, false, 8, 1>(__VA_ARGS__);       \
-    }                                                                                                \
-    if (vpt == 2) {                                                                                  \
-        if (quantize) return nnb == 26 ? FN<2, true, 26, 1>(__VA_ARGS__) : FN<2, true, 8, 1>(__VA_ARGS__); \
-        return nnb == 26 ? FN<2, false, 26, 1>(__VA_ARGS__) : FN<2, false, 8, 1>(__VA_ARGS__);       \
+        if (quantize) return nnb == 26 ? FN<W, true, 26, 2>(__VA_ARGS__) : FN<W, true, 8, 2>(__VA_ARGS__); \
+        return nnb == 26 ? FN<W, false, 26, 2>(__VA_ARGS__) : FN<W, false, 8, 2>(__VA_ARGS__);       \
     }                                                                                                \
     if (vpt == 1) {                                                                                  \
         if (quantize) return nnb == 26 ? FN<1, true, 26, 1>(__VA_ARGS__) : FN<1, true, 8, 1>(__VA_ARGS__); \
         return nnb == 26 ? FN<1, false, 26, 1>(__VA_ARGS__) : FN<1, false, 8, 1>(__VA_ARGS__);       \
     }                                                                                                \
-    if (quantize) return nnb == 26 ? FN<4, true, 26, 1>(__VA_ARGS__) : FN<4, true, 8, 1>(__VA_ARGS__); \
-    return nnb == 26 ? FN<4, false, 26, 1>(__VA_ARGS__) : FN<4, false, 8, 1>(__VA_ARGS__);
+    if (quantize) return nnb == 26 ? FN<W, true, 26, 1>(__VA_ARGS__) : FN<W, true, 8, 1>(__VA_ARGS__); \
+    return nnb == 26 ? FN<W, false, 26, 1>(__VA_ARGS__) : FN<W, false, 8, 1>(__VA_ARGS__);
 
 }  // namespace
 

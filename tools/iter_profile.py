@@ -28,14 +28,20 @@ g = M.Geometry(cfg.n, cfg.n, cfg.nz, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dch
 r = M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=cfg.nbhd),
                     M.Options(sv_side=a.sv_side or cfg.sv_side, zero_skip=a.zero_skip,
                               batch_svs=a.batch_svs, cluster=a.cluster, quantize_A=a.quantize))
-r.set_sinogram(y, w)
+import time  # noqa: E402
+for k in range(2):
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    r.set_sinogram(y, w)
+    torch.cuda.synchronize()
+    print(f"set_sinogram {k} {(time.perf_counter() - t0) * 1e3:.2f} ms")
 print(json.dumps(r.sizes()))
 for rep in range(2):
     r.set_image(None)
     for it in range(a.iters):
         s = r.iterate(1)
-        if rep == 1:
-            print(f"iter {it + 1:3d} upd {s['updates']:10d} skip {s['skipped']:10d} visits {s['sv_visits']:7d} "
+        if rep == 1 or it == 0:
+            print(f"{'iter' if rep else 'first'} {it + 1:3d} upd {s['updates']:10d} skip {s['skipped']:10d} visits {s['sv_visits']:7d} "
                   f"t {s['seconds'] * 1e3:8.2f} ms  kernel {s['kernel_seconds'] * 1e3:8.2f} ms  "
                   f"ns/upd {1e9 * s['kernel_seconds'] / max(s['updates'], 1):7.2f}  "
                   f"us/visit {1e6 * s['kernel_seconds'] / max(s['sv_visits'], 1) * 148:8.2f}")
