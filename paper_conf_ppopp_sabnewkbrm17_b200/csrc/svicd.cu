@@ -12,19 +12,21 @@
 //     with a row length that is a multiple of 32 views, so a warp's 32 lanes hit 32 distinct
 //     banks for any per-view offsets: conflict-free gathers and scatters, no atomics (a thread is
 //     the only writer of its views).
-//   * the DELTA warp derives the two deltas of each voxel pair (Alg1:7-8, q-GGMRF surrogate,
-//     reading R1) from the view warps' partial sums and the surrogate terms;
-//   * the PRIOR warp computes the next pair's surrogate terms from the shared-memory x tile while
-//     the current pair is in flight.
-// Voxels of the SV are updated in a random order exactly as sequential ICD, two per step: both
-// voxels' theta1 partials are gathered from the same e together with their overlap
-// H = sum w A_b A_a; the delta warp corrects b's theta1 by a's change (theta1_b' = theta1_b +
-// s_b s_a delta_a H) and b's prior if a is its neighbour.  A view thread keeps the pair's
-// dequantised A values, w*A and e in registers from preparation through gather to scatter (no
-// recomputation), and prepares the next pair while the deltas are derived.  A records (uint8
-// codes + band offsets) are streamed R voxels ahead by per-thread cp.async.  theta2 = A^T W A is
-// precomputed per (slice, voxel).  The write-back is delta e = final - e_init per aligned band
-// window with red.global.add.v4.f32 (same-colour SVs share sinogram entries).
+//   * the DELTA warp derives each voxel's delta (Alg1:7-8, q-GGMRF surrogate, reading R1) from
+//     the view warps' partial sums and the surrogate terms, and writes the new value into the
+//     shared-memory x tile;
+//   * the PRIOR warp computes the next voxel's surrogate terms from the x tile (one neighbour per
+//     lane) while the current voxel is in flight, with the previous voxel's OLD value; the delta
+//     warp replaces that one neighbour's term once the new value is known (exact).
+// Voxels of the SV are updated in a random order exactly as sequential ICD, one per step: the
+// view warps gather theta1's partials of voxel i from e (holding voxel i - 1's scatter), prepare
+// voxel i + 1 (A record from the cp.async ring, dequantised; w*A in registers) while the delta
+// is derived, then scatter voxel i into their own views.  A records (uint8 codes + band offsets)
+// are streamed R voxels ahead by per-thread cp.async.  theta2 = A^T W A is stored per (slice,
+// voxel); the first iteration after new weights reduces it here (T2) alongside theta1.  The
+// write-back is delta e = final - e_init per aligned band window with red.global.add.v4.f32
+// (same-colour SVs share sinogram entries).  The next task's inputs are prepared
+// while the current one runs.
 #include "mbir_internal.h"
 
 namespace mbir {
@@ -219,7 +221,7 @@ constexpr int kStg = 36;
 // from one address
 __host__ __device__ constexpr int svb_cols(int vpt, int cl = 1) { return (vpt == 1 ? 128 : 768) / cl; }
 
-constexpr int kNSL = 16;  // partial-sum slots per quantity in the pair exchange (>= view warps)
+constexpr int kNSL = 16;  // partial-sum slots per quantity and step (>= view warps)
 
 // the pack and the write-back move 32-view tiles; tile warp w (< VA / 128: the record stride VA
 // is a multiple of 128) handles tiles 4w ... 4w + 3 whatever the voxel loop's view ownership
@@ -231,10 +233,10 @@ __host__ __device__ constexpr int tile_warps(int va) { return va / (32 * kTileW)
 // + the delta and prior warps
 __host__ __device__ constexpr int max_threads(int vpt) { return vpt == 2 ? 448 : vpt == 3 ? 320 : 256; }
 
-// named barriers of the pair protocol (0 is __syncthreads)
+// named barriers of the voxel-loop protocol (0 is __syncthreads)
 constexpr int kBarA = 1;  // the view warps' theta1 partials of a voxel are ready
-constexpr int kBarB = 2;  // the delta warp has published the pair's deltas
-constexpr int kBarX = 3;  // the delta warp has written the pair's new values into the x tile
+constexpr int kBarB = 2;  // the delta warp has published the voxel's delta
+constexpr int kBarX = 3;  // the delta warp has written the previous voxel's new value into the x tile
 constexpr int kBarP = 4;  // task preparation steps (delta + prior warps)
 constexpr int kBarT = 5;  // the prior warp's surrogate terms of a voxel are ready
 
@@ -997,7 +999,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
 }
 
 // A-record ring depth (voxels of cp.async lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
-// (the pair loop needs >= 4: the current pair's two stages plus the next pair's two)
+// (>= 2: the loop holds the current voxel's stage and the next voxel's)
 constexpr int ring_depth(bool u8) { return u8 ? 12 : 4; }
 
 template <int VPT, bool U8, int NNB, int CL>
