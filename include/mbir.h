@@ -104,6 +104,13 @@ typedef struct mbir_options {
                               frozen at 0 are re-examined and the fixed point stays the MAP
                               estimate; 0 = the plain heuristic of P:115, whose fixed point can
                               differ from the MAP (reading R9).  Default 4                      */
+    int voxels_per_step;   /* voxels of one SV updated concurrently by the update kernel (the
+                              paper's intra-SV parallelism): 1 = exact sequential
+                              ICD inside the SV (one voxel per step); 2 = voxel pairs: both
+                              voxels' theta1, theta2 and prior terms from the same e and x (the
+                              second does not see the first's update), then both applied; needs
+                              uint8 A and one CTA per task (else EINVAL).  0 = auto = 1 (pairs
+                              measured 5 % slower on the bench workload) */
 } mbir_options;
 
 /* Placement and (optional) multi-GPU slab partition.  device: CUDA ordinal.  stream: a
@@ -152,10 +159,12 @@ typedef struct mbir_sizes {
     int64_t a_bytes;                /* device bytes of the compressed A                   */
     int64_t band_entries;           /* sum over (SV, view) of band widths                  */
     int max_group;                  /* SVs of one checkerboard colour per slice (max)     */
+    int voxels_per_step;            /* update-kernel voxels per SV step in effect (1, 2)  */
 } mbir_sizes;
 
 /* Fill defaults: sv_side 9, sv_fraction 0.25, batch_svs 0, batch_threshold -1, zero_skip 1,
- * quantize_A 1, seed 3000, deterministic 0, cluster 0 (auto), zero_skip_period 4. */
+ * quantize_A 1, seed 3000, deterministic 0, cluster 0 (auto), zero_skip_period 4,
+ * voxels_per_step 0 (auto). */
 void mbir_default_options(mbir_options* o);
 /* p 1.2, q 2, T 1, sigma 0.005, neighborhood 26, positivity 1. */
 void mbir_default_prior(mbir_prior* p);
@@ -241,13 +250,17 @@ int mbir_link_slabs(mbir_handle** handles, int n);
 
 /* Test hook: record every voxel update the fused update kernel executes from now on -- the
  * (theta1, theta2, delta) of Alg. 1 steps 3-8 exactly as the kernel's delta chain
- * used them (theta1 of the second voxel of a pair includes the first one's update of e, so it
- * equals sequential ICD's theta1 at that update).  capacity = entries kept (0 = off; frees the
- * buffer).  Pairs are recorded first voxel first; in deterministic mode (one CTA) the record
- * is the exact update sequence.  Errors: EINVAL, ENOMEM. */
+ * used them.  capacity = entries kept (0 = off; frees the buffer).  With voxel pairs
+ * (voxels_per_step 2) both updates of a pair are computed from the same state: the second is
+ * recorded right after the first with MBIR_DUMP_SAME_STATE set in its voxel index.  In
+ * deterministic mode (one CTA) the record is the exact update sequence.  Errors: EINVAL,
+ * ENOMEM. */
 int mbir_set_update_dump(mbir_handle* h, int64_t capacity);
 
-/* Copy up to cap recorded updates into host arrays (voxels: local flat (z*ny + y)*nx + x;
+#define MBIR_DUMP_SAME_STATE ((int64_t)1 << 62) /* update record flag (mbir_set_update_dump) */
+
+/* Copy up to cap recorded updates into host arrays (voxels: local flat (z*ny + y)*nx + x,
+ * | MBIR_DUMP_SAME_STATE for the second update of a pair;
  * theta1, theta2, delta float32), set *n to the number recorded since the last call (which
  * can exceed cap and the capacity: then the record was truncated), and restart the record.
  * Errors: EINVAL, ESTATE (no dump buffer), ECUDA. */

@@ -5,6 +5,7 @@ See include/mbir.h for the contract and DESIGN.md for the design.  Building:
 ``python -c "import __graft_entry__ as g; g.build()"`` (or ``make -C csrc``).
 """
 from .api import (  # noqa: F401
+    DUMP_SAME_STATE,
     Geometry,
     Options,
     Prior,

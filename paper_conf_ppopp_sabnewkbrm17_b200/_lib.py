@@ -54,7 +54,7 @@ class mbir_options(C.Structure):
         ("sv_side", C.c_int), ("sv_fraction", C.c_double), ("batch_svs", C.c_int),
         ("batch_threshold", C.c_int), ("zero_skip", C.c_int), ("quantize_A", C.c_int),
         ("seed", C.c_uint64), ("deterministic", C.c_int), ("cluster", C.c_int),
-        ("zero_skip_period", C.c_int),
+        ("zero_skip_period", C.c_int), ("voxels_per_step", C.c_int),
     ]
 
 
@@ -80,7 +80,7 @@ class mbir_sizes(C.Structure):
         ("nsv_x", C.c_int), ("nsv_y", C.c_int), ("nsv", C.c_int), ("K", C.c_int),
         ("band_max", C.c_int), ("svb_rows", C.c_int), ("threads_per_cta", C.c_int), ("cluster", C.c_int), ("resident_ctas", C.c_int),
         ("smem_bytes", C.c_int), ("nnz", C.c_int64), ("a_bytes", C.c_int64),
-        ("band_entries", C.c_int64), ("max_group", C.c_int),
+        ("band_entries", C.c_int64), ("max_group", C.c_int), ("voxels_per_step", C.c_int),
     ]
 
     def as_dict(self):

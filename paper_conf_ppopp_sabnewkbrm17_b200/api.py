@@ -74,11 +74,13 @@ class Options:
     deterministic: int = 0
     cluster: int = 0  # update-kernel CTAs per SV task: 0 (auto) = 1, or 2 (a cluster splits the views)
     zero_skip_period: int = 4  # every n-th iteration without zero-skip (reading R9); 0 = never
+    voxels_per_step: int = 0  # voxels of an SV per kernel step: 0 auto (= 1), 1, or 2 (voxel pairs)
 
     def c(self) -> L.mbir_options:
         return L.mbir_options(self.sv_side, self.sv_fraction, self.batch_svs,
                               self.batch_threshold, self.zero_skip, self.quantize_A, self.seed,
-                              self.deterministic, self.cluster, self.zero_skip_period)
+                              self.deterministic, self.cluster, self.zero_skip_period,
+                              self.voxels_per_step)
 
 
 def _buf(a, n: int | None = None, dtype=np.float32, writable=False):
@@ -258,8 +260,12 @@ def mbir_set_update_dump(h, capacity: int):
     L.check(L.load().mbir_set_update_dump(h, int(capacity)), h, "mbir_set_update_dump")
 
 
+DUMP_SAME_STATE = 1 << 62  # MBIR_DUMP_SAME_STATE: computed from the same state as the previous record
+
+
 def mbir_get_update_dump(h, cap: int):
-    """Returns (voxels int64, theta1, theta2, delta float32, n_recorded)."""
+    """Returns (voxels int64 (| DUMP_SAME_STATE for a pair's second update), theta1, theta2,
+    delta float32, n_recorded)."""
     vox = np.empty(cap, np.int64)
     t1 = np.empty(cap, np.float32)
     t2 = np.empty(cap, np.float32)

@@ -110,6 +110,7 @@ struct mbir_handle {
     int rows = 0, band_max = 0;
     int vpt = 1, nvw = 0, Vs = 0, threads = 0, smem = 0, blocks_per_sm = 1, nsm = 148;
     int cl = 1;  // update-kernel CTAs per SV task (2: thread-block cluster splitting the views)
+    int kv = 1;  // voxels per step of the update kernel (2: voxel pairs)
     int resident = 0;  // update-kernel CTAs resident on the device at once (occupancy query)
     int max_group = 0;
     DevA A{};
@@ -198,6 +199,7 @@ IcdParams make_params(mbir_handle* h)
     p.seed = h->o.seed;
     p.iter = h->iter;
     p.deterministic = h->o.deterministic;
+    p.kv = h->kv;
     p.tprof = h->d_tprof;
     p.pc = h->pc;
     p.dump = h->d_dump;
@@ -501,6 +503,7 @@ void mbir_default_options(mbir_options* o)
     o->deterministic = 0;
     o->cluster = 0;
     o->zero_skip_period = 4;
+    o->voxels_per_step = 0;
 }
 
 void mbir_default_prior(mbir_prior* p)
@@ -757,6 +760,11 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         h->cl = h->o.cluster == 2 ? 2 : 1;
         if (h->cl == 2 && !(h->vpt == 4 && h->nvw % 2 == 0))
             return (fail(h, MBIR_EINVAL, "cluster = 2 needs > 128 views in an even number of 128-view warps"), bail(MBIR_EINVAL));
+        if (h->o.voxels_per_step < 0 || h->o.voxels_per_step > 2)
+            return (fail(h, MBIR_EINVAL, "voxels_per_step must be 0 (auto), 1 or 2"), bail(MBIR_EINVAL));
+        if (h->o.voxels_per_step == 2 && (h->cl == 2 || !quant))
+            return (fail(h, MBIR_EINVAL, "voxels_per_step = 2 needs uint8 A (quantize_A) and one CTA per task"), bail(MBIR_EINVAL));
+        h->kv = h->o.voxels_per_step ? h->o.voxels_per_step : 1;  // auto: exact steps (pairs measured slower)
         h->threads = 32 * (h->nvw / h->cl + 2);
         h->smem = svicd_smem_bytes(p, h->vpt, P.neighborhood, quant, h->cl);
         if (h->smem > (int)prop.sharedMemPerBlockOptin)
@@ -1033,6 +1041,7 @@ int mbir_query_sizes(const mbir_handle* h, mbir_sizes* s)
     s->a_bytes = h->a_bytes;
     s->band_entries = h->band_entries;
     s->max_group = h->max_group;
+    s->voxels_per_step = h->kv;
     return MBIR_OK;
 }
 
@@ -1142,7 +1151,8 @@ int mbir_get_update_dump(mbir_handle* h, int64_t cap, int64_t* voxels, float* th
     for (int64_t i = 0; i < m; ++i) {
         uint32_t v;
         memcpy(&v, &buf[4 * i], 4);
-        voxels[i] = (int64_t)v;
+        // bit 31: the update was computed from the same state as the record before it (pairs)
+        voxels[i] = (int64_t)(v & 0x7fffffffu) | ((v >> 31) ? MBIR_DUMP_SAME_STATE : 0);
         theta1[i] = buf[4 * i + 1];
         theta2[i] = buf[4 * i + 2];
         delta[i] = buf[4 * i + 3];

@@ -94,6 +94,7 @@ struct IcdParams {
     uint64_t seed;
     int iter;
     int zero_skip_active;
+    int kv;           // voxels per step (1: exact sequential within the SV, 2: voxel pairs)
     int theta2_pass;  // this launch reduces theta2 (Alg1:6) with theta1 and stores it (iteration 1)
     int deterministic;
     unsigned long long* tprof;  // optional [8] phase cycle counters (env MBIR_PHASE_PROFILE)

@@ -170,18 +170,21 @@ struct NbrOne {
     float w;
 };
 
-// surrogate terms of voxel i of the visiting order, computed from the x tile in which every update
-// before voxel i - 1 is applied and voxel i - 1 still has its OLD value: the sums
-// s = sum_r b_r phi(v - x_r), sx = sum_r b_r phi(v - x_r) x_r (Alg1:7, reading R1; free boundary),
-// v = x_i, and -- if voxel i - 1 is a neighbour of i -- that neighbour's term (btu) and weight
-// (bwu), which the delta warp replaces by the term at i - 1's new value: exact sequential ICD
+// surrogate terms of voxel i of the visiting order, computed from the x tile in which the voxels
+// of the previous step (voxel ip0 = i - 1, or with voxel pairs the previous pair ip0, ip1) still
+// have their OLD values and every earlier update is applied: the sums s = sum_r b_r phi(v - x_r),
+// sx = sum_r b_r phi(v - x_r) x_r (Alg1:7, reading R1; free boundary), v = x_i, and for each such
+// previous voxel that is a neighbour of i its term (btu) and weight (bwu), which the delta warp
+// replaces by the term at the new value: exact.  (With pairs, the other voxel of i's own pair
+// keeps its old value: both are computed from the same state.)
 struct PriTerm {
-    float s, sx, v, btu, bwu;
+    float s, sx, v, btu0, bwu0, btu1, bwu1;
 };
 
-__device__ __forceinline__ void prior_one(const int* tof, int i, const float* xt, int cslot, int TW, int gx0,
-                                          int gy0, int zg, const IcdParams& P, const NbrOne& nb, int lane,
-                                          PriTerm* out)
+template <int NP>  // previous-step voxels to report (1, or 2 with voxel pairs)
+__device__ __forceinline__ void prior_one(const int* tof, int i, int ip0, int ip1, const float* xt, int cslot,
+                                          int TW, int gx0, int gy0, int zg, const IcdParams& P, const NbrOne& nb,
+                                          int lane, PriTerm* out)
 {
     const int tv = tof[i];
     const int lx = tv & 255, ly = tv >> 8;
@@ -192,20 +195,47 @@ __device__ __forceinline__ void prior_one(const int* tof, int i, const float* xt
     const float xr = xt[c0 + nb.dt];  // always inside the tile (its ring covers the neighbourhood)
     const float bt = ok ? nb.w * phi_f(P.pc, v - xr) : 0.f;
     float s = bt, sx = bt * xr;
-    bool mine = false;
-    if (i > 0) {
-        const int tu = tof[i - 1];
-        mine = ok && nb.dz == 0 && nb.dx == (tu & 255) - lx && nb.dy == (tu >> 8) - ly;
+    bool m0 = false, m1 = false;
+    if (ip0 >= 0) {
+        const int tu = tof[ip0];
+        m0 = ok && nb.dz == 0 && nb.dx == (tu & 255) - lx && nb.dy == (tu >> 8) - ly;
+    }
+    if (NP == 2 && ip1 >= 0) {
+        const int tu = tof[ip1];
+        m1 = ok && nb.dz == 0 && nb.dx == (tu & 255) - lx && nb.dy == (tu >> 8) - ly;
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         s += __shfl_xor_sync(kFull, s, o);
         sx += __shfl_xor_sync(kFull, sx, o);
     }
-    const unsigned who = __ballot_sync(kFull, mine);
-    const int src = who ? __ffs(who) - 1 : 0;
-    const float btu = __shfl_sync(kFull, bt, src), bwu = __shfl_sync(kFull, nb.w, src);
-    if (lane == 0) *out = PriTerm{s, sx, v, who ? btu : 0.f, who ? bwu : 0.f};
+    const unsigned w0 = __ballot_sync(kFull, m0);
+    const int src0 = w0 ? __ffs(w0) - 1 : 0;
+    const float btu0 = __shfl_sync(kFull, bt, src0), bwu0 = __shfl_sync(kFull, nb.w, src0);
+    float btu1 = 0.f, bwu1 = 0.f;
+    if (NP == 2) {
+        const unsigned w1 = __ballot_sync(kFull, m1);
+        const int src1 = w1 ? __ffs(w1) - 1 : 0;
+        btu1 = __shfl_sync(kFull, bt, src1);
+        bwu1 = __shfl_sync(kFull, nb.w, src1);
+        if (!w1) btu1 = bwu1 = 0.f;
+    }
+    if (lane == 0) *out = PriTerm{s, sx, v, w0 ? btu0 : 0.f, w0 ? bwu0 : 0.f, btu1, bwu1};
+}
+
+// sum of the view warps' partials (slots) in a fixed tree order (<= 8 or 16 slots)
+template <bool N8>
+__device__ __forceinline__ float slot_sum(const float* rq)
+{
+    const float4 r0 = *(const float4*)rq, r1 = *(const float4*)(rq + 4);
+    float2 q = __fadd2_rn(__fadd2_rn(make_float2(r0.x, r0.y), make_float2(r0.z, r0.w)),
+                          __fadd2_rn(make_float2(r1.x, r1.y), make_float2(r1.z, r1.w)));
+    if (!N8) {
+        const float4 r2 = *(const float4*)(rq + 8), r3 = *(const float4*)(rq + 12);
+        q = __fadd2_rn(q, __fadd2_rn(__fadd2_rn(make_float2(r2.x, r2.y), make_float2(r2.z, r2.w)),
+                                     __fadd2_rn(make_float2(r3.x, r3.y), make_float2(r3.z, r3.w))));
+    }
+    return q.x + q.y;
 }
 
 __host__ __device__ inline int align16(int b) { return (b + 15) & ~15; }
@@ -255,8 +285,8 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     L.list = o;  o = align16(o + 2 * S2 * 4);
     L.flags = o; o = align16(o + S2 * 4);
     L.tof = o;   o = align16(o + 2 * S2 * 4);
-    L.red = o;   o = align16(o + 2 * 2 * kNSL * 4);  // [2 steps][theta1, theta2][kNSL view warps] partials
-    L.pri = o;   o = align16(o + 2 * (int)sizeof(PriTerm));
+    L.red = o;   o = align16(o + 2 * 2 * 2 * kNSL * 4);  // [2 steps][2 voxels][theta1, theta2][kNSL view warps]
+    L.pri = o;   o = align16(o + 2 * 2 * (int)sizeof(PriTerm));  // [2 steps][2 voxels]
     L.vscale = o; o = align16(o + 2 * S2 * 4);
     L.vth2 = o;  o = align16(o + 2 * S2 * 4);
     L.misc = o;  o = align16(o + 16 * 4);
@@ -329,10 +359,11 @@ __device__ __forceinline__ void load_words(const unsigned char* stg, int off_in_
 }
 
 // The update kernel.  VPT views per lane (4, or 1 for <= 128 views), uint8 or fp32 A, 8 or 26
-// neighbours, R-voxel A-record ring; PROF adds per-phase cycle counters.
+// neighbours, R-voxel A-record ring, CL CTAs per task, KV voxels per step (1: exact sequential
+// ICD within the SV; 2: voxel pairs from the same state); PROF adds per-phase cycle counters.
 // T2: the theta2 pass -- theta2 = sum w A^2 (Alg1:6) is not precomputed yet: the view warps reduce
 // it with theta1 in this iteration (which visits every voxel) and the delta warp stores it
-template <int VPT, bool U8, int NNB, int R, int CL, bool T2, bool PROF>
+template <int VPT, bool U8, int NNB, int R, int CL, int KV, bool T2, bool PROF>
 __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
@@ -356,7 +387,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     unsigned char* astage = smem + L.astage;
     float* stg_w = (float*)(smem + L.staging) + vw * 32 * kStg;
     int* s_task = (int*)(smem + L.misc);            // [b]: the task prepared in buffer b, [2 + b]: its kept voxels
-    float* dslot = (float*)(smem + L.misc) + 4;     // [2 steps]: scale * delta of the step's voxel
+    float* dslot = (float*)(smem + L.misc) + 4;     // [2 steps][2 voxels]: scale * delta of the step's voxels
     uint32_t* binfo = (uint32_t*)(smem + L.binfo);  // [2][VA], indexed by (global) view
     float* xs = (float*)(smem + L.cx);               // CL = 2: [2 steps][2 quantities][2 ranks] partial sums
     uint64_t* xbar = (uint64_t*)(smem + L.cx + 32);  // CL = 2: [2 steps] the peer's partials arrived
@@ -368,7 +399,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     const int nab = (nvw + 1) * 32;      // barrier A: view warps + the delta warp
     const int nb2 = (nvw + 1) * 32;      // barrier B: view warps + the delta warp
 
-    for (int i = threadIdx.x; i < 2 * 2 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
+    for (int i = threadIdx.x; i < 2 * 2 * 2 * kNSL; i += blockDim.x) red[i] = 0.f;  // slots >= nvw stay 0
     // the neighbourhood (reading R2) as shared-memory tables [dx | dy | dz | weight bits][32]: a
     // by-value kernel parameter indexed by a run-time value would be copied to local memory
     int* nbt = (int*)(smem + L.mbar);
@@ -624,7 +655,12 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         // the first voxel's surrogate terms (prior warp) and the next task's input copies (delta
         // warp) while the view warps pack
         if (is_prior) {
-            prior_one(tof, 0, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + (gseq & 1));
+            if (KV == 1) {
+                prior_one<1>(tof, 0, -1, -1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + 2 * (gseq & 1));
+            } else {  // pair 0: both from the same state
+                prior_one<2>(tof, 0, -1, -1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri);
+                if (nactv > 1) prior_one<2>(tof, 1, -1, -1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + 1);
+            }
             __syncwarp();
         } else if (is_delta) {
             fetch_and_copy(cb ^ 1);
@@ -771,8 +807,8 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                         if (T2) g2 += __shfl_xor_sync(kFull, g2, o);
                     }
                     if (lane == 0) {
-                        red[sn * 2 * kNSL + vw] = g;
-                        if (T2) red[sn * 2 * kNSL + kNSL + vw] = g2;
+                        red[sn * 4 * kNSL + vw] = g;
+                        if (T2) red[sn * 4 * kNSL + kNSL + vw] = g2;
                     }
                 }
                 bar_arrive(kBarA, nab);
@@ -782,7 +818,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 refill(idx + 1, nxt.sj);
                 bar_sync(kBarB, nb2);
                 // Alg1:9-11 on this thread's views
-                const float sd = dslot[sn];
+                const float sd = dslot[2 * sn];
                 if (sd != 0.f) {
                     const float2 nd = make_float2(-sd, -sd);
 #pragma unroll
@@ -799,15 +835,231 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             };
             // the first R records (the ring region held the pack's staging tiles until the barrier)
             for (int i = 0; i < R; ++i) copy_record_to(i, (sbase + i) % R, i < nactv ? list[i] : 0);
-            VoxState st0, st1;
-            st0.sj = sbase;
-            prep(st0);
-            refill(0, sbase);
-            for (int idx = 0; idx < nactv; idx += 2) {
-                step(idx, st0, st1);
-                if (idx + 1 < nactv) step(idx + 1, st1, st0);
+            if constexpr (KV == 1) {
+                VoxState st0, st1;
+                st0.sj = sbase;
+                prep(st0);
+                refill(0, sbase);
+                for (int idx = 0; idx < nactv; idx += 2) {
+                    step(idx, st0, st1);
+                    if (idx + 1 < nactv) step(idx + 1, st1, st0);
+                }
+            } else {
+                // ---- voxel pairs (intra-SV parallelism): step s updates voxels
+                //      2s and 2s + 1 from the same e and x (Jacobi within the pair); the second
+                //      voxel's scatter re-reads the rows the first one's may have changed
+                auto prep_j = [&](int j, VoxState& vs) {
+                    vs.sj = (sbase + j) % R;
+                    if (j < nactv) {
+                        prep(vs);
+                    } else {  // past the visit's end: a null voxel (no loads, nothing scattered)
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t) {
+                            vs.p[t] = kv[t];
+                            vs.f[t][0] = vs.f[t][1] = vs.wf[t][0] = vs.wf[t][1] = make_float2(0.f, 0.f);
+                        }
+                    }
+                    refill(j, vs.sj);
+                };
+                auto pstep = [&](int s2, VoxState& ca, VoxState& cb, VoxState& na, VoxState& nb) {
+                    const int sn = s2 & 1;
+                    float2 eva[VPT][2], evb[VPT][2];
+                    {
+                        float2 aa = make_float2(0.f, 0.f), ab = make_float2(0.f, 0.f);
+                        float2 qa = make_float2(0.f, 0.f), qb = make_float2(0.f, 0.f);  // T2
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t) {
+                            const float* pa = sb + ca.p[t];
+                            const float* pb = sb + cb.p[t];
+                            eva[t][0] = make_float2(pa[0], pa[RS]);
+                            eva[t][1] = make_float2(pa[2 * RS], pa[3 * RS]);
+                            evb[t][0] = make_float2(pb[0], pb[RS]);
+                            evb[t][1] = make_float2(pb[2 * RS], pb[3 * RS]);
+                            aa = __ffma2_rn(ca.wf[t][0], eva[t][0], aa);
+                            ab = __ffma2_rn(cb.wf[t][0], evb[t][0], ab);
+                            aa = __ffma2_rn(ca.wf[t][1], eva[t][1], aa);
+                            ab = __ffma2_rn(cb.wf[t][1], evb[t][1], ab);
+                            if (T2) {
+                                qa = __ffma2_rn(ca.wf[t][0], ca.f[t][0], qa);
+                                qb = __ffma2_rn(cb.wf[t][0], cb.f[t][0], qb);
+                                qa = __ffma2_rn(ca.wf[t][1], ca.f[t][1], qa);
+                                qb = __ffma2_rn(cb.wf[t][1], cb.f[t][1], qb);
+                            }
+                        }
+                        float ga = aa.x + aa.y, gb = ab.x + ab.y, g2a = qa.x + qa.y, g2b = qb.x + qb.y;
+#pragma unroll
+                        for (int o = 16; o > 0; o >>= 1) {
+                            ga += __shfl_xor_sync(kFull, ga, o);
+                            gb += __shfl_xor_sync(kFull, gb, o);
+                            if (T2) {
+                                g2a += __shfl_xor_sync(kFull, g2a, o);
+                                g2b += __shfl_xor_sync(kFull, g2b, o);
+                            }
+                        }
+                        if (lane == 0) {  // red[step][voxel][theta1, theta2][slot]
+                            red[(4 * sn + 0) * kNSL + vw] = ga;
+                            red[(4 * sn + 2) * kNSL + vw] = gb;
+                            if (T2) {
+                                red[(4 * sn + 1) * kNSL + vw] = g2a;
+                                red[(4 * sn + 3) * kNSL + vw] = g2b;
+                            }
+                        }
+                    }
+                    bar_arrive(kBarA, nab);
+                    // meanwhile: the next pair's e-independent state
+                    prep_j(2 * s2 + 2, na);
+                    prep_j(2 * s2 + 3, nb);
+                    bar_sync(kBarB, nb2);
+                    // Alg1:9-11 on this thread's views: voxel a from its gathered values, then
+                    // voxel b on the current e (a's scatter may have changed rows b reads)
+                    const float sda = dslot[2 * sn], sdb = dslot[2 * sn + 1];
+                    if (sda != 0.f) {
+                        const float2 nd = make_float2(-sda, -sda);
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t) {
+                            float* pe = sb + ca.p[t];
+                            const float2 a0 = __ffma2_rn(ca.f[t][0], nd, eva[t][0]);
+                            const float2 a1 = __ffma2_rn(ca.f[t][1], nd, eva[t][1]);
+                            pe[0] = a0.x;
+                            pe[RS] = a0.y;
+                            pe[2 * RS] = a1.x;
+                            pe[3 * RS] = a1.y;
+                        }
+                    }
+                    if (sdb != 0.f) {
+                        const float2 nd = make_float2(-sdb, -sdb);
+#pragma unroll
+                        for (int t = 0; t < VPT; ++t) {
+                            float* pe = sb + cb.p[t];
+                            if (sda != 0.f && abs(cb.p[t] - ca.p[t]) < 4 * RS) {  // rows overlap
+                                evb[t][0] = make_float2(pe[0], pe[RS]);
+                                evb[t][1] = make_float2(pe[2 * RS], pe[3 * RS]);
+                            }
+                            const float2 b0 = __ffma2_rn(cb.f[t][0], nd, evb[t][0]);
+                            const float2 b1 = __ffma2_rn(cb.f[t][1], nd, evb[t][1]);
+                            pe[0] = b0.x;
+                            pe[RS] = b0.y;
+                            pe[2 * RS] = b1.x;
+                            pe[3 * RS] = b1.y;
+                        }
+                    }
+                };
+                VoxState a0, b0, a1, b1;
+                prep_j(0, a0);
+                prep_j(1, b0);
+                const int nsteps = (nactv + 1) >> 1;
+                for (int s2 = 0; s2 < nsteps; s2 += 2) {
+                    pstep(s2, a0, b0, a1, b1);
+                    if (s2 + 1 < nsteps) pstep(s2 + 1, a1, b1, a0, b0);
+                }
             }
         } else if (is_delta) {
+          if constexpr (KV == 2) {
+            // ---- delta warp, voxel pairs: as below for both voxels of a step, from the same state
+            float upa = 0.f, vpa = 0.f, upb = 0.f, vpb = 0.f;  // the previous pair's new / old values
+            const int nsteps = (nactv + 1) >> 1;
+            auto put_x = [&](int i, float u) {
+                const int tu = tof[i];
+                xt[cslot + (tu >> 8) * TW + (tu & 255)] = u;
+            };
+            // voxel i's prior part with the previous pair's new values (terms reported by the prior warp)
+            auto prior_part = [&](const PriTerm& pp, float& ps, float& psx) {
+                ps = pp.s;
+                psx = pp.sx;
+                if (pp.bwu0 != 0.f) {
+                    const float bn = pp.bwu0 * phi_f(P.pc, pp.v - upa);
+                    ps += bn - pp.btu0;
+                    psx += bn * upa - pp.btu0 * vpa;
+                }
+                if (pp.bwu1 != 0.f) {
+                    const float bn = pp.bwu1 * phi_f(P.pc, pp.v - upb);
+                    ps += bn - pp.btu1;
+                    psx += bn * upb - pp.btu1 * vpb;
+                }
+            };
+            for (int s2 = 0; s2 < nsteps; ++s2) {
+                const int sn = s2 & 1;
+                const int ia = 2 * s2, ib = ia + 1;
+                const bool hb = ib < nactv;
+                bar_sync(kBarT, 64);
+                if (s2 > 0 && lane == 0) {  // the previous pair's new values (a full pair)
+                    put_x(ia - 2, upa);
+                    put_x(ia - 1, upb);
+                }
+                bar_arrive(kBarX, 64);
+                const PriTerm pa = pri[2 * sn], pb = pri[2 * sn + 1];
+                float psa, psxa, psb = 0.f, psxb = 0.f;
+                prior_part(pa, psa, psxa);
+                if (hb) prior_part(pb, psb, psxb);
+                const float sca = vscale[ia], scb = hb ? vscale[ib] : 0.f;
+                float t2a = T2 ? 0.f : vth2[ia], t2b = (T2 || !hb) ? 0.f : vth2[ib];
+                float dena = t2a + 2.f * psa, denb = t2b + 2.f * psb;
+                float c1a = t2a * pa.v + 2.f * psxa, c1b = t2b * pb.v + 2.f * psxb;
+                float ra = dena > 0.f ? __fdividef(1.f, dena) : 0.f, rb = denb > 0.f ? __fdividef(1.f, denb) : 0.f;
+                bar_sync(kBarA, nab);
+                const float Sa = slot_sum<kNSL8>(red + (4 * sn + 0) * kNSL);
+                const float Sb = slot_sum<kNSL8>(red + (4 * sn + 2) * kNSL);
+                if (T2) {  // theta2 of both voxels, stored for the later iterations
+                    const float wa = slot_sum<kNSL8>(red + (4 * sn + 1) * kNSL);
+                    const float wb = slot_sum<kNSL8>(red + (4 * sn + 3) * kNSL);
+                    t2a = U8 ? sca * sca * wa : wa;
+                    t2b = U8 ? scb * scb * wb : wb;
+                    dena = t2a + 2.f * psa;
+                    denb = t2b + 2.f * psb;
+                    c1a = t2a * pa.v + 2.f * psxa;
+                    c1b = t2b * pb.v + 2.f * psxb;
+                    ra = dena > 0.f ? __fdividef(1.f, dena) : 0.f;
+                    rb = denb > 0.f ? __fdividef(1.f, denb) : 0.f;
+                    if (lane == 0) {
+                        float* th = P.theta2 + ((size_t)z * P.nsv + sv) * S2;
+                        th[list[ia]] = t2a;
+                        if (hb) th[list[ib]] = t2b;
+                    }
+                }
+                // Alg1:5-8 for both voxels
+                const float th1a = -sca * Sa, th1b = -scb * Sb;
+                float ua = pa.v, ub = pb.v;
+                if (dena > 0.f) ua = (c1a - th1a) * ra;
+                if (denb > 0.f) ub = (c1b - th1b) * rb;
+                if (P.pc.positivity) {
+                    ua = fmaxf(ua, 0.f);
+                    ub = fmaxf(ub, 0.f);
+                }
+                const float da = ua - pa.v, db = hb ? ub - pb.v : 0.f;
+                if (lane == 0) {
+                    dslot[2 * sn] = sca * da;
+                    dslot[2 * sn + 1] = scb * db;
+                }
+                bar_arrive(kBarB, nb2);
+                upa = ua;
+                vpa = pa.v;
+                upb = ub;
+                vpb = pb.v;
+                if (lane == 0) {
+                    amount += fabsf(da) + fabsf(db);
+                    if (P.dump) {
+                        // test hook: both updates; the second carries bit 31 (computed from the
+                        // same state as the record before it)
+                        const int nrec = hb ? 2 : 1;
+                        const unsigned long long slot = atomicAdd(P.dump_count, (unsigned long long)nrec);
+                        for (int r = 0; r < nrec; ++r) {
+                            const int tv = tof[ia + r];
+                            const uint32_t vox = (uint32_t)(((size_t)z * P.ny + gy0 + (tv >> 8)) * P.nx + gx0 + (tv & 255)) |
+                                                 (r ? 0x80000000u : 0u);
+                            if (slot + r < (unsigned long long)P.dump_cap)
+                                *(float4*)(P.dump + 4 * (slot + r)) =
+                                    make_float4(__uint_as_float(vox), r ? th1b : th1a, r ? t2b : t2a, r ? db : da);
+                        }
+                    }
+                }
+            }
+            if (lane == 0) {  // the last pair's new values
+                const int ia = 2 * (nsteps - 1);
+                put_x(ia, upa);
+                if (ia + 1 < nactv) put_x(ia + 1, upb);
+            }
+            __syncwarp();
+          } else {
             // ---- delta warp (every lane computes the same values; lane 0 publishes).  The prior
             //      side of the update (voxel i - 1's neighbour correction, the numerator's and the
             //      denominator's prior terms, the reciprocal) is done as soon as the prior warp's
@@ -822,12 +1074,12 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                     xt[cslot + (tu >> 8) * TW + (tu & 255)] = u_prev;
                 }
                 bar_arrive(kBarX, 64);
-                const PriTerm pp = pri[sn];
+                const PriTerm pp = pri[2 * sn];
                 float ps = pp.s, psx = pp.sx;
-                if (pp.bwu != 0.f) {  // voxel i - 1 is a neighbour: its term at its new value
-                    const float bn = pp.bwu * phi_f(P.pc, pp.v - u_prev);
-                    ps += bn - pp.btu;
-                    psx += bn * u_prev - pp.btu * v_prev;
+                if (pp.bwu0 != 0.f) {  // voxel i - 1 is a neighbour: its term at its new value
+                    const float bn = pp.bwu0 * phi_f(P.pc, pp.v - u_prev);
+                    ps += bn - pp.btu0;
+                    psx += bn * u_prev - pp.btu0 * v_prev;
                 }
                 const float scale = vscale[idx];
                 float theta2 = T2 ? 0.f : vth2[idx];  // Alg1:6 (precomputed, or reduced below)
@@ -835,20 +1087,8 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 float c1 = theta2 * pp.v + 2.f * psx;  // numerator without -theta1
                 float rden = den > 0.f ? __fdividef(1.f, den) : 0.f;
                 bar_sync(kBarA, nab);
-                // sum of the view warps' partials in a fixed tree order (<= 8 or 16 slots)
-                auto slot_sum = [&](const float* rq) {
-                    const float4 r0 = *(const float4*)rq, r1 = *(const float4*)(rq + 4);
-                    float2 q = __fadd2_rn(__fadd2_rn(make_float2(r0.x, r0.y), make_float2(r0.z, r0.w)),
-                                          __fadd2_rn(make_float2(r1.x, r1.y), make_float2(r1.z, r1.w)));
-                    if (!kNSL8) {
-                        const float4 r2 = *(const float4*)(rq + 8), r3 = *(const float4*)(rq + 12);
-                        q = __fadd2_rn(q, __fadd2_rn(__fadd2_rn(make_float2(r2.x, r2.y), make_float2(r2.z, r2.w)),
-                                                     __fadd2_rn(make_float2(r3.x, r3.y), make_float2(r3.z, r3.w))));
-                    }
-                    return q.x + q.y;
-                };
-                float S = slot_sum(red + sn * 2 * kNSL);
-                float Sw = T2 ? slot_sum(red + sn * 2 * kNSL + kNSL) : 0.f;
+                float S = slot_sum<kNSL8>(red + sn * 4 * kNSL);
+                float Sw = T2 ? slot_sum<kNSL8>(red + sn * 4 * kNSL + kNSL) : 0.f;
                 if (CL == 2) {
                     // this CTA's partial sums to both CTAs; the peer's arrive on xbar[sn] (its
                     // phase flips every second step); both add in rank order: identical bits
@@ -879,7 +1119,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 if (den > 0.f) u = (c1 - theta1) * rden;
                 if (P.pc.positivity) u = fmaxf(u, 0.f);
                 const float d = u - pp.v;  // Alg1:7-8
-                if (lane == 0) dslot[sn] = scale * d;
+                if (lane == 0) dslot[2 * sn] = scale * d;
                 bar_arrive(kBarB, nb2);
                 u_prev = u;
                 v_prev = pp.v;
@@ -901,6 +1141,24 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 xt[cslot + (tu >> 8) * TW + (tu & 255)] = u_prev;
             }
             __syncwarp();
+          }
+        } else if (is_prior && KV == 2) {
+            // ---- prior warp, voxel pairs: pair s + 1's terms (both with pair s's old values,
+            //      reported for the correction) once pair s - 1's new values are in the tile (X)
+            bar_arrive(kBarT, 64);  // pair 0's terms were computed during the pack
+            const int nsteps = (nactv + 1) >> 1;
+            for (int s2 = 0; s2 < nsteps; ++s2) {
+                bar_sync(kBarX, 64);
+                if (s2 + 1 < nsteps) {
+                    const int ia = 2 * s2 + 2;
+                    PriTerm* out = pri + 2 * ((s2 + 1) & 1);
+                    prior_one<2>(tof, ia, ia - 2, ia - 1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, out);
+                    if (ia + 1 < nactv)
+                        prior_one<2>(tof, ia + 1, ia - 2, ia - 1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, out + 1);
+                    __syncwarp();
+                    bar_arrive(kBarT, 64);
+                }
+            }
         } else if (is_prior) {
             // ---- prior warp: voxel i + 1's terms once voxel i - 1's new value is in the tile (X);
             //      its arrival on A completes voxel i + 1's inputs
@@ -908,7 +1166,8 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             for (int idx = 0; idx < nactv; ++idx) {
                 bar_sync(kBarX, 64);
                 if (idx + 1 < nactv) {
-                    prior_one(tof, idx + 1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane, pri + ((g0 + (uint32_t)idx + 1) & 1));
+                    prior_one<1>(tof, idx + 1, idx, -1, xt, cslot, TW, gx0, gy0, zg, P, nb, lane,
+                                 pri + 2 * ((g0 + (uint32_t)idx + 1) & 1));
                     __syncwarp();
                     bar_arrive(kBarT, 64);
                 }
@@ -1002,15 +1261,24 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
 // (>= 2: the loop holds the current voxel's stage and the next voxel's)
 constexpr int ring_depth(bool u8) { return u8 ? 12 : 4; }
 
+template <int VPT, bool U8, int NNB, int R, int CL, int KV>
+auto pick_kernel(const IcdParams& p)
+{
+    // the phase profile (development aid) is built for the production variants only
+    constexpr bool kProf = VPT == MBIR_WIDE_VPT && U8 && CL == 1;
+    return p.theta2_pass ? k_svicd<VPT, U8, NNB, R, CL, KV, true, false>
+           : (kProf && p.tprof) ? k_svicd<VPT, U8, NNB, R, CL, KV, false, kProf>
+                                : k_svicd<VPT, U8, NNB, R, CL, KV, false, false>;
+}
+
 template <int VPT, bool U8, int NNB, int CL>
 cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
 {
     constexpr int R = ring_depth(U8);
-    // the phase profile (development aid) is built for the production variant only
-    constexpr bool kProf = VPT == MBIR_WIDE_VPT && U8 && CL == 1;
-    auto kern = p.theta2_pass ? k_svicd<VPT, U8, NNB, R, CL, true, false>
-                : (kProf && p.tprof) ? k_svicd<VPT, U8, NNB, R, CL, false, kProf>
-                                     : k_svicd<VPT, U8, NNB, R, CL, false, false>;
+    // voxel pairs: uint8 A with one CTA per task (api.cu validates)
+    constexpr bool kPairs = U8 && CL == 1;
+    auto kern = (kPairs && p.kv == 2) ? pick_kernel<VPT, U8, NNB, R, CL, kPairs ? 2 : 1>(p)
+                                      : pick_kernel<VPT, U8, NNB, R, CL, 1>(p);
     IcdParams q = p;
     q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT, p.V, CL);
     const int smem = q.lay.total;
@@ -1041,7 +1309,7 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
 template <int VPT, bool U8, int NNB, int CL>
 int resident_t(const IcdParams& p)
 {
-    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), CL, false, false>;
+    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), CL, 1, false, false>;
     const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT, p.V, CL).total;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
     cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);

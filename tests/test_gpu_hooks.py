@@ -34,7 +34,9 @@ def _state(cfg, case, og, Aq, nbhd, sweeps):
 def _replay(og, pr, Aq, case, x32, vox, t1g, t2g, dg):
     """Walk the GPU's update record: at each step the oracle computes Alg. 1 for that voxel at
     the current state, which is then advanced with the GPU's own delta (so every comparison is
-    a fixed-state comparison and fp32 drift of the state does not accumulate into it)."""
+    a fixed-state comparison and fp32 drift of the state does not accumulate into it).  A record
+    flagged DUMP_SAME_STATE (the second voxel of a pair) is computed at the state before the
+    previous record's update: the pair's updates are applied together after both checks."""
     plane = og.nx * og.ny
     V = og.nviews
     x = x32.astype(np.float64).copy()
@@ -42,7 +44,15 @@ def _replay(og, pr, Aq, case, x32, vox, t1g, t2g, dg):
     w = case.w.astype(np.float64)
     k = np.arange(V)[:, None]
     worst = np.zeros(3)
+    same = (vox & M.DUMP_SAME_STATE) != 0
+    vox = vox & (M.DUMP_SAME_STATE - 1)
+    pending = []  # (j, z, cols, msk, a, delta) of the updates computed from the current state
     for q in range(len(vox)):
+        if not same[q]:
+            for j, z, cols, msk, a, d in pending:  # advance with the GPU's updates (Alg1:8-11)
+                x[j] += d
+                np.subtract.at(e[z], (np.broadcast_to(k, cols.shape)[msk], cols[msk]), a[msk] * d)
+            pending = []
         j = int(vox[q])
         jj, z = j % plane, j // plane
         t1, t2, dl = O.voxel_update(og, pr, Aq, case.w, x, e, j, apply=False)
@@ -60,31 +70,35 @@ def _replay(og, pr, Aq, case, x32, vox, t1g, t2g, dg):
         assert r[0] <= 1e-5, (q, j, t1g[q], t1, s1)
         assert r[1] <= 1e-5, (q, j, t2g[q], t2)
         assert r[2] <= 1.0, (q, j, dg[q], dl, x[j], s1 / t2)
-        d = float(dg[q])  # advance with the GPU's update (Alg1:8-11)
-        x[j] += d
-        np.subtract.at(e[z], (np.broadcast_to(k, cols.shape)[msk], cols[msk]), a[msk] * d)
+        pending.append((j, z, cols, msk, a, float(dg[q])))
     return worst
 
 
 CASES = {
-    # (config, nbhd, quantize_A, sweeps of the oracle to reach the fixed state, CTAs per task)
-    "cfg1-u8": (CONFIGS["cfg1"], 8, 1, 3, 1),
-    "cfg1-f32": (CONFIGS["cfg1"], 8, 0, 3, 1),
-    "mini720-u8": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 1),
-    "mini720-u8-cluster2": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 2),
-    "mini3d-f32": (WorkloadConfig("mini3d", 40, 4, 60, 64, 7, 26, 0.002), 26, 0, 2, 1),
+    # (config, nbhd, quantize_A, sweeps of the oracle to reach the fixed state, CTAs per task,
+    #  voxels per step)
+    "cfg1-u8": (CONFIGS["cfg1"], 8, 1, 3, 1, 1),
+    "cfg1-f32": (CONFIGS["cfg1"], 8, 0, 3, 1, 1),
+    "mini720-u8": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 1, 1),
+    "mini720-u8-cluster2": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 2, 1),
+    "mini3d-f32": (WorkloadConfig("mini3d", 40, 4, 60, 64, 7, 26, 0.002), 26, 0, 2, 1, 1),
+    "cfg1-u8-pairs": (CONFIGS["cfg1"], 8, 1, 3, 1, 2),
+    "mini720-u8-pairs": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 1, 2),
+    "mini3d-u8-pairs-odd": (WorkloadConfig("mini3d", 40, 4, 60, 64, 7, 26, 0.002), 26, 1, 2, 1, 2),
 }
 
 
 @pytest.mark.parametrize("name", list(CASES))
 def test_hot_kernel_every_update_matches_oracle(name):
-    """The fused update kernel's own theta1 (incl. the pair-corrected theta1 of the second voxel
-    of each pair), theta2 (precomputed per sinogram) and delta (neighbour-corrected prior) for every
-    update of one deterministic sweep from a non-trivial state, against Alg. 1 in the oracle at the
-    identical state: reading R20's 1e-5.  mini720 is the bench's launch shape (720 views, 4 views
-    per lane, six view warps, uint8 A, 26-neighbourhood); cluster2 splits every task's views over a
-    2-CTA cluster that exchanges the partial sums through distributed shared memory."""
-    cfg, nbhd, quant, sweeps, cl = CASES[name]
+    """The fused update kernel's own theta1, theta2 (reduced by the kernel in this first iteration
+    after set_sinogram) and delta (neighbour-corrected prior) for every update of one deterministic
+    sweep from a non-trivial state, against Alg. 1 in the oracle at the identical state: reading
+    R20's 1e-5.  mini720 is the bench's launch shape (720 views, 4 views per lane, six view warps,
+    uint8 A, 26-neighbourhood); cluster2 splits every task's views over a 2-CTA cluster that
+    exchanges the partial sums through distributed shared memory; *-pairs run the voxel-pair
+    kernel (two voxels per step from one state), replayed pair by pair; mini3d's
+    side-7 tiles of a 40-pixel slice leave odd visits (a lone last voxel)."""
+    cfg, nbhd, quant, sweeps, cl, kv = CASES[name]
     case = make_case(cfg)
     g, og = geoms(cfg)
     A = O.sysmatrix(og)
@@ -93,32 +107,49 @@ def test_hot_kernel_every_update_matches_oracle(name):
     nvox = x32.size
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=nbhd),
                          M.Options(sv_side=cfg.sv_side, deterministic=1, zero_skip=0, quantize_A=quant,
-                                   cluster=cl)) as r:
-        assert r.sizes()["cluster"] == cl
+                                   cluster=cl, voxels_per_step=kv)) as r:
+        assert r.sizes()["cluster"] == cl and r.sizes()["voxels_per_step"] == kv
         r.set_sinogram(case.y, case.w)
         r.set_image(x32.reshape(cfg.nz, cfg.n, cfg.n))
         r.set_update_dump(nvox + 16)
         st = r.iterate(1)
         vox, t1g, t2g, dg, n = r.update_dump(nvox + 16)
     assert st["updates"] == nvox and n == nvox
-    np.testing.assert_array_equal(vox, deterministic_order(cfg.n, cfg.nz, cfg.sv_side, nbhd))
+    same = (vox & M.DUMP_SAME_STATE) != 0
+    order = deterministic_order(cfg.n, cfg.nz, cfg.sv_side, nbhd)
+    np.testing.assert_array_equal(vox & (M.DUMP_SAME_STATE - 1), order)
+    # pairs within each SV visit (runs of one (slice, SV) in the order): positions 1, 3, 5, ...
+    # of a visit share the state of the update before them
+    s = cfg.sv_side
+    iz, iy, ix = order // (cfg.n * cfg.n), (order // cfg.n) % cfg.n, order % cfg.n
+    visit = iz * 10 ** 6 + (iy // s) * 1000 + ix // s
+    pos = np.zeros(len(order), np.int64)
+    for q in range(1, len(order)):
+        pos[q] = pos[q - 1] + 1 if visit[q] == visit[q - 1] else 0
+    np.testing.assert_array_equal(same, (pos % 2 == 1) if kv == 2 else np.zeros_like(same))
     worst = _replay(og, pr, Ause, case, x32, vox, t1g, t2g, dg)
     print(name, "worst error / tolerance  theta1 %.3g  theta2 %.3g  delta %.3g" % (worst[0] / 1e-5, worst[1] / 1e-5, worst[2]))
 
 
-def test_update_dump_in_asynchronous_mode_is_consistent():
+@pytest.mark.parametrize("vps", [0, 2])
+def test_update_dump_in_asynchronous_mode_is_consistent(vps):
     """Outside deterministic mode the record holds every executed update once (in a nondeterministic
-    interleaving): the counts match mbir_stats and each voxel of iteration 1 appears exactly once."""
+    interleaving): the counts match mbir_stats and each voxel of iteration 1 appears exactly once;
+    with voxel pairs no two consecutive records are both a pair's second update."""
     cfg = CONFIGS["cfg1"]
     case = make_case(cfg)
     g, _ = geoms(cfg)
-    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=8), M.Options(sv_side=cfg.sv_side)) as r:
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=8),
+                         M.Options(sv_side=cfg.sv_side, voxels_per_step=vps)) as r:
         r.set_sinogram(case.y, case.w)
         r.set_update_dump(10000)
         st = r.iterate(1)
         vox, t1, t2, dl, n = r.update_dump(10000)
         assert n == st["updates"] == cfg.n * cfg.n
-        assert np.array_equal(np.sort(vox), np.arange(cfg.n * cfg.n))
+        assert r.sizes()["voxels_per_step"] == (vps or 1)
+        same = (vox & M.DUMP_SAME_STATE) != 0
+        assert same.any() == (vps == 2) and not (same[1:] & same[:-1]).any()
+        assert np.array_equal(np.sort(vox & (M.DUMP_SAME_STATE - 1)), np.arange(cfg.n * cfg.n))
         assert np.all(t2 > 0) and np.isfinite(t1).all() and np.isfinite(dl).all()
         st = r.iterate(1)
         n2 = r.update_dump(0)[4]

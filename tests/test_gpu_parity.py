@@ -409,17 +409,20 @@ def test_bench_shape_deterministic_tracks_oracle(m720, cluster):
     assert np.abs(eg.ravel() - e.ravel()).max() < 1e-4 * np.abs(case.y).max()
 
 
-@pytest.mark.parametrize("cluster", [1, 2])
-def test_bench_shape_converged_matches_oracle(m720, cluster):
+@pytest.mark.parametrize("cluster,vps", [(1, 1), (2, 1), (1, 2)])
+def test_bench_shape_converged_matches_oracle(m720, cluster, vps):
     """Asynchronous GPU-ICD in the bench's launch shape (persistent grid, random orders, 25 %
-    SV selection, zero-skipping off) reaches the oracle's MAP point: 1 HU / 1e-4."""
+    SV selection, zero-skipping off) reaches the oracle's MAP point: 1 HU / 1e-4 -- also with a
+    2-CTA cluster per task and with voxel pairs (same fixed points: a pair's update of x and e is
+    the sum of two exact single-voxel updates from one state)."""
     cfg, case, g, og, Aq = m720
     pr = O.Prior(sigma=cfg.sigma, nbhd=26)
     x = np.zeros(cfg.nz * cfg.n * cfg.n)
     e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
     O.icd_run(og, pr, Aq, case.w, x, e, 80, seed=3000, zero_skip=False)
     with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26),
-                         M.Options(sv_side=cfg.sv_side, zero_skip=0, cluster=cluster)) as r:
+                         M.Options(sv_side=cfg.sv_side, zero_skip=0, cluster=cluster, voxels_per_step=vps)) as r:
+        assert r.sizes()["voxels_per_step"] == vps
         r.set_sinogram(case.y, case.w)
         r.reconstruct(200)
         xg = r.image().ravel().astype(np.float64)
@@ -446,6 +449,21 @@ def test_cluster_option_validation():
     g, _ = geoms(cfg)
     with M.Reconstructor(g, M.Prior(neighborhood=26), M.Options(sv_side=cfg.sv_side, cluster=2)) as r:
         assert r.sizes()["cluster"] == 2 and r.sizes()["threads_per_cta"] == 32 * (3 + 2)
+
+
+def test_voxels_per_step_option_validation():
+    """mbir_options.voxels_per_step: 0 (auto) = 1, 1, or 2 (voxel pairs, uint8 A and one CTA per
+    task only); anything else is EINVAL."""
+    cfg = mini720()
+    g, _ = geoms(cfg)
+    for kw in ({"voxels_per_step": 3}, {"voxels_per_step": -1}, {"voxels_per_step": 2, "quantize_A": 0},
+               {"voxels_per_step": 2, "cluster": 2}):
+        with pytest.raises(M.MbirError) as ei:
+            M.Reconstructor(g, M.Prior(neighborhood=26), M.Options(sv_side=cfg.sv_side, **kw))
+        assert ei.value.code == -1, kw
+    for v, want in ((0, 1), (1, 1), (2, 2)):
+        with M.Reconstructor(g, M.Prior(neighborhood=26), M.Options(sv_side=cfg.sv_side, voxels_per_step=v)) as r:
+            assert r.sizes()["voxels_per_step"] == want
 
 
 # ------------------------------------------------------------------ FBP initial image (R23)

@@ -21,13 +21,15 @@ ap.add_argument("--sv-side", type=int, default=0)
 ap.add_argument("--batch-svs", type=int, default=0)
 ap.add_argument("--cluster", type=int, default=0)
 ap.add_argument("--quantize", type=int, default=1)
+ap.add_argument("--vps", type=int, default=0, help="voxels_per_step (0 auto)")
 a = ap.parse_args()
 cfg = CONFIGS[a.config]
 y, w = make_sinogram_torch(cfg, 0, "cuda")
 g = M.Geometry(cfg.n, cfg.n, cfg.nz, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dchannel)
 r = M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=cfg.nbhd),
                     M.Options(sv_side=a.sv_side or cfg.sv_side, zero_skip=a.zero_skip,
-                              batch_svs=a.batch_svs, cluster=a.cluster, quantize_A=a.quantize))
+                              batch_svs=a.batch_svs, cluster=a.cluster, quantize_A=a.quantize,
+                              voxels_per_step=a.vps))
 import time  # noqa: E402
 for k in range(2):
     torch.cuda.synchronize()
