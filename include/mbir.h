@@ -93,11 +93,14 @@ typedef struct mbir_options {
     int deterministic;     /* debug: every iteration visits all SVs one at a time (one CTA) in
                               the order z-parity half (3-D prior only), colour, SV rank within
                               the colour (SV index order), slice; voxels in raster order        */
-    int cluster;           /* CTAs per SV task in the update kernel: 0 = auto (1), 1 = one CTA
-                              owns a task, 2 = a 2-CTA thread-block cluster splits the task's views
+    int cluster;           /* CTAs per SV task in the update kernel: 0 = auto (1, or 2 when one
+                              CTA's shared memory cannot hold the SV buffer: large SVs, e.g.
+                              side 11-15 at the paper's 720 x 1024 geometry), 1 = one CTA owns a
+                              task, 2 = a 2-CTA thread-block cluster splits the task's views
                               (each holds half the SV buffer; one partial sum per voxel crosses
                               distributed shared memory; two SMs per SV).  2 needs > 128 views in
-                              an even number of 128-view warps.  Same arithmetic either way       */
+                              an even number of 128-view warps.  Same arithmetic either way.  SV
+                              bands of up to 61 rows (channels) per view are supported          */
     int zero_skip_period;  /* with zero_skip: iterations 1 + k*zero_skip_period, k >= 1 (numbers
                               counted from the last set_sinogram / set_image) run
                               WITHOUT zero-skipping on a random sv_fraction of the SVs, so voxels

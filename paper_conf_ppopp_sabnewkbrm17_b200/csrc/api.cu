@@ -107,7 +107,7 @@ struct mbir_handle {
     ncclComm_t comm = nullptr;
     LocalGroup* lg = nullptr;  // mbir_link_slabs group (shared by its members; rank 0 frees it)
     int side = 0, nsvx = 0, nsvy = 0, nsv = 0, S2 = 0, nsv_pad = 0;
-    int rows = 0, band_max = 0;
+    int rows = 0, band_max = 0, nwin = 1;
     int vpt = 1, nvw = 0, Vs = 0, threads = 0, smem = 0, blocks_per_sm = 1, nsm = 148;
     int cl = 1;  // update-kernel CTAs per SV task (2: thread-block cluster splitting the views)
     int kv = 1;  // voxels per step of the update kernel (2: voxel pairs)
@@ -184,6 +184,7 @@ IcdParams make_params(mbir_handle* h)
     p.S2 = h->S2;
     p.Vs = h->Vs;
     p.rows = h->rows;
+    p.nwin = h->nwin;
     p.nvw = h->nvw;
     p.A = h->A;
     p.e = h->d_e;
@@ -740,13 +741,14 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if (info[0] & 2) return (fail(h, MBIR_EINVAL, "SV band wider than 255 channels"), bail(MBIR_EINVAL));
     h->rows = info[1];
     h->band_max = info[2];
-    // a band row plus its misalignment (<= 3 floats) must fit one aligned 32-float window
+    // a band row plus its misalignment (<= 3 floats) must fit one or two aligned 32-float windows
     if (h->rows > kMaxSvbRows - 3)
-        return (fail(h, MBIR_EINVAL, "SV band needs " + std::to_string(h->rows) + " > 29 buffer rows: reduce sv_side"), bail(MBIR_EINVAL));
+        return (fail(h, MBIR_EINVAL, "SV band needs " + std::to_string(h->rows) + " > 61 buffer rows: reduce sv_side"), bail(MBIR_EINVAL));
+    h->nwin = h->rows + 3 > 32 ? 2 : 1;
     if (((size_t)G.nviews * G.nchannels) % 4 != 0)
         return (fail(h, MBIR_EINVAL, "nviews * nchannels must be a multiple of 4"), bail(MBIR_EINVAL));
-    if ((size_t)G.nviews * G.nchannels >= (size_t(1) << 27))  // band row offsets are packed << 5
-        return (fail(h, MBIR_EINVAL, "nviews * nchannels must be < 2^27"), bail(MBIR_EINVAL));
+    if ((size_t)G.nviews * G.nchannels >= (size_t(1) << 26))  // band row offsets are packed << 6
+        return (fail(h, MBIR_EINVAL, "nviews * nchannels must be < 2^26"), bail(MBIR_EINVAL));
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
     {
@@ -758,6 +760,10 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
         if (h->o.cluster < 0 || h->o.cluster > 2)
             return (fail(h, MBIR_EINVAL, "cluster must be 0 (auto), 1 or 2"), bail(MBIR_EINVAL));
         h->cl = h->o.cluster == 2 ? 2 : 1;
+        // auto: a 2-CTA cluster when one CTA cannot hold the SV buffer (large SVs, NEXT-2)
+        if (h->o.cluster == 0 && h->vpt == MBIR_WIDE_VPT && h->nvw % 2 == 0 &&
+            svicd_smem_bytes(p, h->vpt, P.neighborhood, quant, 1) > (int)prop.sharedMemPerBlockOptin)
+            h->cl = 2;
         if (h->cl == 2 && !(h->vpt == 4 && h->nvw % 2 == 0))
             return (fail(h, MBIR_EINVAL, "cluster = 2 needs > 128 views in an even number of 128-view warps"), bail(MBIR_EINVAL));
         if (h->o.voxels_per_step < 0 || h->o.voxels_per_step > 2)
@@ -776,21 +782,20 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
 
     // ---- state buffers
     const size_t ns = sino_elems(h), pl = plane_elems(h);
-    // (+32 floats: the update kernel reads whole 32-float windows around band rows)
-    if ((r = dalloc(h, &h->d_y, ns + 32))) return bail(r);
-    if ((r = dalloc(h, &h->d_w, ns + 32))) return bail(r);
-    if ((r = dalloc(h, &h->d_e, ns + 32))) return bail(r);
-    // the pack reads whole 16-byte-aligned 32-float windows around band rows, up to 32 floats past
-    // the last row: the padding is zero, never uninitialised
-    cudaMemsetAsync(h->d_y, 0, (ns + 32) * 4, h->st);
-    cudaMemsetAsync(h->d_w, 0, (ns + 32) * 4, h->st);
-    cudaMemsetAsync(h->d_e, 0, (ns + 32) * 4, h->st);
+    // (+64 floats: the update kernel reads whole 32-float windows around band rows, up to 64
+    // floats past the last row with two windows; the padding is zero, never uninitialised)
+    if ((r = dalloc(h, &h->d_y, ns + 64))) return bail(r);
+    if ((r = dalloc(h, &h->d_w, ns + 64))) return bail(r);
+    if ((r = dalloc(h, &h->d_e, ns + 64))) return bail(r);
+    cudaMemsetAsync(h->d_y, 0, (ns + 64) * 4, h->st);
+    cudaMemsetAsync(h->d_w, 0, (ns + 64) * 4, h->st);
+    cudaMemsetAsync(h->d_e, 0, (ns + 64) * 4, h->st);
     if ((r = dalloc(h, &h->d_x, pl * (G.nz_local + 2)))) return bail(r);
     if ((r = dalloc(h, &h->d_theta2, (size_t)G.nz_local * h->nsv * h->S2))) return bail(r);
     cudaMemset(h->d_theta2, 0, (size_t)G.nz_local * h->nsv * h->S2 * sizeof(float));
     if ((r = dalloc(h, &h->d_amount, (size_t)G.nz_local * h->nsv))) return bail(r);
     // e_init tiles of the concurrently running SV visits: one per CTA of the largest grid
-    if ((r = dalloc(h, &h->d_scratch, (size_t)h->nsm * h->blocks_per_sm * svicd_scratch_floats(h->vpt)))) return bail(r);
+    if ((r = dalloc(h, &h->d_scratch, (size_t)h->nsm * h->blocks_per_sm * svicd_scratch_floats(h->vpt, h->nwin)))) return bail(r);
     if ((r = dalloc(h, &h->d_task_list, (size_t)G.nz_local * 4 * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_task_count, (size_t)G.nz_local * 4))) return bail(r);
     if ((r = dalloc(h, &h->d_flat, (size_t)8 * G.nz_local * h->max_group))) return bail(r);

@@ -20,7 +20,7 @@ namespace mbir {
 
 constexpr int kK = 4;             // max channels per (voxel, view) (reading R5; K=4 for dc > 0.4714 dxy)
 constexpr int kMaxNbr = 26;       // 3-D neighbourhood (reading R2)
-constexpr int kMaxSvbRows = 32;   // SV-buffer rows held by one 32-lane transpose tile
+constexpr int kMaxSvbRows = 64;   // SV-buffer rows: two 32-float windows per band row (pack / write-back)
 constexpr int kMaxPhaseSlices = 1024;  // slices of one (z-parity, colour) phase (sched.cu k_flatten)
 constexpr int kAutoCapDiv = 12;  // batch_svs = 0: at most N / 12 concurrently updated SVs per slice (R22)
 constexpr int kAutoCapMin = 4;
@@ -94,6 +94,7 @@ struct IcdParams {
     uint64_t seed;
     int iter;
     int zero_skip_active;
+    int nwin;         // 32-float windows per band row in the pack / write-back (1, or 2 for > 29 rows)
     int kv;           // voxels per step (1: exact sequential within the SV, 2: voxel pairs)
     int theta2_pass;  // this launch reduces theta2 (Alg1:6) with theta1 and stores it (iteration 1)
     int deterministic;
@@ -126,7 +127,7 @@ cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, i
 // warp, vpt = 4 (or 1 for <= 128 views) views per lane; cl = 2: a 2-CTA cluster splits a task's views
 int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
 int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
-int svicd_scratch_floats(int vpt);  // per-CTA e_init scratch tile
+int svicd_scratch_floats(int vpt, int nwin);  // per-CTA e_init scratch tile
 cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int cl, int grid, cudaStream_t st);
 cudaError_t launch_theta2(const IcdParams& p, bool quantize, cudaStream_t st);
 cudaError_t launch_forward(const IcdParams& p, bool quantize, const float* y, cudaStream_t st);

@@ -177,8 +177,8 @@ struct NbrOne {
 // previous voxel that is a neighbour of i its term (btu) and weight (bwu), which the delta warp
 // replaces by the term at the new value: exact.  (With pairs, the other voxel of i's own pair
 // keeps its old value: both are computed from the same state.)
-struct PriTerm {
-    float s, sx, v, btu0, bwu0, btu1, bwu1;
+struct __align__(16) PriTerm {
+    float s, sx, v, btu0, bwu0, btu1, bwu1, pad;  // 32 B: read as two 16-byte words
 };
 
 template <int NP>  // previous-step voxels to report (1, or 2 with voxel pairs)
@@ -220,7 +220,7 @@ __device__ __forceinline__ void prior_one(const int* tof, int i, int ip0, int ip
         bwu1 = __shfl_sync(kFull, nb.w, src1);
         if (!w1) btu1 = bwu1 = 0.f;
     }
-    if (lane == 0) *out = PriTerm{s, sx, v, w0 ? btu0 : 0.f, w0 ? bwu0 : 0.f, btu1, bwu1};
+    if (lane == 0) *out = PriTerm{s, sx, v, w0 ? btu0 : 0.f, w0 ? bwu0 : 0.f, btu1, bwu1, 0.f};
 }
 
 // sum of the view warps' partials (slots) in a fixed tree order (<= 8 or 16 slots)
@@ -302,21 +302,10 @@ __host__ __device__ inline SmemLayout svicd_layout(int rows, int side, int S2, i
     L.rth2 = o;  o = align16(o + S2 * 4);       //   per-slot scales and theta2,
     L.rbs = o;   o = align16(o + V * 4);        //   band start and width per view
     L.rbw = o;   o = align16(o + V);
-    L.binfo = o; o = align16(o + 2 * VA * cl * 4);  // band (row offset << 5 | width) per view, 2 tasks
+    L.binfo = o; o = align16(o + 2 * VA * cl * 4);  // band (row offset << 6 | width) per view, 2 tasks
     L.cx = o;    o = align16(o + 2 * 2 * 2 * 4 + 4 * 8);  // CL = 2: partial sums [2 steps][2 quantities][2 CTAs], mbarriers
     L.total = o;
     return L;
-}
-
-// band of task tk for views k = k0, k0 + stride, ... < V into dst[k] = (k*M + start) << 5 | width
-__device__ __forceinline__ void band_info(const IcdParams& P, int tk, uint32_t* dst, int k0, int stride)
-{
-    const int sv = tk & 16383;
-    for (int k = k0; k < P.V; k += stride) {
-        const int r = k * P.M + P.A.band_start[(size_t)sv * P.V + k];
-        const int wd = P.A.band_width[(size_t)sv * P.V + k];
-        dst[k] = ((uint32_t)r << 5) | (uint32_t)wd;
-    }
 }
 
 // this thread's VPT adjacent records from a stage as raw words (CW = 1: a uint8 code word per
@@ -576,14 +565,14 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                     vtb[i] = rth2[v];
                 }
                 if (n > 0) {
-                    // band info (row offset << 5 | width) and an L2 warm-up of the band rows
+                    // band info (row offset << 6 | width) and an L2 warm-up of the band rows
                     uint32_t* dst = binfo + b * VA;
                     const float* wz = P.w + (size_t)z * V * M;
                     const float* ez = P.e + (size_t)z * V * M;
                     for (int k = lane; k < V; k += 32) {
                         const int wd = (V & 3) == 0 ? rbw[k] : P.A.band_width[(size_t)sv * V + k];
                         const int r = k * M + rbs[k], r1 = r + max(wd, 1) - 1;
-                        dst[k] = ((uint32_t)r << 5) | (uint32_t)wd;
+                        dst[k] = ((uint32_t)r << 6) | (uint32_t)wd;
                         asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r));
                         asm volatile("prefetch.global.L2 [%0];" ::"l"(wz + r1));
                         asm volatile("prefetch.global.L2 [%0];" ::"l"(ez + r));
@@ -669,26 +658,28 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
 
         // ---- 4. view warps: SVB pack (coalesced band-row windows transposed through staging
         //         tiles); e_init rows go to this CTA's L2-resident scratch tile for the write-back
-        float* scr = P.scratch + (size_t)blockIdx.x * (size_t)VS * 32;
+        const int nwin = P.nwin;  // 32-float windows per band row (2: bands of 30..61 rows)
+        float* scr = P.scratch + (size_t)blockIdx.x * (size_t)nwin * VS * 32;
         const int ntw = tile_warps(VAL);
         if (is_view && vw < ntw) {
             const float* wz = P.w + (size_t)z * V * M;
             float* ez = P.e + (size_t)z * V * M;
-            // Each band row is read as the 16-byte-aligned 32-float window that contains it (the
+            // Each band row is read as the 16-byte-aligned 32-float window(s) that contain it (the
             // slice base is 16-byte aligned, V*M % 4 == 0): 8 lanes x float4 per row, 4 rows per
             // LDG.128; the window goes through the warp's staging tile and band column
             // c = p - s_k lands in sb row c, column k (bank k)
             const int sub = lane >> 3, ch = lane & 7;  // row-in-quad and float4 chunk of this lane
+            int wq = 0;                                // window of the band rows (0, 1)
             auto issue = [&](int t, bool isw, float4 (&v4)[8]) {
                 const int kk = vbase + (vw * kTileW + t) * 32 + lane;  // global view
                 const uint32_t bi = kk < V ? binfo[tb * VA + kk] : 0u;
-                const int rot = (int)(bi >> 5);
+                const int rot = (int)(bi >> 6);
 #pragma unroll
                 for (int m = 0; m < 8; ++m) {
                     const int oi = __shfl_sync(kFull, rot, 4 * m + sub);
                     // unconditional loads: the whole aligned window is read (padded views read the
-                    // slice start; the sinogram allocations carry 32 floats of tail padding)
-                    const size_t a4 = (size_t)(oi - (oi & 3)) + 4 * ch;
+                    // slice start; the sinogram allocations carry 64 floats of tail padding)
+                    const size_t a4 = (size_t)(oi - (oi & 3)) + 32 * wq + 4 * ch;
                     v4[m] = isw ? __ldg((const float4*)(wz + a4)) : __ldcg((const float4*)(ez + a4));
                 }
             };
@@ -696,13 +687,15 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 const int k0 = (vw * kTileW + t) * 32;  // local column of the tile
                 const uint32_t bi = vbase + k0 + lane < V ? binfo[tb * VA + vbase + k0 + lane] : 0u;
                 const int kk = k0 + lane;
-                const int bwt = (int)(bi & 31u), sk = (int)(bi >> 5) & 3;
-                const uint32_t bmask = ((1u << bwt) - 1u) << sk;  // band's window positions
+                const int bwt = (int)(bi & 63u), sk = (int)(bi >> 6) & 3;
+                // the band's positions in this window
+                const uint32_t bmask = (uint32_t)((((1ull << bwt) - 1ull) << sk) >> (32 * wq));
                 if (!isw) {
 #pragma unroll
-                    for (int m = 0; m < 8; ++m) __stcg((float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch), v4[m]);
+                    for (int m = 0; m < 8; ++m)
+                        __stcg((float4*)(scr + ((size_t)wq * VS + k0 + 4 * m + sub) * 32 + 4 * ch), v4[m]);
                 }
-                float* d = sb + (isw ? VS : 0) + kk - sk * RS;  // + p RS = band row p - sk of view kk
+                float* d = sb + (isw ? VS : 0) + kk + (32 * wq - sk) * RS;  // + p RS = band row 32 wq + p - sk
 #pragma unroll
                 for (int m = 0; m < 8; ++m) *(float4*)(stg_w + (4 * m + sub) * kStg + 4 * ch) = v4[m];
                 __syncwarp();
@@ -716,17 +709,19 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 }
                 __syncwarp();
             };
-            float4 wa4[2][8], ea4[2][8];
-            issue(0, true, wa4[0]);
-            issue(0, false, ea4[0]);
+            for (wq = 0; wq < nwin; ++wq) {
+                float4 wa4[2][8], ea4[2][8];
+                issue(0, true, wa4[0]);
+                issue(0, false, ea4[0]);
 #pragma unroll
-            for (int t = 0; t < kTileW; ++t) {
-                if (t + 1 < kTileW) {
-                    issue(t + 1, true, wa4[(t + 1) & 1]);
-                    issue(t + 1, false, ea4[(t + 1) & 1]);
+                for (int t = 0; t < kTileW; ++t) {
+                    if (t + 1 < kTileW) {
+                        issue(t + 1, true, wa4[(t + 1) & 1]);
+                        issue(t + 1, false, ea4[(t + 1) & 1]);
+                    }
+                    finish(t, true, wa4[t & 1]);
+                    finish(t, false, ea4[t & 1]);
                 }
-                finish(t, true, wa4[t & 1]);
-                finish(t, false, ea4[t & 1]);
             }
         }
         __syncthreads();
@@ -1181,10 +1176,12 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
         if (is_view && vw < ntw) {
             float* ez = P.e + (size_t)z * V * M;
             const int sub = lane >> 3, ch = lane & 7;
+            for (int wq = 0; wq < nwin; ++wq) {
             auto ld_init = [&](int t, float4 (&s4)[8]) {
                 const int k0 = (vw * kTileW + t) * 32;
 #pragma unroll
-                for (int m = 0; m < 8; ++m) s4[m] = __ldcg((const float4*)(scr + (k0 + 4 * m + sub) * 32 + 4 * ch));
+                for (int m = 0; m < 8; ++m)
+                    s4[m] = __ldcg((const float4*)(scr + ((size_t)wq * VS + k0 + 4 * m + sub) * 32 + 4 * ch));
             };
             float4 s4b[2][8];
             ld_init(0, s4b[0]);
@@ -1195,10 +1192,10 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
                 const int k0 = (vw * kTileW + t) * 32;  // local column of the tile
                 const int kk = k0 + lane;
                 const uint32_t bi = vbase + kk < V ? binfo[tb * VA + vbase + kk] : 0u;
-                const int bw = (int)(bi & 31u), roff = (int)(bi >> 5);
-                const uint32_t bmask = ((1u << bw) - 1u) << (roff & 3);
-                // this view's final band -> its staging row (positions outside the band: 0)
-                const float* se = sb + kk - (roff & 3) * RS;
+                const int bw = (int)(bi & 63u), roff = (int)(bi >> 6);
+                const uint32_t bmask = (uint32_t)((((1ull << bw) - 1ull) << (roff & 3)) >> (32 * wq));
+                // this view's final band in window wq -> its staging row (positions outside: 0)
+                const float* se = sb + kk + (32 * wq - (roff & 3)) * RS;
 #pragma unroll
                 for (int q4 = 0; q4 < 8; ++q4) {
                     float rv[4];
@@ -1222,9 +1219,10 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
 #pragma unroll
                     for (int j = 0; j < 4; ++j) d[j] = (nib & (1u << j)) ? fv[j] - e0[j] : 0.f;
                     if (vbase + k0 + i < V && (d[0] != 0.f || d[1] != 0.f || d[2] != 0.f || d[3] != 0.f))
-                        red_add_v4(ez + (oi - (oi & 3)) + 4 * ch, d[0], d[1], d[2], d[3]);
+                        red_add_v4(ez + (oi - (oi & 3)) + 32 * wq + 4 * ch, d[0], d[1], d[2], d[3]);
                 }
                 __syncwarp();
+            }
             }
         } else if (is_delta) {
             // the image and the counters, then the next task's preparation (with the prior warp)
@@ -1363,7 +1361,7 @@ int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int
     SVICD_DISPATCH(resident_t, p)
 }
 
-int svicd_scratch_floats(int vpt) { return svb_cols(vpt) * 32; }
+int svicd_scratch_floats(int vpt, int nwin) { return svb_cols(vpt) * 32 * nwin; }
 
 cudaError_t launch_svicd(const IcdParams& p, int vpt, int nnb, bool quantize, int cl, int grid, cudaStream_t st)
 {

@@ -85,6 +85,9 @@ CASES = {
     "cfg1-u8-pairs": (CONFIGS["cfg1"], 8, 1, 3, 1, 2),
     "mini720-u8-pairs": (WorkloadConfig("mini720", 48, 2, 720, 96, 9, 26, 0.005), 26, 1, 2, 1, 2),
     "mini3d-u8-pairs-odd": (WorkloadConfig("mini3d", 40, 4, 60, 64, 7, 26, 0.002), 26, 1, 2, 1, 2),
+    # side 11 at the paper's pitch: 35-row bands (two 32-float windows per band row in the pack and
+    # write-back), the SV buffer held by a 2-CTA cluster (NEXT-2)
+    "mini720-u8-side11-cluster2": (WorkloadConfig("mini720", 48, 2, 720, 96, 11, 26, 0.005), 26, 1, 2, 2, 1),
 }
 
 

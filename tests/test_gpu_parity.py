@@ -451,6 +451,45 @@ def test_cluster_option_validation():
         assert r.sizes()["cluster"] == 2 and r.sizes()["threads_per_cta"] == 32 * (3 + 2)
 
 
+def test_large_svs_use_two_windows_and_a_cluster():
+    """NEXT-2 (larger SVs): at the paper's pitch (dc = dxy/2) side 9 needs <= 29
+    band rows (one 32-float window per row, one CTA); sides 11 and 13 need 35-41 rows: two
+    windows per row, and auto cluster selection splits the SV buffer over a 2-CTA cluster; a side
+    whose band exceeds 61 rows is EINVAL."""
+    for side, want_cl in ((9, 1), (11, 2), (13, 2)):
+        cfg = WorkloadConfig("mini720", 48, 2, 720, 96, side, 26, 0.005)
+        g, _ = geoms(cfg)
+        with M.Reconstructor(g, M.Prior(neighborhood=26), M.Options(sv_side=side)) as r:
+            s = r.sizes()
+            assert s["cluster"] == want_cl, (side, s)
+            assert (s["svb_rows"] > 29) == (side > 9), (side, s)
+    cfg = WorkloadConfig("big", 96, 1, 720, 192, 24, 8, 0.005)
+    g, _ = geoms(cfg)
+    with pytest.raises(M.MbirError) as ei:
+        M.Reconstructor(g, M.Prior(neighborhood=8), M.Options(sv_side=24))
+    assert ei.value.code == -1
+
+
+@pytest.mark.parametrize("side", [11, 13])
+def test_large_sv_converged_matches_oracle(m720, side):
+    """Asynchronous GPU-ICD with side-11 / side-13 SVs (two-window bands, 2-CTA clusters) reaches
+    the oracle's MAP point on the bench-shaped case: 1 HU / 1e-4."""
+    cfg, case, g, og, Aq = m720
+    pr = O.Prior(sigma=cfg.sigma, nbhd=26)
+    x = np.zeros(cfg.nz * cfg.n * cfg.n)
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+    O.icd_run(og, pr, Aq, case.w, x, e, 80, seed=3000, zero_skip=False)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26), M.Options(sv_side=side, zero_skip=0)) as r:
+        assert r.sizes()["cluster"] == 2
+        r.set_sinogram(case.y, case.w)
+        r.reconstruct(200)
+        xg = r.image().ravel().astype(np.float64)
+    assert O.rmse_hu(xg, x) < 1.0
+    cg = O.cost(og, pr, Aq, case.y, case.w, xg)
+    co = O.cost(og, pr, Aq, case.y, case.w, x)
+    assert abs(cg - co) <= 1e-4 * abs(co), (cg, co)
+
+
 def test_voxels_per_step_option_validation():
     """mbir_options.voxels_per_step: 0 (auto) = 1, 1, or 2 (voxel pairs, uint8 A and one CTA per
     task only); anything else is EINVAL."""
