@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-converge", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-psv", action="store_true", help="skip the PSV-ICD CPU comparison leg")
     ap.add_argument("--conv-iters", type=int, default=300, help="max iterations of a convergence run")
     return ap.parse_args()
 
@@ -144,6 +145,47 @@ def cpu_baseline(budget_s=12.0):
             "sample": f"sequential C oracle (double), {sweeps} equits of a 128x128 slice at "
                       f"config-4 pitch (0.5 mm), 720 views x 256 channels (dc = dxy/2, "
                       f"{int(Aq.count.sum() / (cfg.n * cfg.n))} nnz/voxel), {upd} updates in {el:.1f} s"}
+
+
+def psv_baseline(max_s=40.0, side=13):
+    """The paper's CPU comparison system, PSV-ICD (Alg. 2; psvicd/, SURVEY 8(f)
+    NEXT-4), on all host cores: time from the oracle's FBP image to < 10 HU RMSE against the
+    committed cfg3 oracle golden on cfg3 (the paper's T1 workload shape), 20 % SV
+    selection, SV side 13 (T1's PSV-ICD column).  A and the FBP image come from the oracle
+    (test infrastructure; setup not timed).  The paper's 4.43x GPU-ICD / PSV-ICD is
+    context only."""
+    import oracle as O
+    from psvicd import PSVICD
+    from synth import CONFIGS, make_case
+    t_setup = time.perf_counter()
+    cfg = CONFIGS["cfg3"]
+    case = make_case(cfg, 0, with_truth=False)
+    og = O.Geometry(cfg.n, cfg.n, 1, cfg.dxy, cfg.nviews, cfg.nchannels, cfg.dchannel)
+    _, _, Aq = O.quantize(O.sysmatrix(og))
+    z = np.load(os.path.join(ROOT, "tests", "golden", "golden_cfg3.npz"))
+    gold = z["x"].ravel().astype(np.float64)
+    x = O.fbp(og, case.y).astype(np.float32).reshape(1, cfg.n, cfg.n).copy()
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x.ravel().astype(np.float64))
+    e = np.ascontiguousarray(e.astype(np.float32).reshape(case.y.shape))
+    w = np.ascontiguousarray(case.w, np.float32)
+    psv = PSVICD(cfg.n, cfg.n, 1, cfg.nviews, cfg.nchannels, Aq, sigma=cfg.sigma, nbhd=cfg.nbhd, sv_side=side)
+    t_setup = time.perf_counter() - t_setup
+    t, upd, hit, it, rm, nt = 0.0, 0, None, 0, None, None
+    while t < max_s:
+        st = psv.iterate(w, x, e, 1, frac=0.2)
+        it += 1
+        t += st["seconds"]
+        upd += st["updates"]
+        nt = st["threads"]
+        rm = O.rmse_hu(x.ravel().astype(np.float64), gold)
+        if rm < 10.0:
+            hit = t
+            break
+    psv.close()
+    return {"kind": "PSV-ICD (Alg. 2) on host threads", "workload": "cfg3: 512x512, 720 views x 1024 channels",
+            "cores": nt, "sv_side": side, "frac": 0.2, "init": "oracle FBP (not timed)",
+            "time_to_10hu_s": hit, "equits_to_10hu": upd / cfg.n ** 2 if hit else None, "iterations": it,
+            "final_rmse_hu": rm, "updates_per_s": upd / t if t > 0 else None, "setup_s": t_setup}
 
 
 def workload_config(cfg, side, args, world):
@@ -402,6 +444,14 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_baseline()
+    psv = None
+    if rank == 0 and world == 1 and not args.no_psv and not args.no_cpu:
+        psv = psv_baseline()
+        g3 = ((conv or {}).get("cfg3") or {}).get("from_fbp") or {}
+        if args.config == "cfg3":
+            g3 = (conv or {}).get("from_fbp") or {}
+        if psv.get("time_to_10hu_s") and g3.get("time_to_10hu_s"):
+            psv["gpu_speedup_time_to_10hu"] = psv["time_to_10hu_s"] / g3["time_to_10hu_s"]
 
     if rank == 0:
         clocks = clk.summary()
@@ -414,7 +464,7 @@ def main():
             "config": workload_config(cfg, side, args, world),
             "updates_per_step": updates / args.steps,
             "time_to_converge": conv,
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "roofline": roof, "cpu_baseline": cpu, "psv_icd": psv, "e2e": e2e,
             "gpu_launches": launches, "clocks": clocks,
             "setup_s": setup_s, "sizes": sizes,
         }
