@@ -245,21 +245,22 @@ def make_case(cfg: WorkloadConfig, case_id: int = 0, *, phantom_seed=None, noise
 SWEEP_SIGMA = {64: 0.002, 128: 0.003, 256: 0.004}
 
 
-def sweep_configs(n_cases: int = 200, seed: int = 5000, sizes=(128, 256)):
+def sweep_configs(n_cases: int = 200, seed: int = 5000, sizes=(128, 256), sides=(5, 7, 9), prefix="sweep"):
     """BASELINE.json configs[4]: synthetic 2-D cases varying phantom, dose, view count and SV side
     (the paper's 3200-case suite, in miniature), sampled without replacement from the
     grid phantom {Shepp-Logan, 3 baggage seeds} x lambda0 {1e3, 1e4, 1e5} x V {90, 180, 360, 720}
     x side {5, 7, 9} x N `sizes`, M = 2N (the paper's channel:pixel ratio, so dc = dxy/2).
-    Side 11 and 13 of the survey's grid need SV bands wider than the update kernel's 29 buffer
-    rows at dc = dxy/2 (reading R13) and are left out.  Returns [(WorkloadConfig, case_id)]."""
+    The 200-case sample keeps sides {5, 7, 9}; sides 11 and 13 of the survey's grid (two-window
+    bands, 2-CTA clusters) form a supplementary sample: sweep_configs(40, 5001, sides=(11, 13),
+    prefix="sweepL").  Returns [(WorkloadConfig, case_id)]."""
     rng = np.random.default_rng(seed)
     grid = [(ph, lam, v, s, n) for ph in ("shepp_logan", "baggage:0", "baggage:1", "baggage:2")
-            for lam in (1e3, 1e4, 1e5) for v in (90, 180, 360, 720) for s in (5, 7, 9) for n in sizes]
+            for lam in (1e3, 1e4, 1e5) for v in (90, 180, 360, 720) for s in sides for n in sizes]
     pick = rng.choice(len(grid), size=min(n_cases, len(grid)), replace=False)
     out = []
     for i, gi in enumerate(sorted(pick)):
         ph, lam, v, s, n = grid[gi]
         base, _, bseed = ph.partition(":")
-        cfg = WorkloadConfig(f"sweep{i}", n, 1, v, 2 * n, s, 8, SWEEP_SIGMA[n], phantom=base, lambda0=lam)
+        cfg = WorkloadConfig(f"{prefix}{i}", n, 1, v, 2 * n, s, 8, SWEEP_SIGMA[n], phantom=base, lambda0=lam)
         out.append((cfg, 100 + (int(bseed) if bseed else 0)))
     return out

@@ -51,10 +51,12 @@ def run(r, golden, init, max_iter=400):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=None)
+    ap.add_argument("--set", default="main", choices=["main", "large"])
     a = ap.parse_args()
-    allc = sweep_configs()
+    allc = sweep_configs(40, 5001, sides=(11, 13), prefix="sweepL") if a.set == "large" else sweep_configs()
+    pref = "sweepL" if a.set == "large" else "sweep"
     rows = []
-    for path in sorted(glob.glob(os.path.join(ROOT, "goldens", "sweep", "sweep*.npz"))):
+    for path in sorted(glob.glob(os.path.join(ROOT, "goldens", "sweep", f"{pref}[0-9]*.npz"))):
         z = np.load(path)
         meta = json.loads(str(z["meta"]))
         cfg, cid = allc[meta["idx"]]

@@ -10,6 +10,8 @@ is < 10 HU from the golden.  Writes goldens/sweep/<case>.npz and appends one JSO
 to goldens/sweep/oracle.jsonl.
 
   python tools/sweep_goldens.py --cases 0,4,8,...   (indices into sweep_configs())
+  python tools/sweep_goldens.py --set large --cases all --jobs 32   (the side-11/13 supplement,
+                                                                    one process per case)
 """
 import argparse
 import json
@@ -27,15 +29,34 @@ from synth import make_case, sweep_configs  # noqa: E402
 from tools.make_golden import sino_hash  # noqa: E402
 
 
+def case_set(name):
+    """the 200-case config-5 sample, or the side-11/13 supplement"""
+    return sweep_configs(40, 5001, sides=(11, 13), prefix="sweepL") if name == "large" else sweep_configs()
+
+
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--cases", required=True)
+    ap.add_argument("--cases", required=True, help="comma-separated indices, or 'all'")
     ap.add_argument("--equits", type=int, default=60)
+    ap.add_argument("--set", default="main", choices=["main", "large"])
+    ap.add_argument("--jobs", type=int, default=1, help="cases run in parallel processes")
     a = ap.parse_args()
-    allc = sweep_configs()
+    allc = case_set(a.set)
+    idxs = list(range(len(allc))) if a.cases == "all" else [int(v) for v in a.cases.split(",") if v]
+    if a.jobs > 1:
+        import subprocess
+        procs = []
+        for i, idx in enumerate(idxs):
+            procs.append(subprocess.Popen([sys.executable, os.path.abspath(__file__), "--cases", str(idx),
+                                           "--equits", str(a.equits), "--set", a.set]))
+            if len(procs) >= a.jobs:
+                procs.pop(0).wait()
+        for pr_ in procs:
+            pr_.wait()
+        return
     out = os.path.join(ROOT, "goldens", "sweep")
     os.makedirs(out, exist_ok=True)
-    for idx in [int(v) for v in a.cases.split(",") if v]:
+    for idx in idxs:
         cfg, cid = allc[idx]
         path = os.path.join(out, f"{cfg.name}.npz")
         if os.path.exists(path):
