@@ -98,8 +98,9 @@ typedef struct mbir_options {
                               side 11-15 at the paper's 720 x 1024 geometry), 1 = one CTA owns a
                               task, 2 = a 2-CTA thread-block cluster splits the task's views
                               (each holds half the SV buffer; one partial sum per voxel crosses
-                              distributed shared memory; two SMs per SV).  2 needs > 128 views in
-                              an even number of 128-view warps.  Same arithmetic either way.  SV
+                              distributed shared memory; two SMs per SV).  2 needs > 128 views;
+                              an odd number of 128-view warps is padded by one warp of empty
+                              views (zero records).  Same arithmetic either way.  SV
                               bands of up to 61 rows (channels) per view are supported          */
     int zero_skip_period;  /* with zero_skip: iterations 1 + k*zero_skip_period, k >= 1 (numbers
                               counted from the last set_sinogram / set_image) run

@@ -705,10 +705,15 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     h->vpt = G.nviews > 128 ? MBIR_WIDE_VPT : 1;
     h->nvw = (G.nviews + 32 * h->vpt - 1) / (32 * h->vpt);
     if (h->nvw * h->vpt > 24) return (fail(h, MBIR_EINVAL, "nviews > 768 not supported"), bail(MBIR_EINVAL));
+    // an explicit 2-CTA cluster splits the view warps evenly: an odd count is padded by one warp
+    // whose views (>= nviews) carry zero records (no loads, no contribution)
+    if (h->vpt == MBIR_WIDE_VPT && (h->nvw & 1) && h->o.cluster == 2) h->nvw += 1;
+    size_t nA = 0;
+    for (int attempt = 0;; ++attempt) {
     h->Vs = (h->nvw * 32 * h->vpt + 127) / 128 * 128;  // record stride: whole 128-view tiles
     h->A.vpt = h->vpt;
     h->A.VA = h->Vs;  // thread-major record positions (apos); a multiple of 32 -> TMA-sized
-    const size_t nA = (size_t)h->nsv * h->S2 * h->A.VA;
+    nA = (size_t)h->nsv * h->S2 * h->A.VA;
     if (quant) {
         if ((r = dalloc(h, &h->A.codes, nA))) return bail(r);
         cudaMemsetAsync(h->A.codes, 0, nA * 4, h->st);
@@ -745,10 +750,27 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if (h->rows > kMaxSvbRows - 3)
         return (fail(h, MBIR_EINVAL, "SV band needs " + std::to_string(h->rows) + " > 61 buffer rows: reduce sv_side"), bail(MBIR_EINVAL));
     h->nwin = h->rows + 3 > 32 ? 2 : 1;
-    if (((size_t)G.nviews * G.nchannels) % 4 != 0)
-        return (fail(h, MBIR_EINVAL, "nviews * nchannels must be a multiple of 4"), bail(MBIR_EINVAL));
-    if ((size_t)G.nviews * G.nchannels >= (size_t(1) << 26))  // band row offsets are packed << 6
-        return (fail(h, MBIR_EINVAL, "nviews * nchannels must be < 2^26"), bail(MBIR_EINVAL));
+    // automatic cluster (below) for a buffer one CTA cannot hold, with an odd view-warp count:
+    // rebuild A once with the count padded to even
+    if (attempt == 0 && h->o.cluster == 0 && h->vpt == MBIR_WIDE_VPT && (h->nvw & 1)) {
+        IcdParams t = make_params(h);
+        t.A.VA = h->Vs;
+        if (svicd_smem_bytes(t, h->vpt, P.neighborhood, quant, 1) > (int)prop.sharedMemPerBlockOptin) {
+            void* ptrs[] = {h->A.codes, h->A.vals, h->A.off, h->A.count, h->A.scale, h->A.band_start, h->A.band_width};
+            for (void* q : ptrs)
+                if (q) cudaFree(q);
+            h->A.codes = nullptr;
+            h->A.vals = nullptr;
+            h->A.off = h->A.count = nullptr;
+            h->A.scale = nullptr;
+            h->A.band_start = nullptr;
+            h->A.band_width = nullptr;
+            h->nvw += 1;
+            continue;
+        }
+    }
+    break;
+    }
     h->a_bytes = (int64_t)nA * ((quant ? 4 : 16) + 2) + (int64_t)h->nsv * h->S2 * 4 + (int64_t)h->nsv * G.nviews * 5;
 
     {

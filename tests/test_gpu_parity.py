@@ -490,6 +490,36 @@ def test_large_sv_converged_matches_oracle(m720, side):
     assert abs(cg - co) <= 1e-4 * abs(co), (cg, co)
 
 
+def test_large_sv_odd_view_warps_padded_cluster_matches_oracle():
+    """360 views at the paper's pitch with side-13 SVs: the SV buffer (41 rows) exceeds one CTA and
+    the 3 view warps cannot be split evenly over a 2-CTA cluster, so the library pads a fourth,
+    empty view warp (views >= 360 carry zero records) and clusters.  Converged image and cost
+    match the oracle's MAP (1 HU / 1e-4); the padded run of side 9 (one CTA, odd warps) and an
+    explicit cluster = 2 with 360 views are accepted too."""
+    cfg = WorkloadConfig("mini360", 48, 2, 360, 96, 13, 26, 0.005)
+    case = make_case(cfg)
+    g, og = geoms(cfg)
+    _, _, Aq = O.quantize(O.sysmatrix(og))
+    pr = O.Prior(sigma=cfg.sigma, nbhd=26)
+    x = np.zeros(cfg.nz * cfg.n * cfg.n)
+    e = O.error_sinogram(og, Aq, case.y.astype(np.float64), x)
+    O.icd_run(og, pr, Aq, case.w, x, e, 80, seed=3000, zero_skip=False)
+    with M.Reconstructor(g, M.Prior(sigma=cfg.sigma, neighborhood=26), M.Options(sv_side=13)) as r:
+        s = r.sizes()
+        assert s["cluster"] == 2 and s["threads_per_cta"] == 32 * (2 + 2), s
+        r.set_sinogram(case.y, case.w)
+        r.reconstruct(200)
+        xg = r.image().ravel().astype(np.float64)
+    assert O.rmse_hu(xg, x) < 1.0
+    cg = O.cost(og, pr, Aq, case.y, case.w, xg)
+    co = O.cost(og, pr, Aq, case.y, case.w, x)
+    assert abs(cg - co) <= 1e-4 * abs(co), (cg, co)
+    with M.Reconstructor(g, M.Prior(neighborhood=26), M.Options(sv_side=9)) as r:
+        assert r.sizes()["cluster"] == 1 and r.sizes()["threads_per_cta"] == 32 * (3 + 2)
+    with M.Reconstructor(g, M.Prior(neighborhood=26), M.Options(sv_side=9, cluster=2)) as r:
+        assert r.sizes()["cluster"] == 2 and r.sizes()["threads_per_cta"] == 32 * (2 + 2)
+
+
 def test_voxels_per_step_option_validation():
     """mbir_options.voxels_per_step: 0 (auto) = 1, 1, or 2 (voxel pairs, uint8 A and one CTA per
     task only); anything else is EINVAL."""
