@@ -260,21 +260,20 @@ int exchange_halo(mbir_handle* h, int parity)
     return MBIR_OK;
 }
 
-// one fused-update-kernel launch bracketed by CUDA events on the handle's stream
-int timed_icd(mbir_handle* h, const IcdParams& p, int nnb, bool q, int gx, int gy)
+// CUDA event pair around a run of update-kernel launches on the handle's stream (the batches of
+// one phase: only batch-boundary gaps fall inside it; one pair per phase keeps the per-launch host
+// work low for many-batch 2-D iterations)
+int kev_mark(mbir_handle* h, bool begin)
 {
-    if ((int)h->kev.size() < 2 * (h->kev_used + 1)) {
+    if (begin && (int)h->kev.size() < 2 * (h->kev_used + 1)) {
         for (int i = 0; i < 2; ++i) {
             cudaEvent_t e;
             CK(cudaEventCreate(&e));
             h->kev.push_back(e);
         }
     }
-    CK(cudaEventRecord(h->kev[2 * h->kev_used], h->st));
-    (void)gy;
-    CK(launch_svicd(p, h->vpt, nnb, q, h->cl, gx, h->st));
-    CK(cudaEventRecord(h->kev[2 * h->kev_used + 1], h->st));
-    h->kev_used++;
+    CK(cudaEventRecord(h->kev[2 * h->kev_used + (begin ? 0 : 1)], h->st));
+    if (!begin) h->kev_used++;
     return MBIR_OK;
 }
 
@@ -397,12 +396,15 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
                     ++launches;
                     p.keep = h->d_keep;
                 }
+                if (int r = kev_mark(h, true)) return r;
                 for (int b = 0; b < nb; ++b) {
                     p.brange = h->d_brange + ph * (nb + 1) + b;
                     p.fetch = h->d_fetch + ph * nb + b;
-                    if (int r = timed_icd(h, p, nnb, q, grid, 1)) return r;
+                    CK(launch_svicd(p, h->vpt, nnb, q, h->cl, grid, h->st));
                     ++launches;
+                    ++klaunches;
                 }
+                if (int r = kev_mark(h, false)) return r;
             }
             if (h->nranks > 1 && parities == 2) {
                 // slices updated in this half have global parity zp
@@ -425,7 +427,6 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
             CK(cudaEventElapsedTime(&kms, h->kev[2 * i], h->kev[2 * i + 1]));
             ksec += kms * 1e-3;
         }
-        klaunches += h->kev_used;
         updates += (int64_t)h->h_counters[0];
         skipped += (int64_t)h->h_counters[1];
         visits += (int64_t)h->h_counters[2];

@@ -29,6 +29,9 @@
 // while the current one runs.
 #include "mbir_internal.h"
 
+#include <map>
+#include <mutex>
+
 namespace mbir {
 
 namespace {
@@ -1255,6 +1258,26 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     if (CL == 2) cluster_sync_all();  // no CTA leaves while its peer may still write into it
 }
 
+// the dynamic shared-memory opt-in and carveout of a kernel, set once per (device, kernel) for
+// the largest size seen (driver calls per launch would dominate short many-batch 2-D iterations)
+cudaError_t ensure_smem_attr(const void* kern, int smem)
+{
+    static std::mutex mu;
+    static std::map<std::pair<int, const void*>, int> done;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lk(mu);
+    int& have = done[{dev, kern}];
+    if (have >= smem) return cudaSuccess;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e != cudaSuccess) return e;
+    have = smem;
+    return cudaSuccess;
+}
+
 // A-record ring depth (voxels of cp.async lookahead): u8 records are 5 B/view, fp32 ones 17 B/view
 // (>= 2: the loop holds the current voxel's stage and the next voxel's)
 constexpr int ring_depth(bool u8) { return u8 ? 12 : 4; }
@@ -1280,9 +1303,7 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
     IcdParams q = p;
     q.lay = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, R, p.nvw, VPT, p.V, CL);
     const int smem = q.lay.total;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    cudaError_t e = ensure_smem_attr((const void*)kern, smem);
     if (e != cudaSuccess) return e;
     const int threads = 32 * (p.nvw / CL + 2);
     if (CL == 1) {
