@@ -121,6 +121,7 @@ struct mbir_handle {
     static constexpr int kNPerm = 64;
     int *d_task_list = nullptr, *d_task_count = nullptr;
     int *d_flat = nullptr, *d_brange = nullptr, *d_fetch = nullptr;
+    unsigned int* d_gbar = nullptr;  // [8 phases] grid-barrier counters of the update kernel
     int* d_keep = nullptr;  // zero-skip pre-filter flags of the current phase list
     unsigned long long* d_counters = nullptr;  // [updates, skipped, visits, empty visits]
     double* d_sum_delta = nullptr;
@@ -186,6 +187,8 @@ IcdParams make_params(mbir_handle* h)
     p.rows = h->rows;
     p.nwin = h->nwin;
     p.nvw = h->nvw;
+    p.nbatch = 1;
+    p.gbar = h->d_gbar;
     p.A = h->A;
     p.e = h->d_e;
     p.w = h->d_w;
@@ -361,6 +364,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
                           h->max_group, B, thr, nb, h->d_flat, h->d_brange, h->st));
         ++launches;
         CK(cudaMemsetAsync(h->d_fetch, 0, sizeof(int) * 8 * nb, h->st));
+        CK(cudaMemsetAsync(h->d_gbar, 0, sizeof(unsigned int) * 8, h->st));
         IcdParams p = make_params(h);
         // theta2 = sum w A^2 (Alg1:6) after new weights: reduced inside the update kernel during an
         // iteration that visits every voxel (the first one, unless a batch threshold drops tasks);
@@ -397,12 +401,24 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
                     p.keep = h->d_keep;
                 }
                 if (int r = kev_mark(h, true)) return r;
-                for (int b = 0; b < nb; ++b) {
-                    p.brange = h->d_brange + ph * (nb + 1) + b;
-                    p.fetch = h->d_fetch + ph * nb + b;
+                if (h->cl == 1) {
+                    // one cooperative launch runs the phase's batches with grid barriers between
+                    p.brange = h->d_brange + ph * (nb + 1);
+                    p.fetch = h->d_fetch + ph * nb;
+                    p.nbatch = nb;
+                    p.gbar = h->d_gbar + ph;
                     CK(launch_svicd(p, h->vpt, nnb, q, h->cl, grid, h->st));
                     ++launches;
                     ++klaunches;
+                } else {
+                    for (int b = 0; b < nb; ++b) {
+                        p.brange = h->d_brange + ph * (nb + 1) + b;
+                        p.fetch = h->d_fetch + ph * nb + b;
+                        p.nbatch = 1;
+                        CK(launch_svicd(p, h->vpt, nnb, q, h->cl, grid, h->st));
+                        ++launches;
+                        ++klaunches;
+                    }
                 }
                 if (int r = kev_mark(h, false)) return r;
             }
@@ -580,7 +596,7 @@ void mbir_destroy(mbir_handle* h)
     void* ptrs[] = {h->A.codes, h->A.vals, h->A.off, h->A.count, h->A.scale, h->A.band_start,
                     h->A.band_width, h->d_cs, h->d_y, h->d_w, h->d_e, h->d_x, h->d_theta2,
                     h->d_scratch, h->d_amount, h->d_task_list, h->d_task_count,
-                    h->d_flat, h->d_brange, h->d_fetch, h->d_keep, h->d_perm, h->d_counters, h->d_sum_delta,
+                    h->d_flat, h->d_brange, h->d_fetch, h->d_gbar, h->d_keep, h->d_perm, h->d_counters, h->d_sum_delta,
                     h->d_flag, h->d_acc, h->d_tprof, h->d_dump, h->d_dump_count};
     for (void* p : ptrs)
         if (p) cudaFree(p);
@@ -825,6 +841,7 @@ int mbir_create(const mbir_geometry* g, const mbir_prior* pr, const mbir_options
     if ((r = dalloc(h, &h->d_brange, (size_t)8 * (h->max_group + 1)))) return bail(r);
     if ((r = dalloc(h, &h->d_keep, (size_t)G.nz_local * h->max_group))) return bail(r);
     if ((r = dalloc(h, &h->d_fetch, (size_t)8 * h->max_group))) return bail(r);
+    if ((r = dalloc(h, &h->d_gbar, 8))) return bail(r);
     {
         // random voxel visiting orders within an SV ("randomized order"; reading R10):
         // kNPerm Fisher-Yates permutations from a seeded splitmix64, one picked per SV visit

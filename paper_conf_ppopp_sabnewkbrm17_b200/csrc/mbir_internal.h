@@ -86,8 +86,10 @@ struct IcdParams {
     const uint8_t* perm;     // [nperm][S2] random permutations of an SV's voxel slots
     int nperm;
     const int* flat;         // phase task list, entries (local slice << 14) | SV
-    const int* brange;       // [2]: this launch's batch = flat[brange[0] .. brange[1])
-    int* fetch;              // task counter of this launch (zeroed per iteration)
+    const int* brange;       // [nbatch + 1]: batch b = flat[brange[b] .. brange[b + 1])
+    int* fetch;              // [nbatch] task counters (zeroed per iteration)
+    int nbatch;              // batches run by this launch, a grid barrier between two (Alg3:24-27)
+    unsigned int* gbar;      // grid-barrier arrival counter of this launch (zeroed per iteration)
     const int* keep;         // optional [list]: 0 = the task's whole tile is zero (zero-skip pre-filter)
     unsigned long long* counters;  // [0] updates [1] skipped [2] sv visits
     double* sum_delta;

@@ -429,9 +429,10 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     // this launch's batch: flat tasks [start, end) of the phase list (sched.cu k_flatten), pulled
     // one at a time by the persistent CTAs (dynamic distribution, Alg3:4 / T3); with the zero-skip
     // pre-filter (P.keep), tasks whose whole tile is zero are accounted as skipped visits here
-    const int tstart = P.brange[0], tend = P.brange[1];
+    int tstart = P.brange[0], tend = P.brange[1];
+    int* fetchp = P.fetch;
     auto fetch_task = [&]() {
-        int q = tstart + atomicAdd(P.fetch, 1);
+        int q = tstart + atomicAdd(fetchp, 1);
         while (P.keep && q < tend && !P.keep[q]) {
             const int tkq = P.flat[q];
             const int zq = tkq >> 14, svq = tkq & 16383;
@@ -440,7 +441,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             atomicAdd(P.counters + 1, (unsigned long long)(twq * thq));
             atomicAdd(P.counters + 2, 1ull);
             atomicAdd(P.counters + 3, 1ull);
-            q = tstart + atomicAdd(P.fetch, 1);
+            q = tstart + atomicAdd(fetchp, 1);
         }
         return q;
     };
@@ -588,6 +589,13 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             if (is_delta) fetch_and_copy(b);  // fully skipped: the next task, synchronously
         }
     };
+    // the launch's batches (Alg3:24-27: each batch sees the previous one's write-backs): a grid
+    // barrier between two (the launch is cooperative when nbatch > 1, so every CTA is resident).
+    // Task inputs other than e are stable within a phase, so only e needs the barrier's ordering
+    for (int bt = 0; bt < P.nbatch; ++bt) {
+    tstart = P.brange[bt];
+    tend = P.brange[bt + 1];
+    fetchp = P.fetch + bt;
     int cb = 0;  // buffer of the current task (binfo, x tile, order, scales)
     if (is_delta) fetch_and_copy(0);
     if (!is_view) finish_prepare(0);
@@ -1255,6 +1263,23 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             atomicAdd(P.tprof + 5, 1ull);
         }
     }
+    if (bt + 1 < P.nbatch) {  // grid barrier (bar.sync, fence + arrival, acquire spin, bar.sync)
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            atomicAdd(P.gbar, 1u);
+            const unsigned target = (unsigned)(bt + 1) * gridDim.x;
+            for (;;) {
+                unsigned v;
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.gbar) : "memory");
+                if (v >= target) break;
+                __nanosleep(32);
+            }
+            __threadfence();
+        }
+        __syncthreads();
+    }
+    }
     if (CL == 2) cluster_sync_all();  // no CTA leaves while its peer may still write into it
 }
 
@@ -1306,7 +1331,7 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
     cudaError_t e = ensure_smem_attr((const void*)kern, smem);
     if (e != cudaSuccess) return e;
     const int threads = 32 * (p.nvw / CL + 2);
-    if (CL == 1) {
+    if (CL == 1 && p.nbatch <= 1) {
         kern<<<gx, threads, smem, st>>>(q);
         return cudaGetLastError();
     }
@@ -1315,6 +1340,14 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
     cfg.blockDim = dim3(threads);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = st;
+    if (CL == 1) {  // several batches with grid barriers: every CTA must be resident
+        cudaLaunchAttribute co[1];
+        co[0].id = cudaLaunchAttributeCooperative;
+        co[0].val.cooperative = 1;
+        cfg.attrs = co;
+        cfg.numAttrs = 1;
+        return cudaLaunchKernelEx(&cfg, kern, q);
+    }
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
     at[0].val.clusterDim.x = CL;
