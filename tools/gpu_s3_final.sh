@@ -1,7 +1,7 @@
 #!/bin/bash
 # Session-3 measurement set on one B200 (outputs under gpurun_out/s3z_*): the GPU test suite, the
-# default bench line (with the cfg4 oracle golden when goldens/golden_cfg4.npz is present, the
-# oracle cpu_baseline and the PSV-ICD leg), the cfg3 / cfg2 lines, the update kernel's ncu
+# default bench line (with the oracle cpu_baseline and the PSV-ICD leg; the cfg4 golden when
+# goldens/golden_cfg4.npz is present), the cfg3 / cfg2 lines, the update kernel's ncu
 # --set full capture, the bench's launch list and the update kernel's DRAM traffic per step.
 # Nothing here is a bench value except the bench*.json lines.
 set -x
@@ -14,4 +14,6 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"
 python tools/launch_summary.py gpurun_out/s3z_launches.csv > gpurun_out/s3z_launch_summary.txt 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_svicd -s 2 -c 1 -o gpurun_out/s3z_svicd python tools/iter_profile.py --iters 1 > gpurun_out/s3z_ncu_full.log 2>&1
 python tools/ncu_summary.py gpurun_out/s3z_svicd.ncu-rep 40 > gpurun_out/s3z_ncu_summary.txt 2>&1
+ncu -i gpurun_out/s3z_svicd.ncu-rep --page raw --csv > gpurun_out/s3z_svicd_raw.csv 2>/dev/null
+rm -f gpurun_out/s3z_svicd.ncu-rep  # (45 MB: gpurun copies back <= 64 MiB)
 timeout 900 bash tools/traffic.sh gpurun_out/s3z_traffic
