@@ -6,6 +6,16 @@
 # Nothing here is a bench value except the bench*.json lines.
 set -x
 nproc > gpurun_out/s3z_nproc.txt
+# same-box A/B: the in-tree kernel (in-kernel batches) against tools/alt/libmbir_ff.so (one launch
+# per batch), cfg4 and cfg3 per-iteration device time
+if [ -f tools/alt/libmbir_ff.so ]; then
+  for r in 1 2; do
+    for c in cfg4 cfg3; do
+      echo "== in-tree $c" >> gpurun_out/s3z_ab.log; timeout 200 python tools/iter_profile.py --config $c --iters 6 2>&1 | grep "^iter" >> gpurun_out/s3z_ab.log
+      echo "== ff $c" >> gpurun_out/s3z_ab.log; MBIR_LIB=tools/alt/libmbir_ff.so timeout 200 python tools/iter_profile.py --config $c --iters 6 2>&1 | grep "^iter" >> gpurun_out/s3z_ab.log
+    done
+  done
+fi
 timeout 1500 python -m pytest tests -q -m gpu -p no:cacheprovider -rf > gpurun_out/s3z_pytest_gpu.log 2>&1; echo "rc=$?" >> gpurun_out/s3z_pytest_gpu.log
 timeout 1500 python bench.py > gpurun_out/s3z_bench.json 2> gpurun_out/s3z_bench.err
 timeout 900 python bench.py --config cfg3 --no-cpu > gpurun_out/s3z_bench_cfg3.json 2> gpurun_out/s3z_bench_cfg3.err
