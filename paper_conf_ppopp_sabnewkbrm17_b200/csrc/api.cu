@@ -401,7 +401,7 @@ int run_iterations(mbir_handle* h, int n_iter, double target_equits, mbir_stats*
                     p.keep = h->d_keep;
                 }
                 if (int r = kev_mark(h, true)) return r;
-                if (h->cl == 1) {
+                if (h->cl == 1 && h->kv == 1 && nb > 1) {
                     // one cooperative launch runs the phase's batches with grid barriers between
                     p.brange = h->d_brange + ph * (nb + 1);
                     p.fetch = h->d_fetch + ph * nb;

@@ -355,7 +355,9 @@ __device__ __forceinline__ void load_words(const unsigned char* stg, int off_in_
 // ICD within the SV; 2: voxel pairs from the same state); PROF adds per-phase cycle counters.
 // T2: the theta2 pass -- theta2 = sum w A^2 (Alg1:6) is not precomputed yet: the view warps reduce
 // it with theta1 in this iteration (which visits every voxel) and the delta warp stores it
-template <int VPT, bool U8, int NNB, int R, int CL, int KV, bool T2, bool PROF>
+// MB: the launch runs P.nbatch batches with grid barriers between them (cooperative launch);
+// without it the batch loop compiles away (one batch per launch)
+template <int VPT, bool U8, int NNB, int R, int CL, int KV, bool T2, bool PROF, bool MB>
 __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P)
 {
     extern __shared__ __align__(16) unsigned char smem[];
@@ -592,10 +594,13 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
     // the launch's batches (Alg3:24-27: each batch sees the previous one's write-backs): a grid
     // barrier between two (the launch is cooperative when nbatch > 1, so every CTA is resident).
     // Task inputs other than e are stable within a phase, so only e needs the barrier's ordering
-    for (int bt = 0; bt < P.nbatch; ++bt) {
-    tstart = P.brange[bt];
-    tend = P.brange[bt + 1];
-    fetchp = P.fetch + bt;
+    const int nbatch = MB ? P.nbatch : 1;
+    for (int bt = 0; bt < nbatch; ++bt) {
+    if (MB) {
+        tstart = P.brange[bt];
+        tend = P.brange[bt + 1];
+        fetchp = P.fetch + bt;
+    }
     int cb = 0;  // buffer of the current task (binfo, x tile, order, scales)
     if (is_delta) fetch_and_copy(0);
     if (!is_view) finish_prepare(0);
@@ -1263,7 +1268,7 @@ __global__ void __launch_bounds__(max_threads(VPT), 1) k_svicd(const IcdParams P
             atomicAdd(P.tprof + 5, 1ull);
         }
     }
-    if (bt + 1 < P.nbatch) {  // grid barrier (bar.sync, fence + arrival, acquire spin, bar.sync)
+    if (MB && bt + 1 < nbatch) {  // grid barrier (bar.sync, fence + arrival, acquire spin, bar.sync)
         __syncthreads();
         if (threadIdx.x == 0) {
             __threadfence();
@@ -1312,9 +1317,15 @@ auto pick_kernel(const IcdParams& p)
 {
     // the phase profile (development aid) is built for the production variants only
     constexpr bool kProf = VPT == MBIR_WIDE_VPT && U8 && CL == 1;
-    return p.theta2_pass ? k_svicd<VPT, U8, NNB, R, CL, KV, true, false>
-           : (kProf && p.tprof) ? k_svicd<VPT, U8, NNB, R, CL, KV, false, kProf>
-                                : k_svicd<VPT, U8, NNB, R, CL, KV, false, false>;
+    // several batches per launch: one CTA per task, exact single-voxel steps (api.cu launches the
+    // other variants once per batch)
+    constexpr bool kMB = CL == 1 && KV == 1;
+    if (kMB && p.nbatch > 1)
+        return p.theta2_pass ? k_svicd<VPT, U8, NNB, R, CL, KV, true, false, kMB>
+                             : k_svicd<VPT, U8, NNB, R, CL, KV, false, false, kMB>;
+    return p.theta2_pass ? k_svicd<VPT, U8, NNB, R, CL, KV, true, false, false>
+           : (kProf && p.tprof) ? k_svicd<VPT, U8, NNB, R, CL, KV, false, kProf, false>
+                                : k_svicd<VPT, U8, NNB, R, CL, KV, false, false, false>;
 }
 
 template <int VPT, bool U8, int NNB, int CL>
@@ -1361,7 +1372,7 @@ cudaError_t launch_t(const IcdParams& p, int gx, cudaStream_t st)
 template <int VPT, bool U8, int NNB, int CL>
 int resident_t(const IcdParams& p)
 {
-    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), CL, 1, false, false>;
+    auto kern = k_svicd<VPT, U8, NNB, ring_depth(U8), CL, 1, false, false, false>;
     const int smem = svicd_layout(p.rows, p.side, p.S2, NNB, p.A.VA, U8, ring_depth(U8), p.nvw, VPT, p.V, CL).total;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return -1;
     cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
