@@ -997,12 +997,10 @@ int mbir_init_fbp(mbir_handle* h)
 {
     if (!h) return MBIR_EINVAL;
     if (!h->have_sino) return fail(h, MBIR_ESTATE, "mbir_set_sinogram has not been called");
-    const size_t pl = plane_elems(h), ns = sino_elems(h);
-    float* q = nullptr;
-    if (cudaMallocAsync((void**)&q, ns * sizeof(float), h->st) != cudaSuccess)
-        return fail(h, MBIR_ENOMEM, "cudaMallocAsync (FBP filtered sinogram)");
-    cudaError_t e = launch_fbp(h->g, h->d_cs, h->d_y, q, h->d_x + pl, h->pr.positivity, h->st);
-    cudaFreeAsync(q, h->st);
+    const size_t pl = plane_elems(h);
+    // the filtered sinogram lives in e, which is recomputed (e = y - A x) right after: no
+    // allocation per call (a stream-ordered malloc/free of the sinogram size cost up to 50 ms)
+    cudaError_t e = launch_fbp(h->g, h->d_cs, h->d_y, h->d_e, h->d_x + pl, h->pr.positivity, h->st);
     if (e != cudaSuccess) return fail(h, MBIR_ECUDA, std::string("FBP: ") + cudaGetErrorString(e));
     h->x_zero = false;
     int r = exchange_halo(h, -1);
