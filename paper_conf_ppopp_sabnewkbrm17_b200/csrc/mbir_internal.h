@@ -125,7 +125,7 @@ struct SchedParams {
 cudaError_t build_sysmatrix(const mbir_geometry& g, const double* d_angles_cs, int side, int nsvx,
                             int nsvy, bool quantize, DevA& A, int* d_err, int* d_maxoff,
                             cudaStream_t st);
-// the fused update kernel (svicd.cu): per CTA nvw / cl view warps + the delta warp + the prior
+// the fused update kernel (svicd_impl.cuh, instantiated in svicd_n*_*.cu): per CTA nvw / cl view warps + the delta warp + the prior
 // warp, vpt = 4 (or 1 for <= 128 views) views per lane; cl = 2: a 2-CTA cluster splits a task's views
 int svicd_smem_bytes(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
 int svicd_resident_ctas(const IcdParams& p, int vpt, int nnb, bool quantize, int cl);
